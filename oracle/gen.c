@@ -1,0 +1,146 @@
+/*
+ * gen.c -- the seeded input generator (oracle side).  TEST INFRASTRUCTURE.
+ *
+ * This module holds none of the method's arithmetic: it only turns
+ * (seed, thread t, transaction index i) into the addresses and constants a
+ * transaction uses (the "input recipe").  The CUDA side
+ * implements the same recipe independently (no shared code or header); the
+ * GPU-vs-oracle descriptor parity test checks that both agree bit for bit.
+ *
+ * Generator: SplitMix64 (Steele, Lea, Flood, "Fast splittable pseudorandom
+ * number generators", OOPSLA 2014; Vigna's public-domain splitmix64.c).
+ * Pinned in tests/test_oracle_gen.py against the published output vectors
+ * (tests/golden/splitmix64_vectors.txt).
+ *
+ * The paper does not define its workloads' values (Table 1
+ * lost at P:260); the recipes below are our readings (SURVEY
+ * §8c-O2 / Q23), each chosen so that a lost update is observable.
+ */
+#include "oracle.h"
+
+#define GOLDEN 0x9E3779B97F4A7C15ull  /* SplitMix64 increment (gamma)     */
+#define TXMUL  0xC2B2AE3D27D4EB4Full  /* odd multiplier separating i      */
+
+/* SplitMix64 output function ("mix64" / Stafford variant 13). */
+uint64_t or_mix64(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+/* First output of a SplitMix64 stream whose state is x. */
+uint64_t or_splitmix64(uint64_t x) { return or_mix64(x + GOLDEN); }
+
+/* k-th draw of the stream keyed by x: the (k+1)-th SplitMix64 output from
+ * state x (draw(x,0), draw(x,1), ... are exactly the stream's outputs). */
+uint64_t or_draw(uint64_t x, uint64_t k) { return or_splitmix64(x + k * GOLDEN); }
+
+/* Uniform integer in [0, n): Lemire's multiply-shift, floor(r * n / 2^64). */
+uint64_t or_bounded(uint64_t r, uint64_t n)
+{
+    return (uint64_t)(((unsigned __int128)r * (unsigned __int128)n) >> 64);
+}
+
+/* Per-transaction stream key.  A re-executed (aborted) transaction derives
+ * the same key, so it regenerates the identical transaction. */
+uint64_t or_txkey(uint64_t seed, uint64_t t, uint64_t i)
+{
+    return or_splitmix64(seed ^ (t * GOLDEN) ^ (i * TXMUL));
+}
+
+static uint32_t lo32(uint64_t v) { return (uint32_t)(v & 0xffffffffull); }
+
+/* Descriptor layouts:
+ *   RA kind 0 : r_0..r_{R-1}, w_0..w_{W-1}, c_0..c_{W-1}   (R + 2W words)
+ *               r_j = bounded(draw(j), N); w_j = bounded(draw(R+j), N);
+ *               c_j = lo32(draw(R+W+j))
+ *   RA kind 1 : r_0..r_{R-1}                                (R words)
+ *   BANK      : a, b, amt     a = bounded(draw0, N); b = bounded(draw1, N-1),
+ *               b += (b >= a); amt = 1 + bounded(draw2, 100)
+ *   HT        : key, is_insert, bucket
+ *               key = 1 + bounded(draw0, KR); is_insert = bounded(draw1,100)
+ *               >= lookup_pct; bucket = mix64(key) & (B-1)
+ *   EB        : x_0..x_{A-1}, c_0..c_{A-1}   x_j = bounded(draw(j), H);
+ *               c_j = lo32(draw(A+j))
+ *   KM        : c, f_0..f_{D-1}   c = bounded(draw0, C); f_d = draw(1+d) >> 56
+ */
+int or_descr(const or_params_t* p, uint64_t seed, uint64_t t, uint64_t i,
+             uint32_t* out, int cap)
+{
+    uint64_t x = or_txkey(seed, t, i);
+    switch (p->workload) {
+    case OR_WL_RA: {
+        uint32_t R = p->n_reads, W = p->n_writes;
+        uint64_t N = p->n_words;
+        if (N == 0) return -1;
+        if (p->ra_kind == 1) {
+            if ((int)R > cap) return -1;
+            for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)or_bounded(or_draw(x, j), N);
+            return (int)R;
+        }
+        if ((int)(R + 2 * W) > cap) return -1;
+        for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)or_bounded(or_draw(x, j), N);
+        for (uint32_t j = 0; j < W; ++j) out[R + j] = (uint32_t)or_bounded(or_draw(x, R + j), N);
+        for (uint32_t j = 0; j < W; ++j) out[R + W + j] = lo32(or_draw(x, R + W + j));
+        return (int)(R + 2 * W);
+    }
+    case OR_WL_BANK: {
+        uint64_t N = p->n_words;
+        if (N < 2 || cap < 3) return -1;
+        uint64_t a = or_bounded(or_draw(x, 0), N);
+        uint64_t b = or_bounded(or_draw(x, 1), N - 1);
+        if (b >= a) b += 1;
+        out[0] = (uint32_t)a; out[1] = (uint32_t)b;
+        out[2] = 1u + (uint32_t)or_bounded(or_draw(x, 2), 100);
+        return 3;
+    }
+    case OR_WL_HT: {
+        if (cap < 3 || p->ht_buckets == 0 || (p->ht_buckets & (p->ht_buckets - 1))) return -1;
+        uint64_t key = 1 + or_bounded(or_draw(x, 0), p->ht_key_range);
+        out[0] = (uint32_t)key;
+        out[1] = or_bounded(or_draw(x, 1), 100) >= p->ht_lookup_pct ? 1u : 0u;
+        out[2] = (uint32_t)(or_mix64(key) & (uint64_t)(p->ht_buckets - 1));
+        return 3;
+    }
+    case OR_WL_EB: {
+        uint32_t A = p->n_accesses;
+        uint64_t H = p->n_words;
+        if (H == 0 || (int)(2 * A) > cap) return -1;
+        for (uint32_t j = 0; j < A; ++j) out[j] = (uint32_t)or_bounded(or_draw(x, j), H);
+        for (uint32_t j = 0; j < A; ++j) out[A + j] = lo32(or_draw(x, A + j));
+        return (int)(2 * A);
+    }
+    case OR_WL_KM: {
+        uint32_t C = p->km_clusters, D = p->km_dims;
+        if (C == 0 || (int)(1 + D) > cap) return -1;
+        out[0] = (uint32_t)or_bounded(or_draw(x, 0), C);
+        for (uint32_t d = 0; d < D; ++d) out[1 + d] = (uint32_t)(or_draw(x, 1 + d) >> 56);
+        return (int)(1 + D);
+    }
+    }
+    return -1;
+}
+
+uint64_t or_footprint(const or_params_t* p, uint64_t T, uint64_t K)
+{
+    switch (p->workload) {
+    case OR_WL_RA: case OR_WL_BANK: case OR_WL_EB: return p->n_words;
+    case OR_WL_HT: return (uint64_t)p->ht_buckets + 2ull * T * K;
+    case OR_WL_KM: return (uint64_t)p->km_clusters * (p->km_dims + 1ull);
+    }
+    return 0;
+}
+
+/* Initial heaps: RA and EB heap[k] = k; bank 1000 per
+ * account; HT empty (all heads null, node words 0); KM all records zero. */
+void or_init_heap(const or_params_t* p, uint32_t* heap, uint64_t words)
+{
+    for (uint64_t k = 0; k < words; ++k) {
+        switch (p->workload) {
+        case OR_WL_RA: case OR_WL_EB: heap[k] = (uint32_t)k; break;
+        case OR_WL_BANK: heap[k] = 1000u; break;
+        default: heap[k] = 0u; break;
+        }
+    }
+}
