@@ -1,0 +1,200 @@
+/*
+ * gstm.h -- C ABI of the B200-native GPU-STM hot path.
+ *
+ * Implements the per-thread transactional memory of Xu et al., "Software
+ * Transactional Memory for GPU Architectures", CGO 2014 (the paper text is
+ * cited as P:<line>; Algorithm 3 lines as A3.l<k>).  The host side mirrors the
+ * paper's usage (Figure 1): STM_STARTUP / STM_SHUTDOWN allocate and
+ * free the global metadata (gstm_create / gstm_destroy), a transactional
+ * kernel runs every thread's transactions (gstm_launch), and the statistics
+ * are read back (gstm_stats).
+ *
+ * Conventions (all functions):
+ *   - extern "C", plain pointers and integers; no C++ types, no exceptions.
+ *   - Functions returning int return GSTM_OK (0) or a negative gstm_status;
+ *     the message for the last failure on the calling thread is in
+ *     gstm_last_error().  The library never calls exit() or abort().
+ *   - "device pointer" = CUDA global memory of the current device;
+ *     "host pointer" = ordinary (optionally pinned) CPU memory.
+ *   - Work is enqueued on the handle's stream (gstm_set_stream; default: a
+ *     private non-blocking stream).  gstm_launch is asynchronous; gstm_stats
+ *     and every gstm_read_* call synchronise that stream.
+ *   - A handle is not thread-safe; use one handle per host thread.
+ *   - Heap words are uint32.  Word w is protected by version lock
+ *     w mod 2^lock_table_bits (reading Q2 in DESIGN.md §4).
+ */
+#ifndef GSTM_H
+#define GSTM_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GSTM_API_VERSION 1
+
+typedef struct gstm_handle gstm_t;   /* opaque; owns the lock table, clock, stats, logs, heap */
+
+enum gstm_status {
+    GSTM_OK = 0,
+    GSTM_EINVAL = -1,     /* bad argument or workload parameters                  */
+    GSTM_ENOMEM = -2,     /* device allocation failed                             */
+    GSTM_ECUDA = -3,      /* CUDA runtime error (message in gstm_last_error)      */
+    GSTM_ELOGOVF = -4,    /* a transaction needed more log entries than compiled  */
+    GSTM_EOVERFLOW = -5,  /* stamp space: n_threads * tx_per_thread >= 2^31       */
+    GSTM_ETIMEOUT = -6,   /* the device watchdog stopped the launch               */
+    GSTM_EBUSY = -7,      /* no launch to report on                               */
+    GSTM_ENODEV = -8      /* no CUDA device                                       */
+};
+
+/* Workloads.  RA = random array (Figure 1);
+ * BANK = two-account transfer; HT = chained hash table, set semantics;
+ * EB = EigenBench-style alternating read/write; KM = k-means
+ * cluster-update transaction (STAMP kmeans). */
+enum gstm_workload { GSTM_WL_RA = 0, GSTM_WL_BANK = 1, GSTM_WL_HT = 2, GSTM_WL_EB = 3, GSTM_WL_KM = 4 };
+
+/* Concurrency control:
+ *   AUTO = STM-Optimized: HV when the workload's shared words exceed the
+ *          number of version locks, else TBV;
+ *   HV   = STM-HV-Sorting (hierarchical validation);
+ *   TBV  = STM-TBV-Sorting (timestamp validation only);
+ *   CGL  = coarse-grain lock baseline, Scheme #3 of Algorithm 1;
+ *   FGL  = fine-grain lock baseline (sorted per-stripe locks; P:288 notes the
+ *          paper did not implement it). */
+enum gstm_mode { GSTM_MODE_AUTO = 0, GSTM_MODE_HV = 1, GSTM_MODE_TBV = 2, GSTM_MODE_CGL = 3, GSTM_MODE_FGL = 4 };
+
+typedef struct {
+    /* workload shape (which fields apply: DESIGN.md §3.3) */
+    uint32_t n_reads;        /* RA: reads per tx (kind 0: <= 8; kind 1: <= 16)          */
+    uint32_t n_writes;       /* RA kind 0: writes per tx (<= 8)                          */
+    uint32_t ra_kind;        /* RA: 0 reads-then-writes, 1 increment each word read     */
+    uint64_t n_words;        /* RA/BANK/EB: words addressed, [0, n_words) (EB: hot set) */
+    uint32_t n_accesses;     /* EB: accesses per tx, alternating r/w (<= 64)            */
+    uint32_t ht_buckets;     /* HT: bucket heads (power of two)                         */
+    uint32_t ht_lookup_pct;  /* HT: percentage of lookups (rest inserts)                */
+    uint64_t ht_key_range;   /* HT: keys uniform in [1, ht_key_range]                   */
+    uint32_t km_clusters;    /* KM: cluster records                                     */
+    uint32_t km_dims;        /* KM: features per point (<= 16)                          */
+    /* runtime knobs */
+    uint32_t prelock_vbv;    /* HV: value-validate before locking (A3.l71), default 1   */
+    uint32_t k_lock;         /* lock-acquisition rounds before abort; 0 = inf   */
+    uint32_t backoff_ns;     /* warp-uniform backoff after an abort; 0 = none           */
+    uint32_t verify;         /* record per-tx stamp and result (gstm_read_tx_log)       */
+    uint32_t block_threads;  /* CUDA block size (multiple of 32, <= 256), default 256   */
+    uint32_t spin_cap;       /* bound on lock spins / PostValidation restarts          */
+    uint32_t timeout_ms;     /* device watchdog per launch, default 60000               */
+} gstm_params_t;
+
+typedef struct {
+    uint64_t commits;            /* committed update transactions (stamped, A3.l83)     */
+    uint64_t commits_ro;         /* committed read-only transactions (A3.l68)           */
+    uint64_t aborts;             /* sum of the abort causes below                       */
+    uint64_t aborts_opacity;     /* isOpaque became false during execution (A3.l33)     */
+    uint64_t aborts_prevbv;      /* pre-lock VBV failed (A3.l71-72)                     */
+    uint64_t aborts_tbv;         /* TBV mode: version newer than snapshot at commit     */
+    uint64_t aborts_commit_vbv;  /* VBV under locks failed (A3.l76-78)                  */
+    uint64_t aborts_lock;        /* k_lock acquisition rounds exhausted         */
+    uint64_t lock_retries;       /* failed lock-acquisition rounds (A3.l73-74)          */
+    uint64_t postvalidations;    /* PostValidation calls (A3.l32)                       */
+    uint64_t vbv_runs;           /* VBV passes (pre-lock, under locks, post-validation) */
+    uint64_t spins;              /* lock-word re-reads while locked (A3.l27-29)         */
+    uint64_t attempts;           /* transaction executions (commits + aborts)           */
+    uint64_t errors;             /* transactions dropped on log overflow                */
+    uint64_t clock_begin;        /* g_clock at launch start                             */
+    uint64_t clock_end;          /* g_clock at launch end                               */
+    double elapsed_ms;           /* device time of the launch (CUDA events)             */
+    double tx_per_s;             /* (commits + commits_ro) / elapsed                    */
+    double abort_ratio;          /* aborts / (aborts + commits + commits_ro)            */
+    int32_t status;              /* GSTM_OK, GSTM_ELOGOVF, GSTM_ETIMEOUT                */
+    int32_t mode_used;           /* gstm_mode actually run (AUTO resolved)              */
+} gstm_stats_t;
+
+/* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */
+/* Allocates a heap of heap_words uint32 (zeroed), a table of
+ * 2^lock_table_bits version locks (0 <= bits <= 30, zeroed), the global clock
+ * (0) and statistics.  Returns NULL on error (gstm_last_error). */
+gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits);
+/* Frees everything the handle owns (not an attached heap).  NULL is a no-op. */
+void gstm_destroy(gstm_t* h);
+/* Message of the last failure on this thread ("" if none).  Static storage. */
+const char* gstm_last_error(void);
+int gstm_api_version(void);
+
+/* ---- configuration ----------------------------------------------------- */
+/* Fills *out with the defaults for a workload (BASELINE-shaped sizes). */
+int gstm_default_params(int workload, gstm_params_t* out);
+int gstm_set_params(gstm_t* h, const gstm_params_t* p);
+int gstm_get_params(const gstm_t* h, gstm_params_t* out);
+int gstm_set_mode(gstm_t* h, int mode);
+/* stream: a cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream);
+ * NULL restores the handle's private stream.  Borrowed, not destroyed. */
+int gstm_set_stream(gstm_t* h, void* stream);
+/* Use caller-owned device memory (>= words uint32, 4-byte aligned) as the
+ * heap instead of the handle's own; borrowed: it must outlive the handle or
+ * the next attach.  words == 0 or dev_ptr == NULL re-selects the own heap. */
+int gstm_attach_heap(gstm_t* h, void* dev_ptr, uint64_t words);
+uint64_t gstm_heap_words(const gstm_t* h);
+/* device pointer of the current heap (for zero-copy views) */
+void* gstm_heap_ptr(const gstm_t* h);
+
+/* ---- data --------------------------------------------------------------- */
+/* Device-side initial heap of a workload. */
+int gstm_init_heap(gstm_t* h, int workload);
+int gstm_write_heap(gstm_t* h, const uint32_t* host_src, uint64_t offset, uint64_t words);
+int gstm_read_heap(gstm_t* h, uint32_t* host_dst, uint64_t offset, uint64_t words);
+/* Version-lock table (2^bits uint32: LSB locked, bits 31..1 version). */
+int gstm_read_locks(gstm_t* h, uint32_t* host_dst, uint64_t n);
+int gstm_read_clock(gstm_t* h, uint64_t* out);
+/* Zero the lock table and the clock (a new version epoch). */
+int gstm_reset_meta(gstm_t* h);
+/* Set the global clock (e.g. to start a scripted test at a given time);
+ * value < 2^31 and >= every version in the lock table. */
+int gstm_set_clock(gstm_t* h, uint64_t value);
+
+/* ---- the hot path -------------------------------------------------------- */
+/* Run n_threads STM threads, each executing tx_per_thread transactions of the
+ * workload (tx_id = i*n_threads + t, generated from seed), under the
+ * handle's mode, on the current heap.  Every transaction commits exactly once
+ * (aborted attempts re-execute) unless the launch reports an error.  Stamps
+ * of this launch are g_clock_begin+1 .. g_clock_end.  Asynchronous. */
+int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed);
+/* Synchronises, then reports the last launch.  Returns the launch status. */
+int gstm_stats(gstm_t* h, gstm_stats_t* out);
+/* Verify mode (params.verify = 1): stamps[tx_id] = commit stamp - clock_begin
+ * (1..C) for an update tx, or 0x80000000 | (snapshot - clock_begin) for a
+ * read-only tx (linearised after that stamp); results[tx_id] = the
+ * workload's observable result.  n = n_threads * tx_per_thread. */
+int gstm_read_tx_log(gstm_t* h, uint32_t* stamps, uint32_t* results, uint64_t n);
+/* End-to-end call with HOST buffers: copy heap_in (words) to the heap, launch,
+ * copy the heap back to heap_out, synchronise and fill *stats (may be NULL).
+ * heap_in/heap_out may alias; pinned memory gives full copy bandwidth. */
+int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
+                  uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed, gstm_stats_t* stats);
+
+/* ---- test and measurement entry points --------------------------------- */
+/* Transaction descriptors as generated on the device:
+ * host_out[(i*n_threads + t) * words_per_tx + k]; short descriptors are
+ * zero-padded.  words_per_tx >= gstm_descr_words(h, workload). */
+int gstm_descr_words(gstm_t* h, int workload);
+int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed,
+                    uint32_t* host_out, uint32_t words_per_tx);
+/* Scripted interleaving of up to 8 transactions on one device thread, on the
+ * handle's heap, lock table and clock.  ops: n_ops x {op, slot, word, value}
+ * with op 0 BEGIN, 1 READ, 2 WRITE, 3 COMMIT; out: n_ops x 4 words (format in
+ * DESIGN.md §5.3).  mode: GSTM_MODE_HV or GSTM_MODE_TBV. */
+int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx);
+/* Insert entries (id<<2 | wr<<1 | rd) into a device lock log (variant 0:
+ * register-resident, capacity 16; 1: local memory, capacity 256) and return
+ * the resulting log in out; returns its length or a negative error. */
+int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant);
+/* Roofline microbenchmark: kind 0 random atom.or, 1
+ * same-address atom.add.u64, 2 random ld.relaxed, 3 random st.relaxed, 4
+ * dependent atom.or chain, 5 warp-aggregated clock increments; over a table
+ * of table_bytes (power of two) with `threads` threads (multiple of 256).
+ * *ops_per_s = operations per second; *ms = kernel time. */
+int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,506 @@
+// api.cu -- the C ABI (include/gstm.h) over the kernels in kernels.cu.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <cuda_runtime.h>
+#include "../../include/gstm.h"
+#include "kernels.cuh"
+
+using namespace gstm;
+
+static thread_local char g_err[512] = "";
+
+static void set_error(const char* fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+#define CUDA_TRY(expr)                                                                    \
+    do {                                                                                  \
+        cudaError_t e__ = (expr);                                                         \
+        if (e__ != cudaSuccess) {                                                         \
+            set_error("%s: %s (%s:%d)", #expr, cudaGetErrorString(e__), __FILE__, __LINE__); \
+            return GSTM_ECUDA;                                                            \
+        }                                                                                 \
+    } while (0)
+
+struct gstm_handle {
+    uint32_t* own_heap = nullptr;
+    uint32_t* heap = nullptr;
+    uint64_t heap_words = 0, own_words = 0;
+    uint32_t* locks = nullptr;
+    uint32_t bits = 0;
+    unsigned long long* meta = nullptr;
+    uint32_t* tx_stamp = nullptr;
+    uint32_t* tx_result = nullptr;
+    uint64_t log_cap = 0;
+    cudaStream_t own_stream = nullptr, stream = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    gstm_params_t params{};
+    int mode = GSTM_MODE_AUTO;
+    // last launch
+    bool launched = false;
+    int last_mode = 0;
+    uint64_t last_n = 0;
+    uint64_t clock_bound = 0;    // upper bound of g_clock (host-tracked)
+};
+
+static gstm_params_t default_params(int workload)
+{
+    gstm_params_t p;
+    memset(&p, 0, sizeof(p));
+    p.n_reads = 4;
+    p.n_writes = 4;
+    p.ra_kind = 0;
+    p.n_words = 1024;
+    p.n_accesses = 16;
+    p.ht_buckets = 1u << 20;
+    p.ht_lookup_pct = 90;
+    p.ht_key_range = 1ull << 22;
+    p.km_clusters = 1024;
+    p.km_dims = 16;
+    p.prelock_vbv = 1;
+    p.k_lock = 8;
+    p.backoff_ns = 0;
+    p.verify = 0;
+    p.block_threads = 256;
+    p.spin_cap = 1u << 16;
+    p.timeout_ms = 60000;
+    if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
+    if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
+    return p;
+}
+
+static WlParams wl_params(const gstm_params_t& p, uint64_t T, uint64_t K)
+{
+    WlParams w;
+    w.n_words = p.n_words;
+    w.n_reads = p.n_reads;
+    w.n_writes = p.n_writes;
+    w.ra_kind = p.ra_kind;
+    w.n_accesses = p.n_accesses;
+    w.ht_buckets = p.ht_buckets;
+    w.ht_lookup_pct = p.ht_lookup_pct;
+    w.ht_key_range = p.ht_key_range;
+    w.km_clusters = p.km_clusters;
+    w.km_dims = p.km_dims;
+    w.T = T;
+    w.K = K;
+    return w;
+}
+
+extern "C" {
+
+const char* gstm_last_error(void) { return g_err; }
+int gstm_api_version(void) { return GSTM_API_VERSION; }
+
+int gstm_default_params(int workload, gstm_params_t* out)
+{
+    if (!out || workload < 0 || workload > 4) { set_error("gstm_default_params: bad argument"); return GSTM_EINVAL; }
+    *out = default_params(workload);
+    return GSTM_OK;
+}
+
+gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits)
+{
+    g_err[0] = 0;
+    if (lock_table_bits > 30) { set_error("gstm_create: lock_table_bits %u > 30", lock_table_bits); return nullptr; }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) { set_error("gstm_create: no CUDA device"); return nullptr; }
+    gstm_t* h = new gstm_t();
+    h->bits = lock_table_bits;
+    h->params = default_params(GSTM_WL_RA);
+    const size_t lock_bytes = sizeof(uint32_t) << lock_table_bits;
+    if (heap_words && cudaMalloc(&h->own_heap, heap_words * 4) != cudaSuccess) goto oom;
+    if (cudaMalloc(&h->locks, lock_bytes) != cudaSuccess) goto oom;
+    if (cudaMalloc(&h->meta, M_WORDS * 8) != cudaSuccess) goto oom;
+    if (cudaStreamCreateWithFlags(&h->own_stream, cudaStreamNonBlocking) != cudaSuccess) goto cuerr;
+    if (cudaEventCreate(&h->ev0) != cudaSuccess || cudaEventCreate(&h->ev1) != cudaSuccess) goto cuerr;
+    h->stream = h->own_stream;
+    h->heap = h->own_heap;
+    h->heap_words = h->own_words = heap_words;
+    if (heap_words && cudaMemsetAsync(h->own_heap, 0, heap_words * 4, h->stream) != cudaSuccess) goto cuerr;
+    if (cudaMemsetAsync(h->locks, 0, lock_bytes, h->stream) != cudaSuccess) goto cuerr;
+    if (cudaMemsetAsync(h->meta, 0, M_WORDS * 8, h->stream) != cudaSuccess) goto cuerr;
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) goto cuerr;
+    return h;
+oom:
+    set_error("gstm_create: out of device memory (heap %llu words, 2^%u locks)", (unsigned long long)heap_words,
+              lock_table_bits);
+    gstm_destroy(h);
+    return nullptr;
+cuerr:
+    set_error("gstm_create: %s", cudaGetErrorString(cudaGetLastError()));
+    gstm_destroy(h);
+    return nullptr;
+}
+
+void gstm_destroy(gstm_t* h)
+{
+    if (!h) return;
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    cudaFree(h->own_heap);
+    cudaFree(h->locks);
+    cudaFree(h->meta);
+    cudaFree(h->tx_stamp);
+    cudaFree(h->tx_result);
+    if (h->ev0) cudaEventDestroy(h->ev0);
+    if (h->ev1) cudaEventDestroy(h->ev1);
+    if (h->own_stream) cudaStreamDestroy(h->own_stream);
+    delete h;
+}
+
+int gstm_set_params(gstm_t* h, const gstm_params_t* p)
+{
+    if (!h || !p) { set_error("gstm_set_params: NULL"); return GSTM_EINVAL; }
+    if (p->block_threads == 0 || p->block_threads > 256 || p->block_threads % 32) {
+        set_error("gstm_set_params: block_threads must be a multiple of 32 in [32, 256]");
+        return GSTM_EINVAL;
+    }
+    h->params = *p;
+    return GSTM_OK;
+}
+
+int gstm_get_params(const gstm_t* h, gstm_params_t* out)
+{
+    if (!h || !out) { set_error("gstm_get_params: NULL"); return GSTM_EINVAL; }
+    *out = h->params;
+    return GSTM_OK;
+}
+
+int gstm_set_mode(gstm_t* h, int mode)
+{
+    if (!h || mode < GSTM_MODE_AUTO || mode > GSTM_MODE_FGL) { set_error("gstm_set_mode: bad mode %d", mode); return GSTM_EINVAL; }
+    h->mode = mode;
+    return GSTM_OK;
+}
+
+int gstm_set_stream(gstm_t* h, void* stream)
+{
+    if (!h) { set_error("gstm_set_stream: NULL"); return GSTM_EINVAL; }
+    h->stream = stream ? static_cast<cudaStream_t>(stream) : h->own_stream;
+    return GSTM_OK;
+}
+
+int gstm_attach_heap(gstm_t* h, void* dev_ptr, uint64_t words)
+{
+    if (!h) { set_error("gstm_attach_heap: NULL"); return GSTM_EINVAL; }
+    if (!dev_ptr || !words) {
+        h->heap = h->own_heap;
+        h->heap_words = h->own_words;
+        return GSTM_OK;
+    }
+    if (reinterpret_cast<uintptr_t>(dev_ptr) & 3) { set_error("gstm_attach_heap: unaligned pointer"); return GSTM_EINVAL; }
+    h->heap = static_cast<uint32_t*>(dev_ptr);
+    h->heap_words = words;
+    return GSTM_OK;
+}
+
+uint64_t gstm_heap_words(const gstm_t* h) { return h ? h->heap_words : 0; }
+void* gstm_heap_ptr(const gstm_t* h) { return h ? h->heap : nullptr; }
+
+int gstm_init_heap(gstm_t* h, int workload)
+{
+    if (!h || workload < 0 || workload > 4) { set_error("gstm_init_heap: bad argument"); return GSTM_EINVAL; }
+    CUDA_TRY(launch_init_heap(workload, h->heap, h->heap_words, h->stream));
+    return GSTM_OK;
+}
+
+int gstm_write_heap(gstm_t* h, const uint32_t* src, uint64_t offset, uint64_t words)
+{
+    if (!h || (!src && words) || offset + words > h->heap_words) { set_error("gstm_write_heap: bad range"); return GSTM_EINVAL; }
+    if (!words) return GSTM_OK;
+    CUDA_TRY(cudaMemcpyAsync(h->heap + offset, src, words * 4, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return GSTM_OK;
+}
+
+int gstm_read_heap(gstm_t* h, uint32_t* dst, uint64_t offset, uint64_t words)
+{
+    if (!h || (!dst && words) || offset + words > h->heap_words) { set_error("gstm_read_heap: bad range"); return GSTM_EINVAL; }
+    if (!words) return GSTM_OK;
+    CUDA_TRY(cudaMemcpyAsync(dst, h->heap + offset, words * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return GSTM_OK;
+}
+
+int gstm_read_locks(gstm_t* h, uint32_t* dst, uint64_t n)
+{
+    if (!h || !dst || n > (1ull << h->bits)) { set_error("gstm_read_locks: bad range"); return GSTM_EINVAL; }
+    CUDA_TRY(cudaMemcpyAsync(dst, h->locks, n * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return GSTM_OK;
+}
+
+int gstm_read_clock(gstm_t* h, uint64_t* out)
+{
+    if (!h || !out) { set_error("gstm_read_clock: NULL"); return GSTM_EINVAL; }
+    unsigned long long c = 0;
+    CUDA_TRY(cudaMemcpyAsync(&c, h->meta + M_CLOCK, 8, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    *out = c;
+    return GSTM_OK;
+}
+
+int gstm_reset_meta(gstm_t* h)
+{
+    if (!h) { set_error("gstm_reset_meta: NULL"); return GSTM_EINVAL; }
+    CUDA_TRY(cudaMemsetAsync(h->locks, 0, sizeof(uint32_t) << h->bits, h->stream));
+    CUDA_TRY(cudaMemsetAsync(h->meta + M_CLOCK, 0, 8, h->stream));
+    h->clock_bound = 0;
+    return GSTM_OK;
+}
+
+int gstm_set_clock(gstm_t* h, uint64_t value)
+{
+    if (!h || value >= (1ull << 31)) { set_error("gstm_set_clock: bad argument"); return GSTM_EINVAL; }
+    unsigned long long v = value;
+    CUDA_TRY(cudaMemcpyAsync(h->meta + M_CLOCK, &v, 8, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (value > h->clock_bound) h->clock_bound = value;
+    return GSTM_OK;
+}
+
+static int resolve_mode(const gstm_t* h, uint64_t footprint)
+{
+    if (h->mode != GSTM_MODE_AUTO) return h->mode;
+    // STM-Optimized: HV when shared data exceeds the version locks
+    return footprint > (1ull << h->bits) ? GSTM_MODE_HV : GSTM_MODE_TBV;
+}
+
+int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed)
+{
+    if (!h) { set_error("gstm_launch: NULL handle"); return GSTM_EINVAL; }
+    const gstm_params_t& P = h->params;
+    WlParams w = wl_params(P, n_threads, tx_per_thread);
+    uint64_t fp = 0;
+    int dw = 0;
+    if (workload < 0 || workload > 4 || !workload_check(workload, w, &fp, &dw)) {
+        set_error("gstm_launch: invalid parameters for workload %d", workload);
+        return GSTM_EINVAL;
+    }
+    if (fp > h->heap_words) {
+        set_error("gstm_launch: workload footprint %llu words > heap %llu words", (unsigned long long)fp,
+                  (unsigned long long)h->heap_words);
+        return GSTM_EINVAL;
+    }
+    if (n_threads > (1ull << 32)) { set_error("gstm_launch: n_threads > 2^32"); return GSTM_EINVAL; }
+    const uint64_t n_tx = n_threads * tx_per_thread;
+    if (n_tx >= (1ull << 31) - 2) { set_error("gstm_launch: %llu transactions >= 2^31", (unsigned long long)n_tx); return GSTM_EOVERFLOW; }
+    // 31-bit versions: start a new version epoch before they can wrap
+    if (h->clock_bound + n_tx >= (1ull << 31) - 2) {
+        int rc = gstm_reset_meta(h);
+        if (rc) return rc;
+    }
+    if (P.verify && n_tx > h->log_cap) {
+        cudaFree(h->tx_stamp);
+        cudaFree(h->tx_result);
+        h->tx_stamp = h->tx_result = nullptr;
+        h->log_cap = 0;
+        if (cudaMalloc(&h->tx_stamp, n_tx * 4) != cudaSuccess || cudaMalloc(&h->tx_result, n_tx * 4) != cudaSuccess) {
+            cudaFree(h->tx_stamp);
+            h->tx_stamp = nullptr;
+            set_error("gstm_launch: cannot allocate the verify log (%llu tx)", (unsigned long long)n_tx);
+            return GSTM_ENOMEM;
+        }
+        h->log_cap = n_tx;
+    }
+    const int mode = resolve_mode(h, fp);
+    KParams kp;
+    memset(&kp, 0, sizeof(kp));
+    kp.m.heap = h->heap;
+    kp.m.locks = h->locks;
+    kp.m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
+    kp.m.clock = h->meta + M_CLOCK;
+    kp.m.spin_cap = P.spin_cap ? P.spin_cap : (1u << 16);
+    kp.w = w;
+    kp.meta = h->meta;
+    kp.tx_stamp = P.verify ? h->tx_stamp : nullptr;
+    kp.tx_result = P.verify ? h->tx_result : nullptr;
+    kp.T = n_threads;
+    kp.K = tx_per_thread;
+    kp.seed = seed;
+    kp.prelock_vbv = P.prelock_vbv;
+    kp.k_lock = P.k_lock;
+    kp.backoff_ns = P.backoff_ns;
+    const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
+    CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
+    CUDA_TRY(launch_prepare(h->meta, timeout_ns, h->stream));
+    CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
+    CUDA_TRY(launch_finish(h->meta, h->stream));
+    CUDA_TRY(cudaEventRecord(h->ev1, h->stream));
+    h->clock_bound += n_tx;
+    h->launched = true;
+    h->last_mode = mode;
+    h->last_n = n_tx;
+    return GSTM_OK;
+}
+
+int gstm_stats(gstm_t* h, gstm_stats_t* out)
+{
+    if (!h || !out) { set_error("gstm_stats: NULL"); return GSTM_EINVAL; }
+    if (!h->launched) { set_error("gstm_stats: no launch"); return GSTM_EBUSY; }
+    CUDA_TRY(cudaEventSynchronize(h->ev1));
+    unsigned long long m[M_WORDS];
+    CUDA_TRY(cudaMemcpyAsync(m, h->meta, sizeof(m), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    float ms = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&ms, h->ev0, h->ev1));
+    memset(out, 0, sizeof(*out));
+    const unsigned long long* s = m + M_STATS;
+    out->commits = s[S_COMMITS];
+    out->commits_ro = s[S_COMMITS_RO];
+    out->aborts_opacity = s[S_AB_OPACITY];
+    out->aborts_prevbv = s[S_AB_PREVBV];
+    out->aborts_tbv = s[S_AB_TBV];
+    out->aborts_commit_vbv = s[S_AB_COMMITVBV];
+    out->aborts_lock = s[S_AB_LOCK];
+    out->aborts = out->aborts_opacity + out->aborts_prevbv + out->aborts_tbv + out->aborts_commit_vbv + out->aborts_lock;
+    out->lock_retries = s[S_LOCK_RETRIES];
+    out->postvalidations = s[S_POSTVAL];
+    out->vbv_runs = s[S_VBV];
+    out->spins = s[S_SPINS];
+    out->attempts = s[S_ATTEMPTS];
+    out->errors = s[S_ERRORS];
+    out->clock_begin = m[M_CLOCK_BEGIN];
+    out->clock_end = m[M_CLOCK_END];
+    out->elapsed_ms = ms;
+    const double done = static_cast<double>(out->commits + out->commits_ro);
+    out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
+    out->abort_ratio = (done + out->aborts) > 0 ? out->aborts / (done + out->aborts) : 0.0;
+    out->mode_used = h->last_mode;
+    const uint32_t err = static_cast<uint32_t>(m[M_ERR]);
+    out->status = (err & ERR_TIMEOUT) ? GSTM_ETIMEOUT : (err & (ERR_LOGOVF | ERR_INVALID)) ? GSTM_ELOGOVF : GSTM_OK;
+    if (out->status) set_error("gstm_stats: launch reported %s", out->status == GSTM_ETIMEOUT ? "watchdog timeout" : "log overflow");
+    return out->status;
+}
+
+int gstm_read_tx_log(gstm_t* h, uint32_t* stamps, uint32_t* results, uint64_t n)
+{
+    if (!h) { set_error("gstm_read_tx_log: NULL"); return GSTM_EINVAL; }
+    if (!h->launched || !h->tx_stamp || n > h->log_cap) { set_error("gstm_read_tx_log: no verify log of %llu entries", (unsigned long long)n); return GSTM_EBUSY; }
+    if (stamps) CUDA_TRY(cudaMemcpyAsync(stamps, h->tx_stamp, n * 4, cudaMemcpyDeviceToHost, h->stream));
+    if (results) CUDA_TRY(cudaMemcpyAsync(results, h->tx_result, n * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return GSTM_OK;
+}
+
+int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
+                  uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed, gstm_stats_t* stats)
+{
+    if (!h || words > h->heap_words || (words && (!heap_in || !heap_out))) { set_error("gstm_run_host: bad buffers"); return GSTM_EINVAL; }
+    if (words) CUDA_TRY(cudaMemcpyAsync(h->heap, heap_in, words * 4, cudaMemcpyHostToDevice, h->stream));
+    int rc = gstm_launch(h, workload, n_threads, tx_per_thread, seed);
+    if (rc) return rc;
+    if (words) CUDA_TRY(cudaMemcpyAsync(heap_out, h->heap, words * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    gstm_stats_t local;
+    return gstm_stats(h, stats ? stats : &local);
+}
+
+int gstm_descr_words(gstm_t* h, int workload)
+{
+    if (!h) { set_error("gstm_descr_words: NULL"); return GSTM_EINVAL; }
+    WlParams w = wl_params(h->params, 1, 1);
+    uint64_t fp;
+    int dw = 0;
+    if (!workload_check(workload, w, &fp, &dw)) { set_error("gstm_descr_words: invalid workload params"); return GSTM_EINVAL; }
+    return dw;
+}
+
+int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed,
+                    uint32_t* host_out, uint32_t words_per_tx)
+{
+    if (!h || !host_out) { set_error("gstm_dump_descr: NULL"); return GSTM_EINVAL; }
+    WlParams w = wl_params(h->params, n_threads, tx_per_thread);
+    uint64_t fp;
+    int dw = 0;
+    if (!workload_check(workload, w, &fp, &dw) || static_cast<int>(words_per_tx) < dw) {
+        set_error("gstm_dump_descr: invalid workload params or words_per_tx < %d", dw);
+        return GSTM_EINVAL;
+    }
+    const uint64_t n = n_threads * tx_per_thread * words_per_tx;
+    if (!n) return GSTM_OK;
+    uint32_t* d = nullptr;
+    CUDA_TRY(cudaMalloc(&d, n * 4));
+    KParams kp;
+    memset(&kp, 0, sizeof(kp));
+    kp.w = w;
+    kp.T = n_threads;
+    kp.K = tx_per_thread;
+    kp.seed = seed;
+    cudaError_t e = launch_descr(workload, kp, d, static_cast<int>(words_per_tx), h->stream);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(host_out, d, n * 4, cudaMemcpyDeviceToHost, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+    cudaFree(d);
+    if (e != cudaSuccess) { set_error("gstm_dump_descr: %s", cudaGetErrorString(e)); return GSTM_ECUDA; }
+    return GSTM_OK;
+}
+
+int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx)
+{
+    if (!h || !ops || !out || n_ops < 0 || n_tx < 1 || n_tx > 8 || (mode != GSTM_MODE_HV && mode != GSTM_MODE_TBV)) {
+        set_error("gstm_script: bad argument");
+        return GSTM_EINVAL;
+    }
+    for (int k = 0; k < n_ops; ++k) {
+        const uint32_t op = ops[4 * k], slot = ops[4 * k + 1], word = ops[4 * k + 2];
+        if (op > 3 || slot >= static_cast<uint32_t>(n_tx) || ((op == 1 || op == 2) && word >= h->heap_words)) {
+            set_error("gstm_script: bad op %d", k);
+            return GSTM_EINVAL;
+        }
+    }
+    if (!n_ops) return GSTM_OK;
+    uint32_t *dops = nullptr, *dout = nullptr;
+    CUDA_TRY(cudaMalloc(&dops, n_ops * 16));
+    cudaError_t e = cudaMalloc(&dout, n_ops * 16);
+    Meta m;
+    m.heap = h->heap;
+    m.locks = h->locks;
+    m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
+    m.clock = h->meta + M_CLOCK;
+    m.spin_cap = 64;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dops, ops, n_ops * 16, cudaMemcpyHostToDevice, h->stream);
+    if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, h->stream);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(out, dout, n_ops * 16, cudaMemcpyDeviceToHost, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+    cudaFree(dops);
+    cudaFree(dout);
+    if (e != cudaSuccess) { set_error("gstm_script: %s", cudaGetErrorString(e)); return GSTM_ECUDA; }
+    return GSTM_OK;
+}
+
+int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant)
+{
+    if (!entries || !out || n < 0 || n > 4096 || (variant != 0 && variant != 1)) { set_error("gstm_lock_log: bad argument"); return GSTM_EINVAL; }
+    uint32_t *de = nullptr, *dout = nullptr;
+    int* dn = nullptr;
+    CUDA_TRY(cudaMalloc(&de, (n + 1) * 4));
+    CUDA_TRY(cudaMalloc(&dout, 256 * 4));
+    CUDA_TRY(cudaMalloc(&dn, 4));
+    int cnt = 0;
+    cudaError_t e = cudaMemcpy(de, entries, n * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = launch_lock_log(de, n, dout, dn, variant, 0);
+    if (e == cudaSuccess) e = cudaMemcpy(&cnt, dn, 4, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess && cnt > 0) e = cudaMemcpy(out, dout, cnt * 4, cudaMemcpyDeviceToHost);
+    cudaFree(de);
+    cudaFree(dout);
+    cudaFree(dn);
+    if (e != cudaSuccess) { set_error("gstm_lock_log: %s", cudaGetErrorString(e)); return GSTM_ECUDA; }
+    if (cnt < 0) { set_error("gstm_lock_log: capacity exceeded"); return GSTM_ELOGOVF; }
+    return cnt;
+}
+
+int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms)
+{
+    if (!ops_per_s) { set_error("gstm_ubench: NULL"); return GSTM_EINVAL; }
+    const int rc = ubench(kind, table_bytes, n_ops, threads, ops_per_s, ms);
+    if (rc == -1) { set_error("gstm_ubench: bad argument"); return GSTM_EINVAL; }
+    if (rc) { set_error("gstm_ubench: CUDA failure %d", rc); return GSTM_ECUDA; }
+    return GSTM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,123 @@
+// prim.cuh -- scoped memory operations and warp helpers for sm_100a.
+//
+// The paper's metadata lived in Fermi global memory accessed through
+// `volatile` with __threadfence() fences.  On sm_70+ the L1 is
+// not coherent for weak loads, so every access to shared STM data or metadata
+// here is a *strong* gpu-scope operation (SASS LDG/STG/ATOMG .STRONG.GPU,
+// which are served by the L2, the device's coherence point), and the paper's
+// fences (A3.l5, l12, l26, l79, l82) become PTX acquire/release operations or
+// `fence.acq_rel.gpu` (DESIGN.md §6.2 gives the ordering argument).
+//
+// SASS each helper compiles to (nvcc 12.9, sm_100a; checked with cuobjdump):
+//   ld_relaxed        LDG.E.STRONG.GPU
+//   ld_acquire        LDG.E.STRONG.GPU ; CCTL.IVALL
+//   st_relaxed        STG.E.STRONG.GPU
+//   fence_acq_rel     MEMBAR.ALL.GPU ; ERRBAR ; CGAERRBAR ; CCTL.IVALL
+//   atom_or_acquire   ATOMG.E.OR.STRONG.GPU ; CCTL.IVALL
+//   atom_add_acq_rel  MEMBAR.ALL.GPU ; ATOMG.E.ADD.64.STRONG.GPU ; CCTL.IVALL
+#pragma once
+#include <cstdint>
+
+namespace gstm {
+namespace prim {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t ld_relaxed(const uint32_t* p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ unsigned long long ld_acquire64(const unsigned long long* p)
+{
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long* p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_relaxed(uint32_t* p, uint32_t v)
+{
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void st_relaxed64(unsigned long long* p, unsigned long long v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v)
+{
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void fence_acq_rel()
+{
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
+__device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.acquire.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;"
+                 : "=r"(old) : "l"(p), "r"(cmp), "r"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ unsigned long long atom_add_acq_rel64(unsigned long long* p, unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ unsigned long long atom_add_relaxed64(unsigned long long* p, unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ uint32_t lane_id()
+{
+    uint32_t l;
+    asm volatile("mov.u32 %0, %%laneid;" : "=r"(l));
+    return l;
+}
+
+__device__ __forceinline__ uint32_t lanemask_lt()
+{
+    uint32_t m;
+    asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+__device__ __forceinline__ void nanosleep(uint32_t ns)
+{
+    if (ns) __nanosleep(ns);
+}
+
+}  // namespace prim
+}  // namespace gstm

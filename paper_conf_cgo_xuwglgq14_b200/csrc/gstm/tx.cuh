@@ -1,0 +1,384 @@
+// tx.cuh -- GPU-STM per-thread transaction runtime (device side).
+//
+// Implements TXBegin / TXRead / TXWrite / TXCommit of Algorithm 3
+// for one CUDA thread.  Logs live in per-thread arrays sized at compile time:
+// with small capacities (RA, bank, KM) every loop is unrolled and the logs
+// are registers; with large ones (EB, HT, scripts) they are per-thread local
+// memory, which the hardware interleaves across the 32 lanes of a warp --
+// exactly the "coalesced read-/write-set organization" of P:117 (entry i of
+// the merged set belongs to lane i mod 32).
+//
+// Metadata: a global table of 32-bit version locks (LSB = locked,
+// bits 31..1 = version), the global clock, and per transaction a read-set,
+// a write-set with a 64-bit bloom filter and a local lock log kept
+// sorted by lock id with rd/wr bits.
+//
+// The warp-collective parts of TXCommit (the warp-aware retry of P:147 and
+// the aggregated clock increment of A3.l83) are in kernels.cu; this header
+// holds the per-lane steps, which the scripted-interleaving kernel
+// (script.cu) also calls one transaction at a time.
+#pragma once
+#include <cstdint>
+#include "prim.cuh"
+
+namespace gstm {
+
+enum { MODE_HV = 1, MODE_TBV = 2 };
+
+// commit outcome / abort causes (same numbering as the C ABI stats)
+enum { C_OK = 0, C_OPACITY = 1, C_PREVBV = 2, C_TBV = 3, C_COMMITVBV = 4, C_READONLY = 5, C_LOCK = 6 };
+
+struct Meta {
+    uint32_t* heap;
+    uint32_t* locks;
+    uint32_t lock_mask;              // 2^bits - 1: hash(word) = word & mask (Q2)
+    unsigned long long* clock;       // g_clock
+    uint32_t spin_cap;               // bound on the l.27-29 spin and on PostValidation restarts
+};
+
+// bloom-filter bit of a word (reading Q7): top 6 bits of a Fibonacci hash
+__device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
+{
+    return 1ull << ((static_cast<unsigned long long>(w) * 0x9E3779B97F4A7C15ull) >> 58);
+}
+
+template <int RCAP, int WCAP, int LCAP>
+struct Tx {
+    static constexpr bool kUnroll = (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
+    static constexpr int kRcap = RCAP, kWcap = WCAP, kLcap = LCAP;
+
+    uint32_t r_addr[RCAP], r_val[RCAP];   // read-set  <addr,val>
+    uint32_t w_addr[WCAP], w_val[WCAP];   // write-set <addr,val> (redo log)
+    uint32_t l_ent[LCAP], l_old[LCAP];    // sorted lock log; old lock words
+    unsigned long long bloom;
+    int nr, nw, nl, n_acq;
+    uint32_t snapshot;
+    bool opaque, passTBV, overflow;
+    uint32_t n_postval, n_vbv, n_spin;    // per-thread statistics
+
+    __device__ __forceinline__ void reset_stats() { n_postval = n_vbv = n_spin = 0; }
+
+    // ---- A3.l1-5 TXBegin (the clock load and fence are done by the caller,
+    //      once per warp, see kernels.cu warp_snapshot) --------------------
+    __device__ __forceinline__ void begin(uint32_t snap)
+    {
+        nr = nw = nl = n_acq = 0;                 // l.2
+        bloom = 0ull;
+        opaque = passTBV = true;                  // l.3
+        overflow = false;
+        snapshot = snap;                          // l.4
+    }
+
+    __device__ __forceinline__ bool read_only() const { return nw == 0; }
+
+    // ---- A3.l22-23: read-after-write through the bloom filter ------------
+    __device__ __forceinline__ bool raw_lookup(uint32_t a, uint32_t& v) const
+    {
+        if (!(bloom & bloom_bit(a))) return false;
+        bool hit = false;
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < WCAP; ++k)
+                if (k < nw && w_addr[k] == a) { v = w_val[k]; hit = true; }
+        } else {
+            for (int k = 0; k < nw; ++k)
+                if (w_addr[k] == a) { v = w_val[k]; hit = true; break; }
+        }
+        return hit;
+    }
+
+    // ---- A3.l25: append to the read-set (reading Q5: duplicates kept) ----
+    __device__ __forceinline__ void append_read(uint32_t a, uint32_t v)
+    {
+        if (nr >= RCAP) { overflow = true; opaque = false; return; }
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+                if (k == nr) { r_addr[k] = a; r_val[k] = v; }
+        } else {
+            r_addr[nr] = a; r_val[nr] = v;
+        }
+        ++nr;
+    }
+
+    // ---- P:113-115, A3.l34/l38: sorted insert into the local lock log ----
+    // Entries are id<<2 | wr<<1 | rd, ascending by id; a duplicate id only
+    // ORs its bits (no new entry).
+    __device__ __forceinline__ void insert_lock(uint32_t e)
+    {
+        const uint32_t id = e >> 2;
+        if constexpr (kUnroll) {
+            int pos = 0;
+            bool dup = false;
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k) {
+                if (k < nl) {
+                    const uint32_t ik = l_ent[k] >> 2;
+                    pos += (ik < id) ? 1 : 0;
+                    if (ik == id) { l_ent[k] |= (e & 3u); dup = true; }
+                }
+            }
+            if (dup) return;
+            if (nl >= LCAP) { overflow = true; opaque = false; return; }
+#pragma unroll
+            for (int k = LCAP - 1; k > 0; --k)
+                if (k <= nl && k > pos) l_ent[k] = l_ent[k - 1];
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k == pos) l_ent[k] = e;
+            ++nl;
+        } else {
+            int pos = 0;
+            while (pos < nl && (l_ent[pos] >> 2) < id) ++pos;
+            if (pos < nl && (l_ent[pos] >> 2) == id) { l_ent[pos] |= (e & 3u); return; }
+            if (nl >= LCAP) { overflow = true; opaque = false; return; }
+            for (int k = nl; k > pos; --k) l_ent[k] = l_ent[k - 1];
+            l_ent[pos] = e;
+            ++nl;
+        }
+    }
+
+    // ---- A3.l62-66 VBV: every logged value still in memory ---------------
+    __device__ __forceinline__ bool vbv(const Meta& m)
+    {
+        ++n_vbv;
+        bool ok = true;
+        if constexpr (kUnroll) {
+            uint32_t cur[RCAP];
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+                if (k < nr) cur[k] = prim::ld_relaxed(m.heap + r_addr[k]);
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+                if (k < nr) ok &= (cur[k] == r_val[k]);
+        } else {
+            for (int k = 0; k < nr; ++k)
+                ok &= (prim::ld_relaxed(m.heap + r_addr[k]) == r_val[k]);
+        }
+        return ok;
+    }
+
+    // ---- A3.l6-20 PostValidation(version) --------------------------------
+    // "snapshot <- version" (l.7) never lowers the snapshot (reading Q9);
+    // restarts are bounded by spin_cap (the paper loops; bounded => abort).
+    __device__ __forceinline__ bool post_validation(const Meta& m, uint32_t version)
+    {
+        ++n_postval;
+        if (version > snapshot) snapshot = version;                // l.7
+        for (uint32_t restart = 0; restart <= m.spin_cap; ++restart) {   // l.8
+            if (!vbv(m)) return false;                               // l.9-11
+            prim::fence_acq_rel();                                   // l.12
+            bool again = false;
+            uint32_t newsnap = snapshot;
+            if constexpr (kUnroll) {
+                uint32_t vl[RCAP];
+#pragma unroll
+                for (int k = 0; k < RCAP; ++k)                       // l.13
+                    if (k < nr) vl[k] = prim::ld_relaxed(m.locks + (r_addr[k] & m.lock_mask)); // l.14
+#pragma unroll
+                for (int k = 0; k < RCAP; ++k)
+                    if (k < nr && ((vl[k] & 1u) || (vl[k] >> 1) > snapshot)) {   // l.15-17
+                        newsnap = max(newsnap, vl[k] >> 1);          // l.18 (Q9)
+                        again = true;                                // l.19 goto loop
+                    }
+            } else {
+                for (int k = 0; k < nr; ++k) {
+                    const uint32_t vl = prim::ld_relaxed(m.locks + (r_addr[k] & m.lock_mask));
+                    if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                }
+            }
+            snapshot = newsnap;
+            if (!again) return true;                                 // l.20
+            if (restart) __nanosleep(64);
+        }
+        return false;
+    }
+
+    // ---- A3.l27-33: wait while locked, then timestamp check --------------
+    __device__ __forceinline__ void check_lock(const Meta& m, uint32_t a, uint32_t vl, int mode)
+    {
+        uint32_t spins = 0;
+        while (vl & 1u) {                                            // l.29
+            if (++spins > m.spin_cap) { opaque = false; break; }
+            __nanosleep(32);
+            vl = prim::ld_relaxed(m.locks + (a & m.lock_mask));      // l.28
+        }
+        n_spin += spins;
+        const uint32_t version = vl >> 1;                            // l.30
+        if (opaque && version > snapshot) {                          // l.31
+            if (mode == MODE_HV) {
+                if (!post_validation(m, version)) opaque = false;    // l.32-33
+            } else {
+                opaque = false;                                      // TBV-only (Q18)
+            }
+        }
+    }
+
+    // ---- A3.l21-35 TXRead(addr) -------------------------------------------
+    __device__ __forceinline__ uint32_t read(const Meta& m, uint32_t a, int mode)
+    {
+        uint32_t v;
+        if (raw_lookup(a, v)) return v;                              // l.22-23
+        v = prim::ld_relaxed(m.heap + a);                            // l.24
+        append_read(a, v);                                           // l.25
+        prim::fence_acq_rel();                                       // l.26
+        const uint32_t vl = prim::ld_relaxed(m.locks + (a & m.lock_mask));
+        check_lock(m, a, vl, mode);                                  // l.27-33
+        insert_lock(((a & m.lock_mask) << 2) | 1u);                  // l.34
+        return v;                                                    // l.35
+    }
+
+    // Batched TXRead of N words whose addresses are known together: the N
+    // value loads (l.24) are issued back to back, one fence (l.26) orders all
+    // of them before the N lock loads, then each read runs l.27-34 in order.
+    // Equivalent to N sequential TXReads with the value loads hoisted: each
+    // value is still checked against its lock after it was loaded (DESIGN.md
+    // §6.3), but the transaction pays 2 dependent memory round trips instead
+    // of 2N.
+    template <int N>
+    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode)
+    {
+        bool need[N];
+        uint32_t vl[N];
+#pragma unroll
+        for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) v[k] = prim::ld_relaxed(m.heap + a[k]);    // l.24
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) append_read(a[k], v[k]);                    // l.25
+        prim::fence_acq_rel();                                       // l.26
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) vl[k] = prim::ld_relaxed(m.locks + (a[k] & m.lock_mask));
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) {
+                check_lock(m, a[k], vl[k], mode);                    // l.27-33
+                insert_lock(((a[k] & m.lock_mask) << 2) | 1u);       // l.34
+            }
+    }
+
+    // ---- A3.l36-38 TXWrite(addr, val): upsert, bloom, sorted lock insert --
+    __device__ __forceinline__ void write(const Meta& m, uint32_t a, uint32_t v)
+    {
+        bool found = false;
+        if (bloom & bloom_bit(a)) {
+            if constexpr (kUnroll) {
+#pragma unroll
+                for (int k = 0; k < WCAP; ++k)
+                    if (k < nw && w_addr[k] == a) { w_val[k] = v; found = true; }
+            } else {
+                for (int k = 0; k < nw; ++k)
+                    if (w_addr[k] == a) { w_val[k] = v; found = true; break; }
+            }
+        }
+        if (!found) {                                                // l.37
+            if (nw >= WCAP) { overflow = true; opaque = false; return; }
+            if constexpr (kUnroll) {
+#pragma unroll
+                for (int k = 0; k < WCAP; ++k)
+                    if (k == nw) { w_addr[k] = a; w_val[k] = v; }
+            } else {
+                w_addr[nw] = a; w_val[nw] = v;
+            }
+            ++nw;
+            bloom |= bloom_bit(a);
+        }
+        insert_lock(((a & m.lock_mask) << 2) | 2u);                  // l.38
+    }
+
+    // ---- A3.l53-55 ReleaseLocks: restore the words this attempt acquired --
+    __device__ __forceinline__ void release_locks(const Meta& m)
+    {
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k < n_acq) prim::st_relaxed(m.locks + (l_ent[k] >> 2), l_old[k]);
+        } else {
+            for (int k = 0; k < n_acq; ++k) prim::st_relaxed(m.locks + (l_ent[k] >> 2), l_old[k]);
+        }
+        n_acq = 0;
+    }
+
+    // ---- A3.l43-52 GetLocksAndTBV -----------------------------------------
+    // Locks are taken one at a time in ascending id and acquisition stops at
+    // the first lock already held (reading Q15): this global order is what
+    // makes lockstep retry livelock-free.
+    __device__ __forceinline__ bool get_locks_and_tbv(const Meta& m)
+    {
+        n_acq = 0;
+        bool ok = true;
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k) {
+                if (ok && k < nl) {
+                    const uint32_t vl = prim::atom_or_acquire(m.locks + (l_ent[k] >> 2), 1u);  // l.45
+                    if (vl & 1u) {
+                        ok = false;                                  // l.46-48
+                    } else {
+                        l_old[k] = vl;
+                        n_acq = k + 1;
+                        if ((l_ent[k] & 1u) && (vl >> 1) > snapshot) passTBV = false;  // l.49-51
+                    }
+                }
+            }
+        } else {
+            for (int k = 0; k < nl; ++k) {
+                const uint32_t vl = prim::atom_or_acquire(m.locks + (l_ent[k] >> 2), 1u);
+                if (vl & 1u) { ok = false; break; }
+                l_old[k] = vl;
+                n_acq = k + 1;
+                if ((l_ent[k] & 1u) && (vl >> 1) > snapshot) passTBV = false;
+            }
+        }
+        if (!ok) release_locks(m);                                   // l.47
+        return ok;                                                   // l.52
+    }
+
+    // Commit steps up to the write-back (A3.l67-78).  Returns C_OK when all
+    // locks are held and the read-set is valid, C_LOCK on a lock conflict
+    // (nothing held; retry, l.73-74), or an abort cause (nothing held).
+    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv)
+    {
+        if (mode == MODE_HV && prelock_vbv)
+            if (!vbv(m)) return C_PREVBV;                            // l.71-72
+        if (!get_locks_and_tbv(m)) return C_LOCK;                    // l.73
+        if (!passTBV) {                                              // l.75
+            if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18
+            if (!vbv(m)) { release_locks(m); return C_COMMITVBV; }   // l.76-78
+        }
+        return C_OK;
+    }
+
+    // ---- A3.l80-81 write-back (lazy update of the redo log) --------------
+    __device__ __forceinline__ void writeback(const Meta& m)
+    {
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < WCAP; ++k)
+                if (k < nw) prim::st_relaxed(m.heap + w_addr[k], w_val[k]);
+        } else {
+            for (int k = 0; k < nw; ++k) prim::st_relaxed(m.heap + w_addr[k], w_val[k]);
+        }
+    }
+
+    // ---- A3.l56-61 ReleaseAndUpdateLocks(version) -------------------------
+    // Written locks get version<<1; read-only locks get back the exact word
+    // the acquiring atomic returned (reading Q16: == lock - 1).
+    __device__ __forceinline__ void release_and_update(const Meta& m, uint32_t version)
+    {
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k < nl) prim::st_relaxed(m.locks + (l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
+        } else {
+            for (int k = 0; k < nl; ++k)
+                prim::st_relaxed(m.locks + (l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
+        }
+        n_acq = 0;
+    }
+};
+
+}  // namespace gstm

@@ -1,0 +1,330 @@
+// workloads.cuh -- transaction bodies of the five synthetic workloads.
+//
+// The paper's workloads are random array (RA, Figure 1), hash table
+// (HT), EigenBench (EB) and the STAMP ports; their values are not
+// specified (Table 1 is lost).  The bodies here follow our recipe
+// plus a bank transfer (BASELINE configs[1]).
+// Each body is written once against a context type:
+//   StmCtx    -- transactional TXRead / TXWrite (tx.cuh)
+//   DirectCtx -- plain strong loads/stores, used by the CGL and FGL baselines
+//                while they hold their locks.
+// The addresses and constants come from the counter-based generator
+// (gen.cuh), so an aborted transaction re-executes identically.
+#pragma once
+#include <cstdint>
+#include "gen.cuh"
+#include "prim.cuh"
+#include "tx.cuh"
+
+namespace gstm {
+
+struct WlParams {
+    uint64_t n_words;        // RA / bank / EB: address range (EB: hot set H)
+    uint32_t n_reads, n_writes, ra_kind, n_accesses;
+    uint32_t ht_buckets, ht_lookup_pct;
+    uint64_t ht_key_range;
+    uint32_t km_clusters, km_dims;
+    uint64_t T, K;           // launch shape (HT node layout needs M = T*K)
+};
+
+// ---- contexts --------------------------------------------------------------
+template <class TX>
+struct StmCtx {
+    TX& tx;
+    const Meta& m;
+    int mode;
+    __device__ __forceinline__ uint32_t read(uint32_t a) { return tx.read(m, a, mode); }
+    template <int N>
+    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n)
+    {
+        tx.template read_batch<N>(m, a, v, n, mode);
+    }
+    __device__ __forceinline__ void write(uint32_t a, uint32_t v) { tx.write(m, a, v); }
+    __device__ __forceinline__ bool ok() const { return tx.opaque; }
+    // the body found its own view inconsistent (e.g. a chain pointer out of
+    // range): only possible for a transaction that is about to abort
+    __device__ __forceinline__ void invalid() { tx.opaque = false; }
+    // the transaction needs more log entries than compiled in: sticky error
+    __device__ __forceinline__ void overflow() { tx.overflow = true; tx.opaque = false; }
+    static constexpr int kMaxChain = (TX::kRcap - 1) / 2;
+};
+
+struct DirectCtx {
+    uint32_t* heap;
+    int nw;
+    bool bad;
+    __device__ __forceinline__ uint32_t read(uint32_t a) { return prim::ld_relaxed(heap + a); }
+    template <int N>
+    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n)
+    {
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (k < n) v[k] = prim::ld_relaxed(heap + a[k]);
+    }
+    __device__ __forceinline__ void write(uint32_t a, uint32_t v) { prim::st_relaxed(heap + a, v); ++nw; }
+    __device__ __forceinline__ bool ok() const { return !bad; }
+    __device__ __forceinline__ void invalid() { bad = true; }
+    __device__ __forceinline__ void overflow() { bad = true; }
+    static constexpr int kMaxChain = 1 << 30;
+};
+
+__device__ __forceinline__ uint32_t lo32(uint64_t v) { return static_cast<uint32_t>(v); }
+
+// ---- RA kind 0: R reads then W writes (Figure 1 random array) -------------
+// acc = sum of the words read; write w_j <- acc + c_j; result = acc.
+struct RaWL {
+    static constexpr int MAXR = 8, MAXW = 8;
+    static constexpr int RCAP = MAXR, WCAP = MAXW, LCAP = MAXR + MAXW, FGL_LCAP = MAXR + MAXW;
+    static constexpr int DESCR = MAXR + 2 * MAXW;
+    __host__ static bool check(const WlParams& p)
+    {
+        return p.ra_kind == 0 && p.n_reads <= MAXR && p.n_writes <= MAXW && p.n_words > 0;
+    }
+    __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    {
+        const int R = static_cast<int>(p.n_reads), W = static_cast<int>(p.n_writes);
+        uint32_t a[MAXR], v[MAXR];
+#pragma unroll
+        for (int j = 0; j < MAXR; ++j)
+            a[j] = j < R ? static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)) : 0u;
+        c.template read_batch<MAXR>(a, v, R);
+        if (!c.ok()) return;
+        uint32_t acc = 0;
+#pragma unroll
+        for (int j = 0; j < MAXR; ++j)
+            if (j < R) acc += v[j];
+#pragma unroll
+        for (int j = 0; j < MAXW; ++j)
+            if (j < W) {
+                const uint32_t w = static_cast<uint32_t>(gen::bounded(gen::draw(x, R + j), p.n_words));
+                c.write(w, acc + lo32(gen::draw(x, R + W + j)));
+            }
+        result = acc;
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        const uint32_t R = p.n_reads, W = p.n_writes;
+        for (uint32_t j = 0; j < R + W; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        const uint32_t R = p.n_reads, W = p.n_writes;
+        for (uint32_t j = 0; j < R + W; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        for (uint32_t j = 0; j < W; ++j) out[R + W + j] = lo32(gen::draw(x, R + W + j));
+        return static_cast<int>(R + 2 * W);
+    }
+};
+
+// ---- RA kind 1: increment form, read-modify-write of each r_j -------------
+// (Figure 1 style: interleaved TXRead / TXWrite, with read-after-write
+// through the write-set).  result = sum of the values read.
+struct RaIncWL {
+    static constexpr int MAXR = 16;
+    static constexpr int RCAP = MAXR, WCAP = MAXR, LCAP = MAXR, FGL_LCAP = MAXR;
+    static constexpr int DESCR = MAXR;
+    __host__ static bool check(const WlParams& p) { return p.ra_kind == 1 && p.n_reads <= MAXR && p.n_words > 0; }
+    __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    {
+        uint32_t acc = 0;
+        for (uint32_t j = 0; j < p.n_reads; ++j) {
+            const uint32_t a = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+            const uint32_t v = c.read(a);
+            if (!c.ok()) return;       // Figure 1: break when not opaque
+            c.write(a, v + 1u);
+            acc += v;
+        }
+        result = acc;
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        for (uint32_t j = 0; j < p.n_reads; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        for (uint32_t j = 0; j < p.n_reads; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        return static_cast<int>(p.n_reads);
+    }
+};
+
+// ---- bank transfer (BASELINE configs[1]) -----------------------------------
+struct BankWL {
+    static constexpr int RCAP = 2, WCAP = 2, LCAP = 4, FGL_LCAP = 2;
+    static constexpr int DESCR = 3;
+    __host__ static bool check(const WlParams& p) { return p.n_words >= 2 && p.n_words <= (1ull << 32); }
+    __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
+    __device__ __forceinline__ static void accounts(const WlParams& p, uint64_t x, uint32_t& a, uint32_t& b, uint32_t& amt)
+    {
+        a = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.n_words));
+        b = static_cast<uint32_t>(gen::bounded(gen::draw(x, 1), p.n_words - 1));
+        b += (b >= a) ? 1u : 0u;
+        amt = 1u + static_cast<uint32_t>(gen::bounded(gen::draw(x, 2), 100));
+    }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    {
+        uint32_t ad[2], v[2], amt;
+        accounts(p, x, ad[0], ad[1], amt);
+        c.template read_batch<2>(ad, v, 2);
+        if (!c.ok()) return;
+        if (static_cast<int32_t>(v[0]) >= static_cast<int32_t>(amt)) {
+            c.write(ad[0], v[0] - amt);
+            c.write(ad[1], v[1] + amt);
+            result = 1;
+        } else {
+            result = 0;
+        }
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        uint32_t a, b, amt;
+        accounts(p, x, a, b, amt);
+        f(a);
+        f(b);
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        accounts(p, x, out[0], out[1], out[2]);
+        return 3;
+    }
+};
+
+// ---- chained hash table, set semantics (BASELINE configs[2]) ---------------
+// heap = [heads B | key[M] | next[M]], node n (1..M) of tx_id = n-1; 0 = null.
+struct HtWL {
+    static constexpr int MAXCHAIN = 24;
+    static constexpr int RCAP = 1 + 2 * MAXCHAIN, WCAP = 3, LCAP = RCAP + WCAP, FGL_LCAP = 1;
+    static constexpr int DESCR = 3;
+    __host__ static bool check(const WlParams& p)
+    {
+        return p.ht_buckets && !(p.ht_buckets & (p.ht_buckets - 1)) && p.ht_key_range >= 1 &&
+               p.ht_key_range < (1ull << 32) && p.ht_buckets + 2 * p.T * p.K < (1ull << 32);
+    }
+    __host__ static uint64_t footprint(const WlParams& p) { return p.ht_buckets + 2 * p.T * p.K; }
+    __device__ __forceinline__ static void key_of(const WlParams& p, uint64_t x, uint32_t& key, uint32_t& ins, uint32_t& bucket)
+    {
+        key = 1u + static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.ht_key_range));
+        ins = gen::bounded(gen::draw(x, 1), 100) >= p.ht_lookup_pct ? 1u : 0u;
+        bucket = static_cast<uint32_t>(gen::mix64(key) & (p.ht_buckets - 1));
+    }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t t, uint64_t i, uint32_t& result)
+    {
+        uint32_t key, ins, bucket;
+        key_of(p, x, key, ins, bucket);
+        const uint64_t B = p.ht_buckets, M = p.T * p.K;
+        const uint32_t h0 = c.read(bucket);
+        if (!c.ok()) return;
+        uint32_t h = h0, found = 0;
+        for (int steps = 0; h != 0; ++steps) {
+            if (h > M) { c.invalid(); return; }
+            if (steps >= Ctx::kMaxChain) { c.overflow(); return; }
+            uint32_t a[2] = {static_cast<uint32_t>(B + h - 1), static_cast<uint32_t>(B + M + h - 1)}, v[2];
+            c.template read_batch<2>(a, v, 2);            // key[h], next[h]
+            if (!c.ok()) return;
+            if (v[0] == key) { found = 1; break; }
+            h = v[1];
+        }
+        if (!ins) { result = found; return; }
+        if (found) { result = 2; return; }
+        const uint32_t n = static_cast<uint32_t>(1 + i * p.T + t);
+        c.write(static_cast<uint32_t>(B + n - 1), key);
+        c.write(static_cast<uint32_t>(B + M + n - 1), h0);
+        c.write(bucket, n);
+        result = 3;
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        uint32_t key, ins, bucket;
+        key_of(p, x, key, ins, bucket);
+        f(bucket);      // one lock per bucket: node words are private until linked, then immutable
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        key_of(p, x, out[0], out[1], out[2]);
+        return 3;
+    }
+};
+
+// ---- EigenBench-style: A accesses alternating read / write over H words ----
+struct EbWL {
+    static constexpr int MAXA = 64;
+    static constexpr int RCAP = MAXA / 2, WCAP = MAXA / 2, LCAP = MAXA, FGL_LCAP = MAXA;
+    static constexpr int DESCR = 2 * MAXA;
+    __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
+    __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    {
+        const uint32_t A = p.n_accesses;
+        uint32_t acc = 0;
+        for (uint32_t j = 0; j < A; ++j) {
+            const uint32_t a = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+            if ((j & 1u) == 0) {
+                acc += c.read(a);
+                if (!c.ok()) return;
+            } else {
+                c.write(a, acc + lo32(gen::draw(x, A + j)));
+            }
+        }
+        result = acc;
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        for (uint32_t j = 0; j < p.n_accesses; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        const uint32_t A = p.n_accesses;
+        for (uint32_t j = 0; j < A; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        for (uint32_t j = 0; j < A; ++j) out[A + j] = lo32(gen::draw(x, A + j));
+        return static_cast<int>(2 * A);
+    }
+};
+
+// ---- k-means cluster update (STAMP kmeans' transactional step) -------------
+// record of cluster c = [count, sum_0 .. sum_{D-1}] at word c*(D+1).
+struct KmWL {
+    static constexpr int MAXD = 16;
+    static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
+    static constexpr int DESCR = MAXD + 1;
+    __host__ static bool check(const WlParams& p) { return p.km_clusters > 0 && p.km_dims <= MAXD; }
+    __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * (p.km_dims + 1); }
+    template <class Ctx>
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    {
+        const int D = static_cast<int>(p.km_dims);
+        const uint32_t base = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * (p.km_dims + 1);
+        uint32_t a[MAXD + 1], v[MAXD + 1];
+#pragma unroll
+        for (int k = 0; k <= MAXD; ++k) a[k] = base + k;
+        c.template read_batch<MAXD + 1>(a, v, D + 1);
+        if (!c.ok()) return;
+        c.write(base, v[0] + 1u);
+#pragma unroll
+        for (int d = 0; d < MAXD; ++d)
+            if (d < D) c.write(base + 1 + d, v[1 + d] + static_cast<uint32_t>(gen::draw(x, 1 + d) >> 56));
+        result = v[0];
+    }
+    template <class F>
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    {
+        f(static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * (p.km_dims + 1));   // one lock per record
+    }
+    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    {
+        out[0] = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters));
+        for (uint32_t d = 0; d < p.km_dims; ++d) out[1 + d] = static_cast<uint32_t>(gen::draw(x, 1 + d) >> 56);
+        return static_cast<int>(1 + p.km_dims);
+    }
+};
+
+}  // namespace gstm

@@ -1,0 +1,443 @@
+// kernels.cu -- the transaction kernels (STM-HV, STM-TBV, CGL, FGL) and
+// their helpers.
+//
+// One CUDA thread = one STM thread t (Figure 1) that runs K
+// transactions i = 0..K-1 (tx_id = i*T + t).  The loop is warp-uniform:
+// every iteration the 32 lanes each attempt their current transaction
+// together (lanes whose transaction committed move on to the next one, the
+// others re-execute theirs), and commit is a warp-collective phase:
+//   * lock acquisition rounds: lanes that fail to get a lock retry only
+//     after the lanes of the same warp that got theirs finished committing
+//     ("On locking failure, it retries after transactions within the same
+//     warp finish committing"), for at most k_lock rounds;
+//   * the committing lanes of a round take their commit stamps with ONE
+//     atomic on the global clock (A3.l83 aggregated over the warp);
+//   * the snapshot (A3.l4) is read once per warp and broadcast.
+#include <cstdint>
+#include "kernels.cuh"
+
+namespace gstm {
+
+using prim::FULL;
+
+__device__ __forceinline__ unsigned long long globaltimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// A3.l4-5: snapshot <- g_clock; threadfence.  One acquire load per warp; the
+// __syncwarp orders every lane's later accesses after it.
+__device__ __forceinline__ uint32_t warp_snapshot(unsigned long long* clock)
+{
+    unsigned long long s = 0;
+    if (prim::lane_id() == 0) s = prim::ld_acquire64(clock);
+    s = __shfl_sync(FULL, s, 0);
+    __syncwarp();
+    return static_cast<uint32_t>(s);
+}
+
+// warp-aggregated commit stamp (A3.l83): lanes in `got` each receive a
+// distinct stamp; one atom.add per warp round.  The __syncwarp before the
+// atomic orders every committing lane's write-back (l.80-81) before the
+// leader's release-atomic (l.82); the one after orders the leader's acquire
+// before every lane's lock release.
+__device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool got, unsigned& gm)
+{
+    __syncwarp();
+    gm = __ballot_sync(FULL, got);
+    unsigned long long base = 0;
+    if (gm) {
+        const int leader = __ffs(gm) - 1;
+        if (static_cast<int>(prim::lane_id()) == leader) base = prim::atom_add_acq_rel64(clock, __popc(gm));
+        base = __shfl_sync(FULL, base, leader);
+        __syncwarp();
+    }
+    return static_cast<uint32_t>(base) + __popc(gm & prim::lanemask_lt()) + 1u;
+}
+
+struct Counters {
+    uint32_t c[S_NSTATS];
+    __device__ __forceinline__ Counters()
+    {
+#pragma unroll
+        for (int k = 0; k < S_NSTATS; ++k) c[k] = 0;
+    }
+};
+
+// warp reduce -> shared -> one global atomic per counter per block
+__device__ __forceinline__ void flush_counters(const Counters& cnt, unsigned long long* stats)
+{
+    __shared__ unsigned long long sh[S_NSTATS];
+    if (threadIdx.x < S_NSTATS) sh[threadIdx.x] = 0;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < S_NSTATS; ++k) {
+        const uint32_t v = __reduce_add_sync(FULL, cnt.c[k]);
+        if (prim::lane_id() == 0 && v) atomicAdd(&sh[k], static_cast<unsigned long long>(v));
+    }
+    __syncthreads();
+    if (threadIdx.x < S_NSTATS && sh[threadIdx.x]) atomicAdd(stats + threadIdx.x, sh[threadIdx.x]);
+}
+
+__device__ __forceinline__ void set_err(unsigned long long* meta, uint32_t bits)
+{
+    atomicOr(reinterpret_cast<unsigned int*>(meta + M_ERR), bits);
+}
+
+// warp-uniform watchdog check (every 16 iterations)
+__device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long deadline)
+{
+    if (iter & 15u) return false;
+    bool late = false;
+    if (prim::lane_id() == 0) late = globaltimer() > deadline;
+    return __shfl_sync(FULL, late, 0);
+}
+
+// ---------------------------------------------------------------------------
+// STM kernel: GPU-STM with hierarchical validation (MODE_HV, "STM-HV-Sorting")
+// or timestamp-only validation (MODE_TBV, "STM-TBV-Sorting").
+// ---------------------------------------------------------------------------
+template <class WL, int MODE>
+__global__ void __launch_bounds__(256) stm_kernel(const KParams p)
+{
+    using TX = Tx<WL::RCAP, WL::WCAP, WL::LCAP>;
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    const bool valid = t < p.T;
+    const Meta m = p.m;
+    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
+    const unsigned long long deadline = p.meta[M_DEADLINE];
+    Counters cnt;
+    TX tx;
+    tx.reset_stats();
+    uint32_t i = 0, iter = 0, backoff = 0;
+    bool timed_out = false;
+
+    while (__any_sync(FULL, valid && i < p.K)) {
+        if (warp_late(iter++, deadline)) { timed_out = true; break; }
+        const bool act = valid && i < p.K;
+        const uint32_t snap = warp_snapshot(m.clock);                 // TXBegin l.4-5
+        const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
+        uint32_t result = 0;
+        if (act) {
+            ++cnt.c[S_ATTEMPTS];
+            const uint64_t x = gen::tx_key(p.seed, t, i);
+            tx.begin(snap);                                           // TXBegin l.2-3
+            StmCtx<TX> ctx{tx, m, MODE};
+            WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
+        }
+        bool done = false, skip = false;
+        bool pending = act && tx.opaque && !tx.read_only();
+        if (act && !tx.opaque) {
+            if (tx.overflow) { ++cnt.c[S_ERRORS]; skip = true; }    // sticky ELOGOVF, give up this tx
+            else ++cnt.c[S_AB_OPACITY];                              // Figure 1 / Q11
+        }
+        if (act && tx.opaque && tx.read_only()) {                     // l.68: linearized at snapshot
+            if (p.tx_stamp) {
+                p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
+                p.tx_result[tx_id] = result;
+            }
+            ++cnt.c[S_COMMITS_RO];
+            done = true;
+        }
+        // warp-collective TXCommit (l.67-85)
+        for (uint32_t round = 0; __any_sync(FULL, pending); ++round) {
+            bool got = false;
+            if (pending) {
+                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0);
+                if (r == C_OK) {
+                    got = true;
+                    tx.writeback(m);                                  // l.79-81
+                } else if (r == C_LOCK) {
+                    ++cnt.c[S_LOCK_RETRIES];                          // l.73-74 retry next round
+                    if (p.k_lock && round + 1 >= p.k_lock) { pending = false; ++cnt.c[S_AB_LOCK]; }
+                } else {
+                    pending = false;
+                    ++cnt.c[r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV)];
+                }
+            }
+            unsigned gm;
+            const uint32_t stamp = warp_stamp(m.clock, got, gm);     // l.82-83
+            if (got) {
+                prim::fence_acq_rel();
+                tx.release_and_update(m, stamp);                      // l.84
+                if (p.tx_stamp) {
+                    p.tx_stamp[tx_id] = stamp - clock_begin;
+                    p.tx_result[tx_id] = result;
+                }
+                ++cnt.c[S_COMMITS];
+                pending = false;
+                done = true;
+            }
+        }
+        if (done || skip) {
+            ++i;
+            backoff = 0;
+        } else if (p.backoff_ns) {
+            // warp-uniform exponential backoff after an abort (all lanes sleep
+            // together: per-lane delays cannot work under SIMT)
+            if (__any_sync(FULL, act)) {
+                backoff = backoff ? min(backoff * 2u, 64u * p.backoff_ns) : p.backoff_ns;
+                __nanosleep(backoff);
+            }
+        }
+    }
+    cnt.c[S_POSTVAL] = tx.n_postval;
+    cnt.c[S_VBV] = tx.n_vbv;
+    cnt.c[S_SPINS] = tx.n_spin;
+    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
+    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
+    flush_counters(cnt, p.meta + M_STATS);
+}
+
+// ---------------------------------------------------------------------------
+// CGL baseline: one global lock serialises every transaction, taken
+// with Algorithm 1 Scheme #3 (diverge on failure) plus a test before
+// the CAS.  The body runs in place; the stamp is taken under the lock.
+// ---------------------------------------------------------------------------
+template <class WL>
+__global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
+{
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    const bool valid = t < p.T;
+    uint32_t* lock = reinterpret_cast<uint32_t*>(p.meta + M_CGL_LOCK);
+    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
+    const unsigned long long deadline = p.meta[M_DEADLINE];
+    Counters cnt;
+    uint32_t i = 0, iter = 0;
+    bool timed_out = false;
+    while (__any_sync(FULL, valid && i < p.K)) {
+        if (warp_late(iter++, deadline)) { timed_out = true; break; }
+        const bool act = valid && i < p.K;
+        if (act) {
+            ++cnt.c[S_ATTEMPTS];
+            if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
+                const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
+                DirectCtx ctx{p.m.heap, 0, false};
+                uint32_t result = 0;
+                WL::body(ctx, p.w, gen::tx_key(p.seed, t, i), t, i, result);   // critical section
+                uint32_t s;
+                if (ctx.nw) {
+                    s = static_cast<uint32_t>(prim::atom_add_relaxed64(p.m.clock, 1ull)) + 1u - clock_begin;
+                    ++cnt.c[S_COMMITS];
+                } else {
+                    s = 0x80000000u | (static_cast<uint32_t>(prim::ld_relaxed64(p.m.clock)) - clock_begin);
+                    ++cnt.c[S_COMMITS_RO];
+                }
+                if (ctx.bad) ++cnt.c[S_ERRORS];
+                if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
+                prim::fence_acq_rel();
+                prim::st_relaxed(lock, 0u);                           // Scheme #3 l.15
+                ++i;
+            } else {
+                ++cnt.c[S_LOCK_RETRIES];
+                if (p.backoff_ns) __nanosleep(p.backoff_ns);
+            }
+        }
+    }
+    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
+    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_INVALID);
+    flush_counters(cnt, p.meta + M_STATS);
+}
+
+// ---------------------------------------------------------------------------
+// FGL baseline: the hand-locking a programmer would write -- one lock per
+// stripe of the words the transaction will touch (per account, per bucket,
+// per k-means record), acquired in ascending id with try-lock and
+// release-all on failure, then the body in place.  No logs, no validation.
+// (The paper did not implement FGL; north_star asks for it.)
+// ---------------------------------------------------------------------------
+template <class WL>
+__global__ void __launch_bounds__(256) fgl_kernel(const KParams p)
+{
+    using TX = Tx<1, 1, WL::FGL_LCAP>;      // only the sorted lock log is used
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    const bool valid = t < p.T;
+    const Meta m = p.m;
+    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
+    const unsigned long long deadline = p.meta[M_DEADLINE];
+    Counters cnt;
+    TX lk;
+    uint32_t i = 0, iter = 0;
+    bool timed_out = false;
+    while (__any_sync(FULL, valid && i < p.K)) {
+        if (warp_late(iter++, deadline)) { timed_out = true; break; }
+        const bool act = valid && i < p.K;
+        const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
+        bool got = false;
+        int nw = 0;
+        uint32_t result = 0;
+        if (act) {
+            ++cnt.c[S_ATTEMPTS];
+            const uint64_t x = gen::tx_key(p.seed, t, i);
+            lk.begin(0);
+            WL::fgl_words(p.w, x, t, i, [&](uint32_t w) { lk.insert_lock(((w & m.lock_mask) << 2) | 2u); });
+            if (lk.overflow) {
+                ++cnt.c[S_ERRORS];
+            } else if (lk.get_locks_and_tbv(m)) {
+                got = true;
+                DirectCtx ctx{m.heap, 0, false};
+                WL::body(ctx, p.w, x, t, i, result);
+                nw = ctx.nw;
+                if (ctx.bad) ++cnt.c[S_ERRORS];
+            } else {
+                ++cnt.c[S_LOCK_RETRIES];
+            }
+        }
+        unsigned gm;
+        const uint32_t stamp = warp_stamp(m.clock, got && nw > 0, gm);
+        if (got) {
+            uint32_t s;
+            if (nw > 0) {
+                s = stamp - clock_begin;
+                ++cnt.c[S_COMMITS];
+            } else {
+                s = 0x80000000u | (static_cast<uint32_t>(prim::ld_acquire64(m.clock)) - clock_begin);
+                ++cnt.c[S_COMMITS_RO];
+            }
+            if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
+            prim::fence_acq_rel();
+            lk.release_locks(m);
+        }
+        if (got || (act && lk.overflow)) ++i;
+        else if (act && p.backoff_ns) __nanosleep(p.backoff_ns);
+    }
+    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
+    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
+    flush_counters(cnt, p.meta + M_STATS);
+}
+
+// ---------------------------------------------------------------------------
+// descriptor dump (generator parity test): out[(i*T + t) * wpt + k]
+// ---------------------------------------------------------------------------
+template <class WL>
+__global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
+{
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (t >= p.T) return;
+    for (uint32_t i = 0; i < p.K; ++i) {
+        uint32_t d[WL::DESCR];
+        const int n = WL::descr(p.w, gen::tx_key(p.seed, t, i), d);
+        uint32_t* o = out + (static_cast<uint64_t>(i) * p.T + t) * wpt;
+        for (int k = 0; k < wpt; ++k) o[k] = k < n ? d[k] : 0u;
+    }
+}
+
+__global__ void prepare_kernel(unsigned long long* meta, uint64_t timeout_ns)
+{
+    meta[M_CLOCK_BEGIN] = meta[M_CLOCK];
+    meta[M_DEADLINE] = globaltimer() + timeout_ns;
+    for (int k = 0; k < S_NSTATS; ++k) meta[M_STATS + k] = 0;
+    *reinterpret_cast<uint32_t*>(meta + M_ERR) = 0;
+    *reinterpret_cast<uint32_t*>(meta + M_CGL_LOCK) = 0;
+}
+
+__global__ void finish_kernel(unsigned long long* meta) { meta[M_CLOCK_END] = meta[M_CLOCK]; }
+
+// workload-defined initial heaps
+__global__ void init_heap_kernel(int workload, uint32_t* heap, uint64_t words)
+{
+    for (uint64_t k = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k < words;
+         k += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+        uint32_t v = 0;
+        if (workload == WL_RA || workload == WL_EB) v = static_cast<uint32_t>(k);
+        else if (workload == WL_BANK) v = 1000u;
+        heap[k] = v;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// host launchers
+// ---------------------------------------------------------------------------
+cudaError_t launch_prepare(unsigned long long* meta, uint64_t timeout_ns, cudaStream_t s)
+{
+    prepare_kernel<<<1, 1, 0, s>>>(meta, timeout_ns);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_finish(unsigned long long* meta, cudaStream_t s)
+{
+    finish_kernel<<<1, 1, 0, s>>>(meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, cudaStream_t s)
+{
+    if (!words) return cudaSuccess;
+    uint64_t blocks = (words + 255) / 256;
+    if (blocks > 148 * 32) blocks = 148 * 32;
+    init_heap_kernel<<<static_cast<unsigned>(blocks), 256, 0, s>>>(workload, heap, words);
+    return cudaGetLastError();
+}
+
+template <class WL>
+static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
+{
+    const uint64_t grid = (kp.T + block - 1) / block;
+    if (grid == 0) return cudaSuccess;
+    const dim3 g(static_cast<unsigned>(grid)), b(block);
+    switch (kmode) {
+    case KMODE_HV: stm_kernel<WL, MODE_HV><<<g, b, 0, s>>>(kp); break;
+    case KMODE_TBV: stm_kernel<WL, MODE_TBV><<<g, b, 0, s>>>(kp); break;
+    case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
+    case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
+    default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cudaStream_t s)
+{
+    switch (workload) {
+    case WL_RA: return kp.w.ra_kind == 1 ? launch_wl<RaIncWL>(kmode, kp, block, s) : launch_wl<RaWL>(kmode, kp, block, s);
+    case WL_BANK: return launch_wl<BankWL>(kmode, kp, block, s);
+    case WL_HT: return launch_wl<HtWL>(kmode, kp, block, s);
+    case WL_EB: return launch_wl<EbWL>(kmode, kp, block, s);
+    case WL_KM: return launch_wl<KmWL>(kmode, kp, block, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <class WL>
+static cudaError_t launch_descr_wl(const KParams& kp, uint32_t* out, int wpt, cudaStream_t s)
+{
+    const uint64_t grid = (kp.T + 255) / 256;
+    if (grid) descr_kernel<WL><<<static_cast<unsigned>(grid), 256, 0, s>>>(kp, out, wpt);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt, cudaStream_t s)
+{
+    switch (workload) {
+    case WL_RA: return kp.w.ra_kind == 1 ? launch_descr_wl<RaIncWL>(kp, out, wpt, s) : launch_descr_wl<RaWL>(kp, out, wpt, s);
+    case WL_BANK: return launch_descr_wl<BankWL>(kp, out, wpt, s);
+    case WL_HT: return launch_descr_wl<HtWL>(kp, out, wpt, s);
+    case WL_EB: return launch_descr_wl<EbWL>(kp, out, wpt, s);
+    case WL_KM: return launch_descr_wl<KmWL>(kp, out, wpt, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <class WL>
+static bool check_wl(const WlParams& w, uint64_t* fp, int* dw)
+{
+    if (!WL::check(w)) return false;
+    *fp = WL::footprint(w);
+    *dw = WL::DESCR;
+    return true;
+}
+
+bool workload_check(int workload, const WlParams& w, uint64_t* fp, int* dw)
+{
+    switch (workload) {
+    case WL_RA: return w.ra_kind == 1 ? check_wl<RaIncWL>(w, fp, dw) : check_wl<RaWL>(w, fp, dw);
+    case WL_BANK: return check_wl<BankWL>(w, fp, dw);
+    case WL_HT: return check_wl<HtWL>(w, fp, dw);
+    case WL_EB: return check_wl<EbWL>(w, fp, dw);
+    case WL_KM: return check_wl<KmWL>(w, fp, dw);
+    }
+    return false;
+}
+
+}  // namespace gstm

@@ -1,0 +1,56 @@
+// kernels.cuh -- launch parameters shared by the kernels and the C ABI layer.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "gstm/tx.cuh"
+#include "gstm/workloads.cuh"
+
+namespace gstm {
+
+// statistics counters (uint64 each), in the handle's metadata block
+enum {
+    S_COMMITS = 0, S_COMMITS_RO, S_AB_OPACITY, S_AB_PREVBV, S_AB_TBV, S_AB_COMMITVBV, S_AB_LOCK,
+    S_LOCK_RETRIES, S_POSTVAL, S_VBV, S_SPINS, S_ATTEMPTS, S_ERRORS, S_NSTATS
+};
+
+// metadata block layout (uint64 words; hot words on their own 128 B lines)
+enum {
+    M_CLOCK = 0,           // g_clock
+    M_CLOCK_BEGIN = 16,    // g_clock when the launch started (read-only in kernels)
+    M_DEADLINE = 17,       // %globaltimer deadline for the watchdog
+    M_CLOCK_END = 18,
+    M_STATS = 32,          // S_NSTATS counters
+    M_CGL_LOCK = 64,       // coarse-grain lock word (uint32)
+    M_ERR = 80,            // sticky error bits (uint32)
+    M_WORDS = 96
+};
+
+enum { ERR_LOGOVF = 1, ERR_TIMEOUT = 2, ERR_INVALID = 4 };
+
+enum { WL_RA = 0, WL_BANK = 1, WL_HT = 2, WL_EB = 3, WL_KM = 4 };
+enum { KMODE_HV = 1, KMODE_TBV = 2, KMODE_CGL = 3, KMODE_FGL = 4 };
+
+struct KParams {
+    Meta m;
+    WlParams w;
+    unsigned long long* meta;      // metadata block (M_*)
+    uint32_t* tx_stamp;            // verify mode: per tx stamp / RO|snapshot (relative)
+    uint32_t* tx_result;           // verify mode: per tx observable result
+    uint64_t T;
+    uint32_t K;
+    uint64_t seed;
+    uint32_t prelock_vbv, k_lock, backoff_ns;
+};
+
+cudaError_t launch_prepare(unsigned long long* meta, uint64_t timeout_ns, cudaStream_t s);
+cudaError_t launch_finish(unsigned long long* meta, cudaStream_t s);
+cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cudaStream_t s);
+cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt, cudaStream_t s);
+bool workload_check(int workload, const WlParams& w, uint64_t* footprint, int* descr_words);
+cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, cudaStream_t s);
+cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
+                          cudaStream_t s);
+cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s);
+int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
+
+}  // namespace gstm

@@ -1,0 +1,107 @@
+// script.cu -- scripted interleavings of several transactions on ONE device
+// thread, through the same per-lane Tx code the workload kernels use.  Used
+// for step-level parity of TXBegin / TXRead / TXWrite / TXCommit against the
+// CPU model of Algorithm 3 (tests/test_gpu_parity.py).  Output format per op
+// (4 words) matches DESIGN.md §5.3:
+//   BEGIN  [snapshot, 0, 0, 0]
+//   READ   [value, isOpaque, snapshot, postvalidation ran]
+//   WRITE  [0, 0, 0, 0]
+//   COMMIT [ok, cause, stamp, vbv runs]
+#include <cstdint>
+#include "kernels.cuh"
+
+namespace gstm {
+
+using ScriptTx = Tx<64, 64, 128>;
+constexpr int kMaxScriptTx = 8;
+
+__global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out,
+                              int n_tx)
+{
+    if (threadIdx.x || blockIdx.x) return;
+    ScriptTx tx[kMaxScriptTx];
+    for (int k = 0; k < n_ops; ++k) {
+        const uint32_t op = ops[4 * k], s = ops[4 * k + 1], a = ops[4 * k + 2], v = ops[4 * k + 3];
+        uint32_t o[4] = {0, 0, 0, 0};
+        if (static_cast<int>(s) < n_tx) {
+            ScriptTx& x = tx[s];
+            switch (op) {
+            case 0: {  // BEGIN
+                const uint32_t snap = static_cast<uint32_t>(prim::ld_acquire64(m.clock));
+                prim::fence_acq_rel();
+                x.reset_stats();
+                x.begin(snap);
+                o[0] = snap;
+                break;
+            }
+            case 1: {  // READ
+                x.n_postval = 0;
+                o[0] = x.read(m, a, mode);
+                o[1] = x.opaque ? 1u : 0u;
+                o[2] = x.snapshot;
+                o[3] = x.n_postval ? 1u : 0u;
+                break;
+            }
+            case 2:  // WRITE
+                x.write(m, a, v);
+                break;
+            case 3: {  // COMMIT
+                x.n_vbv = 0;
+                if (!x.opaque) { o[1] = C_OPACITY; break; }
+                if (x.read_only()) { o[0] = 1; o[1] = C_READONLY; break; }
+                int r = C_LOCK;
+                for (int attempt = 0; attempt < 1000 && r == C_LOCK; ++attempt) r = x.commit_acquire(m, mode, prelock != 0);
+                if (r == C_OK) {
+                    x.writeback(m);
+                    const uint32_t stamp = static_cast<uint32_t>(prim::atom_add_acq_rel64(m.clock, 1ull)) + 1u;
+                    prim::fence_acq_rel();
+                    x.release_and_update(m, stamp);
+                    o[0] = 1; o[1] = C_OK; o[2] = stamp;
+                } else {
+                    o[1] = static_cast<uint32_t>(r);
+                }
+                o[3] = x.n_vbv;
+                break;
+            }
+            default: o[0] = 0xffffffffu; break;
+            }
+        }
+        for (int j = 0; j < 4; ++j) out[4 * k + j] = o[j];
+    }
+}
+
+// lock-log parity kernel: insert entries into a register-resident (variant 0)
+// or local-memory (variant 1) lock log and dump it.
+template <int LCAP>
+__global__ void lock_log_kernel(const uint32_t* e, int n, uint32_t* out, int* out_n)
+{
+    if (threadIdx.x || blockIdx.x) return;
+    Tx<1, 1, LCAP> tx;
+    tx.begin(0);
+    for (int k = 0; k < n; ++k) tx.insert_lock(e[k]);
+    if constexpr (Tx<1, 1, LCAP>::kUnroll) {
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < tx.nl) out[k] = tx.l_ent[k];
+    } else {
+        for (int k = 0; k < tx.nl; ++k) out[k] = tx.l_ent[k];
+    }
+    *out_n = tx.overflow ? -1 : tx.nl;
+}
+
+cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
+                          cudaStream_t s)
+{
+    if (n_tx > kMaxScriptTx) return cudaErrorInvalidValue;
+    script_kernel<<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s)
+{
+    if (variant == 0) lock_log_kernel<16><<<1, 32, 0, s>>>(entries, n, out, out_n);
+    else lock_log_kernel<256><<<1, 32, 0, s>>>(entries, n, out, out_n);
+    return cudaGetLastError();
+}
+
+}  // namespace gstm

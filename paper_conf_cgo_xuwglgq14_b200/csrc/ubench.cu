@@ -1,0 +1,116 @@
+// ubench.cu -- roofline microbenchmarks for the STM hot path (SURVEY §2.3
+// K10, §8d).  The hot path is bound by L2 atomics / random L2 accesses, not
+// by streaming HBM bandwidth or tensor cores, so its roofline denominators
+// are measured here on the box with the same PTX operations the STM uses:
+//   0  random atom.or.b32 (returning)  over a table of S bytes   (lock acquire)
+//   1  same-address atom.add.u64 (returning), every thread        (global clock)
+//   2  random ld.relaxed.gpu.u32 over S bytes                     (TXRead loads)
+//   3  random st.relaxed.gpu.u32 over S bytes                     (write-back / release)
+//   4  dependent chain of random atom.or (one per thread in flight): latency
+//   5  same-address atom.add.u64 issued by one lane per warp      (aggregated clock)
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "kernels.cuh"
+
+namespace gstm {
+
+__device__ __forceinline__ uint32_t ub_hash(uint64_t a, uint64_t b)
+{
+    return static_cast<uint32_t>(gen::mix64(a * 0x9E3779B97F4A7C15ull + b) >> 32);
+}
+
+__global__ void ubench_kernel(int kind, uint32_t* table, uint32_t mask, unsigned long long* hot, uint32_t n_per_thread,
+                              uint32_t* sink)
+{
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    uint32_t acc = 0;
+    switch (kind) {
+    case 0:
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k) {
+            uint32_t old;
+            uint32_t* p = table + (ub_hash(t, k) & mask);
+            asm volatile("atom.relaxed.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(0u) : "memory");
+            acc += old;
+        }
+        break;
+    case 1:
+        for (uint32_t k = 0; k < n_per_thread; ++k) acc += static_cast<uint32_t>(prim::atom_add_relaxed64(hot, 1ull));
+        break;
+    case 2:
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k) acc += prim::ld_relaxed(table + (ub_hash(t, k) & mask));
+        break;
+    case 3:
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k) prim::st_relaxed(table + (ub_hash(t, k) & mask), k);
+        break;
+    case 4: {
+        uint32_t idx = ub_hash(t, 0) & mask;
+        for (uint32_t k = 0; k < n_per_thread; ++k) {
+            uint32_t old;
+            asm volatile("atom.relaxed.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(table + idx), "r"(0u) : "memory");
+            idx = (idx + 1 + (old & 1u) + ub_hash(t, k + 1)) & mask;
+            acc += old;
+        }
+        break;
+    }
+    case 5:
+        if (prim::lane_id() == 0)
+            for (uint32_t k = 0; k < n_per_thread; ++k) acc += static_cast<uint32_t>(prim::atom_add_relaxed64(hot, 32ull));
+        break;
+    }
+    if (acc == 0xdeadbeefu) sink[0] = acc;
+}
+
+// Runs `kind` over a table of table_bytes (power of two) with `threads`
+// threads doing n_ops in total.  Returns 0 and ops/s (for kind 5: clock
+// increments per second, i.e. 32 per atomic), or a negative error.
+int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms_out)
+{
+    if (kind < 0 || kind > 5 || threads == 0 || threads % 256 || table_bytes < 128 ||
+        (table_bytes & (table_bytes - 1)))
+        return -1;
+    const uint32_t per = static_cast<uint32_t>((n_ops + threads - 1) / threads);
+    uint32_t* table = nullptr;
+    unsigned long long* hot = nullptr;
+    uint32_t* sink = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    cudaStream_t s = nullptr;
+    int rc = 0;
+    if (cudaMalloc(&table, table_bytes) != cudaSuccess || cudaMalloc(&hot, 256) != cudaSuccess ||
+        cudaMalloc(&sink, 256) != cudaSuccess) {
+        rc = -2;
+        goto out;
+    }
+    cudaMemset(table, 0, table_bytes);
+    cudaMemset(hot, 0, 256);
+    cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    {
+        const uint32_t mask = static_cast<uint32_t>(table_bytes / 4 - 1);
+        const unsigned grid = threads / 256;
+        ubench_kernel<<<grid, 256, 0, s>>>(kind, table, mask, hot, per, sink);   // warm-up
+        cudaEventRecord(e0, s);
+        ubench_kernel<<<grid, 256, 0, s>>>(kind, table, mask, hot, per, sink);
+        cudaEventRecord(e1, s);
+        if (cudaEventSynchronize(e1) != cudaSuccess) { rc = -3; goto out; }
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        double total = static_cast<double>(per) * threads;
+        if (kind == 5) total = static_cast<double>(per) * (threads / 32) * 32.0;
+        *ops_per_s = total / (ms * 1e-3);
+        if (ms_out) *ms_out = ms;
+    }
+out:
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    if (s) cudaStreamDestroy(s);
+    cudaFree(table);
+    cudaFree(hot);
+    cudaFree(sink);
+    return rc;
+}
+
+}  // namespace gstm

@@ -1,0 +1,337 @@
+"""Thin ctypes binding of the GPU-STM C ABI (include/gstm.h).
+
+Argument marshalling only: every step of the transaction hot path runs in the
+CUDA kernels of libgstm.so.  There is no CPU fallback: if the shared library
+is missing or no CUDA device is present, calls raise GstmError.
+
+Names follow the C ABI (gstm_create, gstm_launch, gstm_stats, ...).  The
+``Gstm`` class is a convenience wrapper that owns a handle; PyTorch is used
+only for device memory (``attach_heap``) and streams (``set_stream``).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libgstm.so")
+
+WL_RA, WL_BANK, WL_HT, WL_EB, WL_KM = 0, 1, 2, 3, 4
+WORKLOADS = {"ra": WL_RA, "bank": WL_BANK, "ht": WL_HT, "eb": WL_EB, "km": WL_KM}
+MODE_AUTO, MODE_HV, MODE_TBV, MODE_CGL, MODE_FGL = 0, 1, 2, 3, 4
+MODES = {"auto": MODE_AUTO, "hv": MODE_HV, "tbv": MODE_TBV, "cgl": MODE_CGL, "fgl": MODE_FGL}
+MODE_NAMES = {v: k for k, v in MODES.items()}
+RO_FLAG = 0x80000000
+
+STATUS = {0: "GSTM_OK", -1: "GSTM_EINVAL", -2: "GSTM_ENOMEM", -3: "GSTM_ECUDA", -4: "GSTM_ELOGOVF",
+          -5: "GSTM_EOVERFLOW", -6: "GSTM_ETIMEOUT", -7: "GSTM_EBUSY", -8: "GSTM_ENODEV"}
+
+# every symbol include/gstm.h declares (checked by tests/test_abi.py)
+EXPORTS = [
+    "gstm_create", "gstm_destroy", "gstm_last_error", "gstm_api_version", "gstm_default_params",
+    "gstm_set_params", "gstm_get_params", "gstm_set_mode", "gstm_set_stream", "gstm_attach_heap",
+    "gstm_heap_words", "gstm_heap_ptr", "gstm_init_heap", "gstm_write_heap", "gstm_read_heap",
+    "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
+    "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
+    "gstm_lock_log", "gstm_ubench",
+]
+
+
+class GstmError(RuntimeError):
+    pass
+
+
+class gstm_params_t(C.Structure):
+    _fields_ = [
+        ("n_reads", C.c_uint32), ("n_writes", C.c_uint32), ("ra_kind", C.c_uint32),
+        ("n_words", C.c_uint64), ("n_accesses", C.c_uint32), ("ht_buckets", C.c_uint32),
+        ("ht_lookup_pct", C.c_uint32), ("ht_key_range", C.c_uint64), ("km_clusters", C.c_uint32),
+        ("km_dims", C.c_uint32), ("prelock_vbv", C.c_uint32), ("k_lock", C.c_uint32),
+        ("backoff_ns", C.c_uint32), ("verify", C.c_uint32), ("block_threads", C.c_uint32),
+        ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32),
+    ]
+
+
+class gstm_stats_t(C.Structure):
+    _fields_ = [
+        ("commits", C.c_uint64), ("commits_ro", C.c_uint64), ("aborts", C.c_uint64),
+        ("aborts_opacity", C.c_uint64), ("aborts_prevbv", C.c_uint64), ("aborts_tbv", C.c_uint64),
+        ("aborts_commit_vbv", C.c_uint64), ("aborts_lock", C.c_uint64), ("lock_retries", C.c_uint64),
+        ("postvalidations", C.c_uint64), ("vbv_runs", C.c_uint64), ("spins", C.c_uint64),
+        ("attempts", C.c_uint64), ("errors", C.c_uint64), ("clock_begin", C.c_uint64),
+        ("clock_end", C.c_uint64), ("elapsed_ms", C.c_double), ("tx_per_s", C.c_double),
+        ("abort_ratio", C.c_double), ("status", C.c_int32), ("mode_used", C.c_int32),
+    ]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+_lib = None
+
+
+def lib():
+    """Load libgstm.so (fails loudly if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise GstmError(f"{LIB_PATH} missing: run `python -m paper_conf_cgo_xuwglgq14_b200.build` "
+                            "(there is no CPU fallback)")
+        L = C.CDLL(LIB_PATH)
+        P, V = C.POINTER, C.c_void_p
+        u32, u64, i32 = C.c_uint32, C.c_uint64, C.c_int
+        sig = {
+            "gstm_create": (V, [u64, u32]),
+            "gstm_destroy": (None, [V]),
+            "gstm_last_error": (C.c_char_p, []),
+            "gstm_api_version": (i32, []),
+            "gstm_default_params": (i32, [i32, P(gstm_params_t)]),
+            "gstm_set_params": (i32, [V, P(gstm_params_t)]),
+            "gstm_get_params": (i32, [V, P(gstm_params_t)]),
+            "gstm_set_mode": (i32, [V, i32]),
+            "gstm_set_stream": (i32, [V, V]),
+            "gstm_attach_heap": (i32, [V, V, u64]),
+            "gstm_heap_words": (u64, [V]),
+            "gstm_heap_ptr": (V, [V]),
+            "gstm_init_heap": (i32, [V, i32]),
+            "gstm_write_heap": (i32, [V, V, u64, u64]),
+            "gstm_read_heap": (i32, [V, V, u64, u64]),
+            "gstm_read_locks": (i32, [V, V, u64]),
+            "gstm_read_clock": (i32, [V, P(u64)]),
+            "gstm_reset_meta": (i32, [V]),
+            "gstm_set_clock": (i32, [V, u64]),
+            "gstm_launch": (i32, [V, i32, u64, u32, u64]),
+            "gstm_stats": (i32, [V, P(gstm_stats_t)]),
+            "gstm_read_tx_log": (i32, [V, V, V, u64]),
+            "gstm_run_host": (i32, [V, i32, V, V, u64, u64, u32, u64, P(gstm_stats_t)]),
+            "gstm_descr_words": (i32, [V, i32]),
+            "gstm_dump_descr": (i32, [V, i32, u64, u32, u64, V, u32]),
+            "gstm_script": (i32, [V, i32, i32, V, i32, V, i32]),
+            "gstm_lock_log": (i32, [V, i32, V, i32]),
+            "gstm_ubench": (i32, [i32, u64, u64, u32, P(C.c_double), P(C.c_double)]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def last_error() -> str:
+    return lib().gstm_last_error().decode()
+
+
+def _check(rc: int, what: str) -> int:
+    if rc < 0:
+        raise GstmError(f"{what}: {STATUS.get(rc, rc)}: {last_error()}")
+    return rc
+
+
+def _ptr(a: np.ndarray):
+    assert a.flags["C_CONTIGUOUS"]
+    return a.ctypes.data_as(C.c_void_p)
+
+
+# ---- function-style API with the C names --------------------------------
+def gstm_create(heap_words: int, lock_table_bits: int):
+    h = lib().gstm_create(heap_words, lock_table_bits)
+    if not h:
+        raise GstmError(f"gstm_create: {last_error()}")
+    return h
+
+
+def gstm_destroy(h) -> None:
+    lib().gstm_destroy(h)
+
+
+def gstm_default_params(workload) -> gstm_params_t:
+    p = gstm_params_t()
+    _check(lib().gstm_default_params(_wl(workload), C.byref(p)), "gstm_default_params")
+    return p
+
+
+def gstm_set_params(h, p: gstm_params_t) -> None:
+    _check(lib().gstm_set_params(h, C.byref(p)), "gstm_set_params")
+
+
+def gstm_set_mode(h, mode) -> None:
+    _check(lib().gstm_set_mode(h, _mode(mode)), "gstm_set_mode")
+
+
+def gstm_launch(h, workload, n_threads: int, tx_per_thread: int, seed: int) -> None:
+    _check(lib().gstm_launch(h, _wl(workload), n_threads, tx_per_thread, seed), "gstm_launch")
+
+
+def gstm_stats(h, check: bool = True) -> gstm_stats_t:
+    s = gstm_stats_t()
+    rc = lib().gstm_stats(h, C.byref(s))
+    if check:
+        _check(rc, "gstm_stats")
+    return s
+
+
+def _wl(w) -> int:
+    return WORKLOADS[w] if isinstance(w, str) else int(w)
+
+
+def _mode(m) -> int:
+    return MODES[m] if isinstance(m, str) else int(m)
+
+
+class Gstm:
+    """Owning wrapper of a gstm_t handle."""
+
+    def __init__(self, heap_words: int, lock_table_bits: int):
+        self.h = gstm_create(heap_words, lock_table_bits)
+        self.bits = lock_table_bits
+        self._attached = None
+
+    def close(self) -> None:
+        if self.h:
+            gstm_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # configuration
+    def params(self) -> gstm_params_t:
+        p = gstm_params_t()
+        _check(lib().gstm_get_params(self.h, C.byref(p)), "gstm_get_params")
+        return p
+
+    def set_params(self, p: gstm_params_t | None = None, **kw) -> gstm_params_t:
+        if p is None:
+            p = self.params()
+        for k, v in kw.items():
+            if not hasattr(p, k):
+                raise KeyError(k)
+            setattr(p, k, int(v))
+        gstm_set_params(self.h, p)
+        return p
+
+    def set_workload_defaults(self, workload, **kw) -> gstm_params_t:
+        p = gstm_default_params(workload)
+        return self.set_params(p, **kw)
+
+    def set_mode(self, mode) -> None:
+        gstm_set_mode(self.h, mode)
+
+    def set_stream(self, stream) -> None:
+        """stream: a torch.cuda.Stream, an int handle, or None."""
+        ptr = getattr(stream, "cuda_stream", stream)
+        _check(lib().gstm_set_stream(self.h, C.c_void_p(ptr) if ptr else None), "gstm_set_stream")
+
+    def attach_heap(self, tensor) -> None:
+        """Use a torch CUDA tensor (int32/uint32 storage) as the heap."""
+        if tensor is None:
+            _check(lib().gstm_attach_heap(self.h, None, 0), "gstm_attach_heap")
+            self._attached = None
+            return
+        assert tensor.is_cuda and tensor.is_contiguous() and tensor.element_size() == 4
+        _check(lib().gstm_attach_heap(self.h, C.c_void_p(tensor.data_ptr()), tensor.numel()), "gstm_attach_heap")
+        self._attached = tensor
+
+    @property
+    def heap_words(self) -> int:
+        return int(lib().gstm_heap_words(self.h))
+
+    # data
+    def init_heap(self, workload) -> None:
+        _check(lib().gstm_init_heap(self.h, _wl(workload)), "gstm_init_heap")
+
+    def write_heap(self, a: np.ndarray, offset: int = 0) -> None:
+        a = np.ascontiguousarray(a, dtype=np.uint32)
+        _check(lib().gstm_write_heap(self.h, _ptr(a), offset, a.size), "gstm_write_heap")
+
+    def read_heap(self, words: int | None = None, offset: int = 0) -> np.ndarray:
+        n = self.heap_words - offset if words is None else words
+        out = np.empty(n, dtype=np.uint32)
+        _check(lib().gstm_read_heap(self.h, _ptr(out), offset, n), "gstm_read_heap")
+        return out
+
+    def read_locks(self, n: int | None = None) -> np.ndarray:
+        n = (1 << self.bits) if n is None else n
+        out = np.empty(n, dtype=np.uint32)
+        _check(lib().gstm_read_locks(self.h, _ptr(out), n), "gstm_read_locks")
+        return out
+
+    def read_clock(self) -> int:
+        c = C.c_uint64(0)
+        _check(lib().gstm_read_clock(self.h, C.byref(c)), "gstm_read_clock")
+        return c.value
+
+    def reset_meta(self) -> None:
+        _check(lib().gstm_reset_meta(self.h), "gstm_reset_meta")
+
+    def set_clock(self, value: int) -> None:
+        _check(lib().gstm_set_clock(self.h, value), "gstm_set_clock")
+
+    # hot path
+    def launch(self, workload, n_threads: int, tx_per_thread: int, seed: int) -> None:
+        gstm_launch(self.h, workload, n_threads, tx_per_thread, seed)
+
+    def stats(self, check: bool = True) -> gstm_stats_t:
+        return gstm_stats(self.h, check)
+
+    def run(self, workload, n_threads: int, tx_per_thread: int, seed: int, check: bool = True) -> gstm_stats_t:
+        self.launch(workload, n_threads, tx_per_thread, seed)
+        return self.stats(check)
+
+    def read_tx_log(self, n: int):
+        st = np.empty(n, dtype=np.uint32)
+        rs = np.empty(n, dtype=np.uint32)
+        _check(lib().gstm_read_tx_log(self.h, _ptr(st), _ptr(rs), n), "gstm_read_tx_log")
+        return st, rs
+
+    def run_host(self, workload, heap_in: np.ndarray, heap_out: np.ndarray, n_threads: int,
+                 tx_per_thread: int, seed: int) -> gstm_stats_t:
+        s = gstm_stats_t()
+        assert heap_in.dtype == np.uint32 and heap_out.dtype == np.uint32 and heap_in.size == heap_out.size
+        _check(lib().gstm_run_host(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
+                                   n_threads, tx_per_thread, seed, C.byref(s)), "gstm_run_host")
+        return s
+
+    # tests / measurement
+    def descr_words(self, workload) -> int:
+        return _check(lib().gstm_descr_words(self.h, _wl(workload)), "gstm_descr_words")
+
+    def dump_descr(self, workload, n_threads: int, tx_per_thread: int, seed: int, wpt: int | None = None):
+        wpt = self.descr_words(workload) if wpt is None else wpt
+        out = np.empty(n_threads * tx_per_thread * wpt, dtype=np.uint32)
+        _check(lib().gstm_dump_descr(self.h, _wl(workload), n_threads, tx_per_thread, seed, _ptr(out), wpt),
+               "gstm_dump_descr")
+        return out.reshape(n_threads * tx_per_thread, wpt)
+
+    def script(self, mode, ops, n_tx: int = 4, prelock_vbv: bool = True) -> np.ndarray:
+        ops = np.ascontiguousarray(np.asarray(ops, dtype=np.uint32).reshape(-1, 4))
+        out = np.zeros_like(ops)
+        _check(lib().gstm_script(self.h, _mode(mode), 1 if prelock_vbv else 0, _ptr(ops), ops.shape[0],
+                                 _ptr(out), n_tx), "gstm_script")
+        return out
+
+
+def gstm_lock_log(entries, variant: int = 0) -> np.ndarray:
+    e = np.ascontiguousarray(np.asarray(entries, dtype=np.uint32))
+    out = np.zeros(256, dtype=np.uint32)
+    n = _check(lib().gstm_lock_log(_ptr(e), e.size, _ptr(out), variant), "gstm_lock_log")
+    return out[:n].copy()
+
+
+def gstm_ubench(kind: int, table_bytes: int, n_ops: int, threads: int):
+    ops = C.c_double(0)
+    ms = C.c_double(0)
+    _check(lib().gstm_ubench(kind, table_bytes, n_ops, threads, C.byref(ops), C.byref(ms)), "gstm_ubench")
+    return ops.value, ms.value

@@ -1,0 +1,73 @@
+"""C-ABI library checks that need no GPU (-m "not gpu")."""
+import ctypes as C
+import os
+import re
+import subprocess
+
+import pytest
+
+from paper_conf_cgo_xuwglgq14_b200 import build as B
+from paper_conf_cgo_xuwglgq14_b200 import gstm as G
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def so():
+    return B.build()
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "gstm.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return set(re.findall(r"\b(gstm_[a-z_]+)\s*\(", src))
+
+
+def test_header_declares_and_library_exports_every_symbol(so):
+    declared = header_functions()
+    assert len(declared) >= 25
+    out = subprocess.check_output(["nm", "-D", "--defined-only", so], text=True)
+    exported = set(re.findall(r" T (gstm_[a-z_]+)$", out, flags=re.M))
+    assert declared == exported, (declared ^ exported)
+    assert set(G.EXPORTS) == declared
+
+
+def test_library_is_sm100a_and_self_contained(so):
+    out = subprocess.check_output(["cuobjdump", "--list-elf", so], text=True)
+    assert "sm_100a" in out
+    deps = subprocess.check_output(["ldd", so], text=True)
+    assert "libcudart" not in deps          # static cudart: nothing to resolve on the GPU box
+    sass = subprocess.check_output(["cuobjdump", "-sass", "-fun", "_ZN4gstm10stm_kernelINS_6BankWLELi2EEEvNS_7KParamsE", so],
+                                   text=True)
+    # the hot path is made of L2 atomics / strong gpu-scope accesses
+    assert "ATOMG.E.OR.STRONG.GPU" in sass and "LDG.E.STRONG.GPU" in sass
+
+
+def test_loads_and_host_only_calls(so):
+    L = G.lib()
+    assert L.gstm_api_version() == 1
+    p = G.gstm_default_params("bank")
+    assert p.n_words == 1 << 20 and p.block_threads == 256 and p.k_lock == 8
+    with pytest.raises(G.GstmError):
+        G.gstm_default_params(9)
+
+
+def test_create_fails_loudly_without_gpu(so):
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("GPU present")
+    except ImportError:
+        pass
+    with pytest.raises(G.GstmError, match="no CUDA device"):
+        G.Gstm(1024, 10)
+
+
+def test_product_path_does_not_import_the_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_cgo_xuwglgq14_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dirpath, f)).read()
+                assert not re.search(r"^\s*(import|from)\s+oracle", txt, flags=re.M), f
+                assert "oracle/" not in txt.replace("oracle/gen.c", ""), f
