@@ -153,6 +153,124 @@ def measured_peaks():
         return {"hbm_gbs": 6650.0}, "fallback (B200_PROFILING.md)"
 
 
+class SM:
+    """Stats bookkeeping, baselines and roofline arithmetic."""
+    KEYS = ["commits", "commits_ro", "aborts", "aborts_opacity", "aborts_prevbv", "aborts_tbv",
+            "aborts_commit_vbv", "aborts_lock", "lock_retries", "postvalidations", "vbv_runs", "spins",
+            "attempts", "errors"]
+
+    @staticmethod
+    def stats_vector(st):
+        import numpy as np
+        v = np.zeros(16, dtype=np.float64)
+        for i, k in enumerate(SM.KEYS):
+            v[i] = getattr(st, k)
+        v[14] = st.elapsed_ms
+        return v
+
+    @staticmethod
+    def from_vector(v):
+        d = {k: float(v[i]) for i, k in enumerate(SM.KEYS)}
+        d["lib_elapsed_ms"] = float(v[14])
+        return d
+
+    # Algorithmic memory accesses of one bank transaction (Algorithm 3 on
+    # the bank body, TBV mode, verify off), DESIGN.md §7.1.  Every access is
+    # a random 4-byte word, i.e. one 32-byte sector moved between L2 and
+    # the SM (and between HBM and L2 when not resident).
+    UPD = {"ld": 4, "atom": 2, "st": 4}      # 2 values + 2 lock words; 2 lock atom.or; 2 write-back + 2 release
+    RO = {"ld": 4, "atom": 0, "st": 0}       # skipped transfer: values + lock words
+    SECTOR = 32
+
+    @staticmethod
+    def roofline_bank(tot, t_ms, steps, peaks, peak_src, traffic=None):
+        acc_upd = sum(SM.UPD.values())
+        acc_ro = sum(SM.RO.values())
+        bytes_per_launch = (tot["commits"] * acc_upd + tot["commits_ro"] * acc_ro) * SM.SECTOR / steps
+        dur_s = t_ms * 1e-3 / steps
+        achieved = bytes_per_launch / dur_s / 1e9
+        peak = float(peaks.get("hbm_gbs", 6650.0))
+        prof = os.path.join(ROOT, "profiles", "r01_bank_ncu_full.json")
+        if traffic is None and os.path.exists(prof):
+            try:
+                traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+            except Exception:
+                traffic = None
+        return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic, "kernel": "stm_kernel<BankWL, MODE_TBV>",
+                "algorithmic_bytes_per_launch": bytes_per_launch,
+                "bytes_per_unit": {"update_tx": acc_upd * SM.SECTOR, "read_only_tx": acc_ro * SM.SECTOR},
+                "peak_source": peak_src,
+                "note": "random 4 B accesses counted as 32 B sectors; launch duration = CUDA events on the "
+                        "launching stream, averaged over the timed steps"}
+
+    @staticmethod
+    def roofline_l2_bank(G, tot, t_ms, steps):
+        """L2-atomic roofline: the same PTX operations, measured on this box by
+        gstm_ubench over a table of the heap's size (4 MiB, L2-resident)."""
+        threads = 148 * 2048
+        A = G.gstm_ubench(0, 4 << 20, 1 << 26, threads)[0]      # random atom.or.b32
+        L = G.gstm_ubench(2, 4 << 20, 1 << 26, threads)[0]      # random ld.relaxed.gpu
+        S = G.gstm_ubench(3, 4 << 20, 1 << 26, threads)[0]      # random st.relaxed.gpu
+        Cl = G.gstm_ubench(5, 256, 1 << 24, threads)[0]         # warp-aggregated clock increments
+        per = lambda m: m["ld"] / L + m["atom"] / A + m["st"] / S
+        roof_s = (tot["commits"] * (per(SM.UPD) + 1.0 / Cl) + tot["commits_ro"] * per(SM.RO)) / steps
+        dur_s = t_ms * 1e-3 / steps
+        return {"bound": "l2_atomic", "frac": roof_s / dur_s,
+                "roof_tx_per_s": (tot["commits"] + tot["commits_ro"]) / steps / roof_s,
+                "achieved_tx_per_s": (tot["commits"] + tot["commits_ro"]) / steps / dur_s,
+                "peaks_ops_per_s": {"atom_or_random_4MiB": A, "ld_relaxed_random_4MiB": L,
+                                    "st_relaxed_random_4MiB": S, "clock_increments_warp_aggregated": Cl},
+                "ops_per_update_tx": dict(SM.UPD, clock=1), "ops_per_read_only_tx": SM.RO,
+                "model": "time = sum over op classes of count / measured rate (one shared L2 request pipeline)"}
+
+    @staticmethod
+    def baselines(G, stream, accounts, bits, T, seed):
+        out = {}
+        # CGL: serialised, so its rate does not depend on the batch size; time a
+        # bounded sample (same thread count, 1 tx each, fewer threads if slow).
+        g = G.Gstm(accounts, bits)
+        g.set_workload_defaults("bank", n_words=accounts)
+        g.set_mode("cgl")
+        g.set_stream(stream)
+        g.init_heap("bank")
+        # the paper's Scheme #3 (no backoff) and test-and-test-and-set with
+        # exponential backoff; the fastest is the baseline we divide by
+        probes = {}
+        for bo in (0, 64, 256, 1024):
+            g.set_params(backoff_ns=bo)
+            probes[bo] = g.run("bank", 1 << 14, 1, seed + 11 + bo).tx_per_s
+        best = max(probes, key=probes.get)
+        g.set_params(backoff_ns=best)
+        Tc = int(min(T, max(1 << 14, probes[best] * 1.5))) // 256 * 256
+        st = g.run("bank", Tc, 1, seed + 12)
+        out["cgl"] = {"value": st.tx_per_s, "unit": UNIT, "backoff_ns": best,
+                      "probe_tx_per_s_by_backoff_ns": {str(k): v for k, v in probes.items()},
+                      "sample": f"{Tc} threads x 1 tx (serialised; rate is size-independent)",
+                      "elapsed_ms": st.elapsed_ms, "kernel": "cgl_kernel<BankWL>"}
+        g.set_params(backoff_ns=0)
+        g.set_mode("fgl")
+        g.run("bank", T, 16, seed + 13)
+        st = g.run("bank", T, 16, seed + 14)
+        out["fgl"] = {"value": st.tx_per_s, "unit": UNIT, "sample": f"{T} threads x 16 tx (full step)",
+                      "abort_ratio": 0.0, "lock_retries": st.lock_retries, "kernel": "fgl_kernel<BankWL>"}
+        g.close()
+        return out
+
+    @staticmethod
+    def cpu_baseline(accounts, T, K, seed):
+        import oracle as O
+        p = O.params("bank", n_words=accounts)
+        heap = O.init_heap(p, accounts)
+        Ts = T                     # the full step: T x K transfers
+        t0 = time.perf_counter()
+        O.serial(p, heap, Ts, K, seed)
+        dt = time.perf_counter() - t0
+        return {"value": Ts * K / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+                "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread) over one full step: "
+                          f"{Ts} threads x {K} tx = {Ts * K} bank transfers, {dt:.2f} s"}
+
+
 # ---------------------------------------------------------------------------
 # native arm
 # ---------------------------------------------------------------------------
@@ -177,10 +295,13 @@ def run_native(args):
     if world > 1:
         dist.barrier()
     from paper_conf_cgo_xuwglgq14_b200 import gstm as G
-    import stm_metrics as SM
 
     T, K = args.threads, args.tx_per_thread
-    stream = torch.cuda.current_stream()
+    # one non-default stream for everything (the library, the L2 flush, the
+    # CUDA events): torch's legacy default stream has handle 0, which the C
+    # ABI reads as "use the handle's private stream"
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
     g = G.Gstm(ACCOUNTS, BITS)
     g.set_workload_defaults("bank", n_words=ACCOUNTS)
     g.set_mode(args.mode)
@@ -195,7 +316,7 @@ def run_native(args):
         g.launch("bank", T, K, seed0 + k)
 
     for w in range(args.warmup):
-        step(-1 - w)
+        step(100000 + w)
     torch.cuda.synchronize()
 
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]

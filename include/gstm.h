@@ -83,6 +83,9 @@ typedef struct {
     uint32_t block_threads;  /* CUDA block size (multiple of 32, <= 256), default 256   */
     uint32_t spin_cap;       /* bound on lock spins / PostValidation restarts          */
     uint32_t timeout_ms;     /* device watchdog per launch, default 60000               */
+    uint32_t snapshot_reuse; /* 1: a warp that just committed starts its next txs at   */
+                             /*    the clock value after its own commits instead of   */
+                             /*    re-reading g_clock (A3.l4); default 1               */
 } gstm_params_t;
 
 typedef struct {
@@ -126,8 +129,9 @@ int gstm_default_params(int workload, gstm_params_t* out);
 int gstm_set_params(gstm_t* h, const gstm_params_t* p);
 int gstm_get_params(const gstm_t* h, gstm_params_t* out);
 int gstm_set_mode(gstm_t* h, int mode);
-/* stream: a cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream);
- * NULL restores the handle's private stream.  Borrowed, not destroyed. */
+/* stream: a cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream), or
+ * cudaStreamLegacy ((void*)1) for the legacy default stream; NULL restores
+ * the handle's private stream.  Borrowed, not destroyed. */
 int gstm_set_stream(gstm_t* h, void* stream);
 /* Use caller-owned device memory (>= words uint32, 4-byte aligned) as the
  * heap instead of the handle's own; borrowed: it must outlive the handle or

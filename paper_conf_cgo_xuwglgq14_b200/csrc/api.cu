@@ -69,6 +69,7 @@ static gstm_params_t default_params(int workload)
     p.block_threads = 256;
     p.spin_cap = 1u << 16;
     p.timeout_ms = 60000;
+    p.snapshot_reuse = 1;
     if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
     if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
     return p;
@@ -326,6 +327,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.prelock_vbv = P.prelock_vbv;
     kp.k_lock = P.k_lock;
     kp.backoff_ns = P.backoff_ns;
+    kp.snapshot_reuse = P.snapshot_reuse;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, timeout_ns, h->stream));

@@ -13,10 +13,21 @@
 //   ld_acquire        LDG.E.STRONG.GPU ; CCTL.IVALL
 //   st_relaxed        STG.E.STRONG.GPU
 //   fence_acq_rel     MEMBAR.ALL.GPU ; ERRBAR ; CGAERRBAR ; CCTL.IVALL
+//   fence_acquire     CCTL.IVALL                (waits for the prior loads)
+//   fence_release     MEMBAR.ALL.GPU ; ERRBAR ; CGAERRBAR
 //   atom_or_acquire   ATOMG.E.OR.STRONG.GPU ; CCTL.IVALL
+//   atom_add_acquire  ATOMG.E.ADD.64.STRONG.GPU ; CCTL.IVALL
 //   atom_add_acq_rel  MEMBAR.ALL.GPU ; ATOMG.E.ADD.64.STRONG.GPU ; CCTL.IVALL
 #pragma once
 #include <cstdint>
+
+// GSTM_STRICT_FENCES=1 adds the fences a purely formal reading of the PTX
+// memory model asks for on top of the ones the hardware needs (DESIGN.md
+// §6.2): a release fence after lock acquisition (A3.l79), an acq_rel clock
+// increment and a release fence before the lock-release stores.  Default 0.
+#ifndef GSTM_STRICT_FENCES
+#define GSTM_STRICT_FENCES 0
+#endif
 
 namespace gstm {
 namespace prim {
@@ -69,6 +80,30 @@ __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v)
 __device__ __forceinline__ void fence_acq_rel()
 {
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
+// Acquire fence: with the strong reads before it, forms an acquire pattern
+// (orders those reads before every later access).  SASS: CCTL.IVALL only --
+// it waits for the prior loads, no MEMBAR.  This is what A3.l12/l26 need
+// (value loads before lock-word loads).
+__device__ __forceinline__ void fence_acquire()
+{
+    asm volatile("fence.acquire.gpu;" ::: "memory");
+}
+
+// Release fence: orders every earlier access before the strong writes after
+// it (SASS: MEMBAR.ALL.GPU).  A3.l82 (write-back before the clock / lock
+// release).
+__device__ __forceinline__ void fence_release()
+{
+    asm volatile("fence.release.gpu;" ::: "memory");
+}
+
+__device__ __forceinline__ unsigned long long atom_add_acquire64(unsigned long long* p, unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.acquire.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
 }
 
 __device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t v)

@@ -36,6 +36,16 @@ struct Meta {
     uint32_t spin_cap;               // bound on the l.27-29 spin and on PostValidation restarts
 };
 
+// A3.l83 version <- Atomic_inc(g_clock) + 1, for n commits at once (the
+// lanes of a warp that commit together get base+1 .. base+n).  The acquire
+// makes every earlier commit's write-back visible to the caller, so base+n is
+// also a valid snapshot for the warp's next transactions.
+__device__ __forceinline__ unsigned long long clock_fetch_add(unsigned long long* clock, unsigned n)
+{
+    if (GSTM_STRICT_FENCES) return prim::atom_add_acq_rel64(clock, n);
+    return prim::atom_add_acquire64(clock, n);
+}
+
 // bloom-filter bit of a word (reading Q7): top 6 bits of a Fibonacci hash
 __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
 {
@@ -167,7 +177,7 @@ struct Tx {
         if (version > snapshot) snapshot = version;                // l.7
         for (uint32_t restart = 0; restart <= m.spin_cap; ++restart) {   // l.8
             if (!vbv(m)) return false;                               // l.9-11
-            prim::fence_acq_rel();                                   // l.12
+            prim::fence_acquire();                                   // l.12
             bool again = false;
             uint32_t newsnap = snapshot;
             if constexpr (kUnroll) {
@@ -221,7 +231,7 @@ struct Tx {
         if (raw_lookup(a, v)) return v;                              // l.22-23
         v = prim::ld_relaxed(m.heap + a);                            // l.24
         append_read(a, v);                                           // l.25
-        prim::fence_acq_rel();                                       // l.26
+        prim::fence_acquire();                                       // l.26
         const uint32_t vl = prim::ld_relaxed(m.locks + (a & m.lock_mask));
         check_lock(m, a, vl, mode);                                  // l.27-33
         insert_lock(((a & m.lock_mask) << 2) | 1u);                  // l.34
@@ -248,7 +258,7 @@ struct Tx {
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) append_read(a[k], v[k]);                    // l.25
-        prim::fence_acq_rel();                                       // l.26
+        prim::fence_acquire();                                       // l.26
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) vl[k] = prim::ld_relaxed(m.locks + (a[k] & m.lock_mask));
@@ -349,10 +359,17 @@ struct Tx {
             if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18
             if (!vbv(m)) { release_locks(m); return C_COMMITVBV; }   // l.76-78
         }
+        // l.79 threadfence: the acquiring atomics already returned (each
+        // atom.acquire waits for its result), so no write-back below can be
+        // performed before the locks are held; the strict build adds the
+        // formal release fence.
+        if (GSTM_STRICT_FENCES) prim::fence_release();
         return C_OK;
     }
 
-    // ---- A3.l80-81 write-back (lazy update of the redo log) --------------
+    // ---- A3.l80-82 write-back (lazy update of the redo log) + fence ------
+    // The release fence (MEMBAR.GPU) drains the write-back before the commit
+    // stamp is taken and before any lock is released (l.82).
     __device__ __forceinline__ void writeback(const Meta& m)
     {
         if constexpr (kUnroll) {
@@ -362,6 +379,7 @@ struct Tx {
         } else {
             for (int k = 0; k < nw; ++k) prim::st_relaxed(m.heap + w_addr[k], w_val[k]);
         }
+        prim::fence_release();                                       // l.82
     }
 
     // ---- A3.l56-61 ReleaseAndUpdateLocks(version) -------------------------
@@ -369,6 +387,7 @@ struct Tx {
     // the acquiring atomic returned (reading Q16: == lock - 1).
     __device__ __forceinline__ void release_and_update(const Meta& m, uint32_t version)
     {
+        if (GSTM_STRICT_FENCES) prim::fence_release();
         if constexpr (kUnroll) {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k)

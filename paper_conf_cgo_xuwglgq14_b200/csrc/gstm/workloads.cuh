@@ -75,6 +75,7 @@ __device__ __forceinline__ uint32_t lo32(uint64_t v) { return static_cast<uint32
 struct RaWL {
     static constexpr int MAXR = 8, MAXW = 8;
     static constexpr int RCAP = MAXR, WCAP = MAXW, LCAP = MAXR + MAXW, FGL_LCAP = MAXR + MAXW;
+    static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = MAXR + 2 * MAXW;
     __host__ static bool check(const WlParams& p)
     {
@@ -124,6 +125,7 @@ struct RaWL {
 struct RaIncWL {
     static constexpr int MAXR = 16;
     static constexpr int RCAP = MAXR, WCAP = MAXR, LCAP = MAXR, FGL_LCAP = MAXR;
+    static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = MAXR;
     __host__ static bool check(const WlParams& p) { return p.ra_kind == 1 && p.n_reads <= MAXR && p.n_words > 0; }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
@@ -155,6 +157,10 @@ struct RaIncWL {
 // ---- bank transfer (BASELINE configs[1]) -----------------------------------
 struct BankWL {
     static constexpr int RCAP = 2, WCAP = 2, LCAP = 4, FGL_LCAP = 2;
+#ifndef GSTM_BANK_MINB
+#define GSTM_BANK_MINB 4
+#endif
+    static constexpr int kMinBlocks = GSTM_BANK_MINB;   // 256-thread blocks per SM (register budget)
     static constexpr int DESCR = 3;
     __host__ static bool check(const WlParams& p) { return p.n_words >= 2 && p.n_words <= (1ull << 32); }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
@@ -200,6 +206,7 @@ struct BankWL {
 struct HtWL {
     static constexpr int MAXCHAIN = 24;
     static constexpr int RCAP = 1 + 2 * MAXCHAIN, WCAP = 3, LCAP = RCAP + WCAP, FGL_LCAP = 1;
+    static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = 3;
     __host__ static bool check(const WlParams& p)
     {
@@ -257,6 +264,7 @@ struct HtWL {
 struct EbWL {
     static constexpr int MAXA = 64;
     static constexpr int RCAP = MAXA / 2, WCAP = MAXA / 2, LCAP = MAXA, FGL_LCAP = MAXA;
+    static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = 2 * MAXA;
     __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
@@ -295,6 +303,7 @@ struct EbWL {
 struct KmWL {
     static constexpr int MAXD = 16;
     static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
+    static constexpr int kMinBlocks = 1;
     static constexpr int DESCR = MAXD + 1;
     __host__ static bool check(const WlParams& p) { return p.km_clusters > 0 && p.km_dims <= MAXD; }
     __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * (p.km_dims + 1); }

@@ -39,20 +39,23 @@ __device__ __forceinline__ uint32_t warp_snapshot(unsigned long long* clock)
 }
 
 // warp-aggregated commit stamp (A3.l83): lanes in `got` each receive a
-// distinct stamp; one atom.add per warp round.  The __syncwarp before the
-// atomic orders every committing lane's write-back (l.80-81) before the
-// leader's release-atomic (l.82); the one after orders the leader's acquire
-// before every lane's lock release.
-__device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool got, unsigned& gm)
+// distinct stamp; one atom.add per warp round.  Every committing lane has
+// drained its write-back with a release fence (l.82, in Tx::writeback); the
+// __syncwarp orders those fences before the leader's atomic, and the one
+// after orders the leader's acquire before every lane's lock release.  If
+// any lane committed, *next_snap = base + n is the clock value right after
+// the warp's own commits, a valid snapshot for its next transactions.
+__device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool got, unsigned& gm, uint32_t& next_snap)
 {
     __syncwarp();
     gm = __ballot_sync(FULL, got);
     unsigned long long base = 0;
     if (gm) {
         const int leader = __ffs(gm) - 1;
-        if (static_cast<int>(prim::lane_id()) == leader) base = prim::atom_add_acq_rel64(clock, __popc(gm));
+        if (static_cast<int>(prim::lane_id()) == leader) base = clock_fetch_add(clock, __popc(gm));
         base = __shfl_sync(FULL, base, leader);
         __syncwarp();
+        next_snap = static_cast<uint32_t>(base) + __popc(gm);
     }
     return static_cast<uint32_t>(base) + __popc(gm & prim::lanemask_lt()) + 1u;
 }
@@ -100,7 +103,7 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
 // or timestamp-only validation (MODE_TBV, "STM-TBV-Sorting").
 // ---------------------------------------------------------------------------
 template <class WL, int MODE>
-__global__ void __launch_bounds__(256) stm_kernel(const KParams p)
+__global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
     using TX = Tx<WL::RCAP, WL::WCAP, WL::LCAP>;
     const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -111,13 +114,16 @@ __global__ void __launch_bounds__(256) stm_kernel(const KParams p)
     Counters cnt;
     TX tx;
     tx.reset_stats();
-    uint32_t i = 0, iter = 0, backoff = 0;
-    bool timed_out = false;
+    uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0;
+    bool timed_out = false, have_snap = false;
 
     while (__any_sync(FULL, valid && i < p.K)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
         const bool act = valid && i < p.K;
-        const uint32_t snap = warp_snapshot(m.clock);                 // TXBegin l.4-5
+        // TXBegin l.4-5: a fresh clock read, or the clock value right after
+        // this warp's own last commit (p.snapshot_reuse)
+        const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
+        have_snap = false;
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
         uint32_t result = 0;
         if (act) {
@@ -148,7 +154,7 @@ __global__ void __launch_bounds__(256) stm_kernel(const KParams p)
                 const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0);
                 if (r == C_OK) {
                     got = true;
-                    tx.writeback(m);                                  // l.79-81
+                    tx.writeback(m);                                  // l.79-82
                 } else if (r == C_LOCK) {
                     ++cnt.c[S_LOCK_RETRIES];                          // l.73-74 retry next round
                     if (p.k_lock && round + 1 >= p.k_lock) { pending = false; ++cnt.c[S_AB_LOCK]; }
@@ -158,9 +164,9 @@ __global__ void __launch_bounds__(256) stm_kernel(const KParams p)
                 }
             }
             unsigned gm;
-            const uint32_t stamp = warp_stamp(m.clock, got, gm);     // l.82-83
+            const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
+            if (gm) have_snap = true;
             if (got) {
-                prim::fence_acq_rel();
                 tx.release_and_update(m, stamp);                      // l.84
                 if (p.tx_stamp) {
                     p.tx_stamp[tx_id] = stamp - clock_begin;
@@ -197,7 +203,7 @@ __global__ void __launch_bounds__(256) stm_kernel(const KParams p)
 // the CAS.  The body runs in place; the stamp is taken under the lock.
 // ---------------------------------------------------------------------------
 template <class WL>
-__global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
+__global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams p)
 {
     const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
     const bool valid = t < p.T;
@@ -205,7 +211,7 @@ __global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
     Counters cnt;
-    uint32_t i = 0, iter = 0;
+    uint32_t i = 0, iter = 0, backoff = 0;
     bool timed_out = false;
     while (__any_sync(FULL, valid && i < p.K)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
@@ -213,6 +219,7 @@ __global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
         if (act) {
             ++cnt.c[S_ATTEMPTS];
             if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
+                backoff = 0;
                 const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
                 DirectCtx ctx{p.m.heap, 0, false};
                 uint32_t result = 0;
@@ -227,12 +234,17 @@ __global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
                 }
                 if (ctx.bad) ++cnt.c[S_ERRORS];
                 if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
-                prim::fence_acq_rel();
+                prim::fence_release();
                 prim::st_relaxed(lock, 0u);                           // Scheme #3 l.15
                 ++i;
             } else {
                 ++cnt.c[S_LOCK_RETRIES];
-                if (p.backoff_ns) __nanosleep(p.backoff_ns);
+                // optional per-thread exponential backoff (test-and-test-and-set
+                // with backoff; the paper's Scheme #3 has none: backoff_ns = 0)
+                if (p.backoff_ns) {
+                    backoff = backoff ? min(backoff * 2u, 256u * p.backoff_ns) : p.backoff_ns;
+                    __nanosleep(backoff);
+                }
             }
         }
     }
@@ -249,7 +261,7 @@ __global__ void __launch_bounds__(256) cgl_kernel(const KParams p)
 // (The paper did not implement FGL; north_star asks for it.)
 // ---------------------------------------------------------------------------
 template <class WL>
-__global__ void __launch_bounds__(256) fgl_kernel(const KParams p)
+__global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams p)
 {
     using TX = Tx<1, 1, WL::FGL_LCAP>;      // only the sorted lock log is used
     const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -281,12 +293,14 @@ __global__ void __launch_bounds__(256) fgl_kernel(const KParams p)
                 WL::body(ctx, p.w, x, t, i, result);
                 nw = ctx.nw;
                 if (ctx.bad) ++cnt.c[S_ERRORS];
+                prim::fence_release();          // in-place writes before stamp and unlock
             } else {
                 ++cnt.c[S_LOCK_RETRIES];
             }
         }
         unsigned gm;
-        const uint32_t stamp = warp_stamp(m.clock, got && nw > 0, gm);
+        uint32_t unused_snap;
+        const uint32_t stamp = warp_stamp(m.clock, got && nw > 0, gm, unused_snap);
         if (got) {
             uint32_t s;
             if (nw > 0) {
@@ -297,7 +311,7 @@ __global__ void __launch_bounds__(256) fgl_kernel(const KParams p)
                 ++cnt.c[S_COMMITS_RO];
             }
             if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
-            prim::fence_acq_rel();
+            if (GSTM_STRICT_FENCES) prim::fence_release();
             lk.release_locks(m);
         }
         if (got || (act && lk.overflow)) ++i;

@@ -39,7 +39,7 @@ struct KParams {
     uint64_t T;
     uint32_t K;
     uint64_t seed;
-    uint32_t prelock_vbv, k_lock, backoff_ns;
+    uint32_t prelock_vbv, k_lock, backoff_ns, snapshot_reuse;
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, uint64_t timeout_ns, cudaStream_t s);

@@ -27,8 +27,7 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
             ScriptTx& x = tx[s];
             switch (op) {
             case 0: {  // BEGIN
-                const uint32_t snap = static_cast<uint32_t>(prim::ld_acquire64(m.clock));
-                prim::fence_acq_rel();
+                const uint32_t snap = static_cast<uint32_t>(prim::ld_acquire64(m.clock));   // l.4-5
                 x.reset_stats();
                 x.begin(snap);
                 o[0] = snap;
@@ -52,10 +51,9 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
                 int r = C_LOCK;
                 for (int attempt = 0; attempt < 1000 && r == C_LOCK; ++attempt) r = x.commit_acquire(m, mode, prelock != 0);
                 if (r == C_OK) {
-                    x.writeback(m);
-                    const uint32_t stamp = static_cast<uint32_t>(prim::atom_add_acq_rel64(m.clock, 1ull)) + 1u;
-                    prim::fence_acq_rel();
-                    x.release_and_update(m, stamp);
+                    x.writeback(m);                                                          // l.79-82
+                    const uint32_t stamp = static_cast<uint32_t>(clock_fetch_add(m.clock, 1u)) + 1u;   // l.83
+                    x.release_and_update(m, stamp);                                          // l.84
                     o[0] = 1; o[1] = C_OK; o[2] = stamp;
                 } else {
                     o[1] = static_cast<uint32_t>(r);

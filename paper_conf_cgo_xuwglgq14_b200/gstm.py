@@ -50,7 +50,7 @@ class gstm_params_t(C.Structure):
         ("ht_lookup_pct", C.c_uint32), ("ht_key_range", C.c_uint64), ("km_clusters", C.c_uint32),
         ("km_dims", C.c_uint32), ("prelock_vbv", C.c_uint32), ("k_lock", C.c_uint32),
         ("backoff_ns", C.c_uint32), ("verify", C.c_uint32), ("block_threads", C.c_uint32),
-        ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32),
+        ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32), ("snapshot_reuse", C.c_uint32),
     ]
 
 
@@ -230,9 +230,14 @@ class Gstm:
         gstm_set_mode(self.h, mode)
 
     def set_stream(self, stream) -> None:
-        """stream: a torch.cuda.Stream, an int handle, or None."""
-        ptr = getattr(stream, "cuda_stream", stream)
-        _check(lib().gstm_set_stream(self.h, C.c_void_p(ptr) if ptr else None), "gstm_set_stream")
+        """stream: a torch.cuda.Stream, an int handle, or None (the handle's
+        private stream).  torch's legacy default stream has handle 0; it is
+        passed as cudaStreamLegacy (1) so work really lands on it."""
+        if stream is None:
+            _check(lib().gstm_set_stream(self.h, None), "gstm_set_stream")
+            return
+        ptr = int(getattr(stream, "cuda_stream", stream))
+        _check(lib().gstm_set_stream(self.h, C.c_void_p(ptr if ptr else 1)), "gstm_set_stream")
 
     def attach_heap(self, tensor) -> None:
         """Use a torch CUDA tensor (int32/uint32 storage) as the heap."""

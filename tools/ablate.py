@@ -1,0 +1,98 @@
+#!/usr/bin/env python
+"""Ablation runner: time one workload under several parameter variants.
+
+    python tools/ablate.py --wl bank --variants 'mode=tbv' 'mode=hv' 'mode=tbv,snapshot_reuse=0'
+
+Each variant: warm-up launches, then --steps launches timed with CUDA events
+on a dedicated stream (L2 flushed between steps).  Prints one JSON line per
+variant (tx/s, ms/launch, abort ratio, stats).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+SHAPES = {
+    "bank": dict(words=1 << 20, bits=20, T=1 << 20, K=16, params=dict(n_words=1 << 20)),
+    "ra": dict(words=1 << 10, bits=10, T=256, K=4096, params=dict(n_reads=4, n_writes=4, n_words=1 << 10)),
+    "ra_paper": dict(words=1 << 23, bits=20, T=65536, K=16, params=dict(n_reads=4, n_writes=4, n_words=1 << 23)),
+    "ht": dict(words=(1 << 20) + 2 * (1 << 24), bits=22, T=1 << 22, K=4, params=dict()),
+    "km": dict(words=1024 * 17, bits=20, T=1 << 24, K=1, params=dict()),
+    "eb": dict(words=1 << 26, bits=22, T=1 << 18, K=16, params=dict(n_words=1 << 26, n_accesses=16)),
+}
+WL_OF = {"bank": "bank", "ra": "ra", "ra_paper": "ra", "ht": "ht", "km": "km", "eb": "eb"}
+
+
+def parse_variant(s: str) -> dict:
+    out = {}
+    for kv in filter(None, s.split(",")):
+        k, v = kv.split("=")
+        out[k] = v
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--wl", default="bank", choices=list(SHAPES))
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--T", type=int, default=None)
+    ap.add_argument("--K", type=int, default=None)
+    ap.add_argument("--bits", type=int, default=None)
+    ap.add_argument("--variants", nargs="+", default=["mode=auto"])
+    a = ap.parse_args()
+
+    import torch
+    from paper_conf_cgo_xuwglgq14_b200 import build as B
+    B.build()
+    from paper_conf_cgo_xuwglgq14_b200 import gstm as G
+
+    shp = dict(SHAPES[a.wl])
+    T = a.T or shp["T"]
+    K = a.K or shp["K"]
+    bits = a.bits if a.bits is not None else shp["bits"]
+    wl = WL_OF[a.wl]
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
+    for var in a.variants:
+        kv = parse_variant(var)
+        mode = kv.pop("mode", "auto")
+        g = G.Gstm(shp["words"], bits)
+        g.set_workload_defaults(wl, **shp["params"], **{k: int(v) for k, v in kv.items()})
+        g.set_mode(mode)
+        g.set_stream(stream)
+        g.init_heap(wl)
+        for w in range(a.warmup):
+            g.run(wl, T, K, 1000 + w)
+        tot_ms, done, ab = 0.0, 0, 0
+        agg = {}
+        for s in range(a.steps):
+            flush.fill_(float(s))
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            g.launch(wl, T, K, s)
+            e1.record(stream)
+            st = g.stats(check=False)
+            tot_ms += e0.elapsed_time(e1)
+            done += st.commits + st.commits_ro
+            ab += st.aborts
+            for k, v in st.as_dict().items():
+                if isinstance(v, int):
+                    agg[k] = agg.get(k, 0) + v
+            if st.status:
+                agg["status"] = st.status
+        line = {"wl": a.wl, "variant": var, "T": T, "K": K, "bits": bits, "mode_used": G.MODE_NAMES[st.mode_used],
+                "tx_per_s": done / (tot_ms * 1e-3), "ms_per_launch": tot_ms / a.steps,
+                "abort_ratio": ab / max(1, ab + done), "stats": agg}
+        print(json.dumps(line), flush=True)
+        g.close()
+
+
+if __name__ == "__main__":
+    main()
