@@ -86,6 +86,9 @@ typedef struct {
     uint32_t snapshot_reuse; /* 1: a warp that just committed starts its next txs at   */
                              /*    the clock value after its own commits instead of   */
                              /*    re-reading g_clock (A3.l4); default 1               */
+    uint32_t lock_pipeline;  /* 1: a transaction's first lock-acquisition round issues */
+                             /*    all atom.or at once; later rounds  */
+                             /*    are sequential in ascending id; default 0           */
 } gstm_params_t;
 
 typedef struct {
@@ -110,6 +113,7 @@ typedef struct {
     double abort_ratio;          /* aborts / (aborts + commits + commits_ro)            */
     int32_t status;              /* GSTM_OK, GSTM_ELOGOVF, GSTM_ETIMEOUT                */
     int32_t mode_used;           /* gstm_mode actually run (AUTO resolved)              */
+    int32_t clock_slot;          /* metadata line chosen for g_clock (-1: fixed word)   */
 } gstm_stats_t;
 
 /* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */
@@ -164,6 +168,14 @@ int gstm_set_clock(gstm_t* h, uint64_t value);
 int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed);
 /* Synchronises, then reports the last launch.  Returns the launch status. */
 int gstm_stats(gstm_t* h, gstm_stats_t* out);
+/* Synchronises, then reports the counters summed over every launch since
+ * gstm_reset_stats_total (or creation), so many launches can be enqueued
+ * back to back without a host sync in between.  elapsed_ms / tx_per_s use
+ * the device's %globaltimer between each launch's first and last kernel;
+ * *launches (may be NULL) = number of launches summed.  Returns GSTM_OK or
+ * the first error any of them reported. */
+int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches);
+int gstm_reset_stats_total(gstm_t* h);
 /* Verify mode (params.verify = 1): stamps[tx_id] = commit stamp - clock_begin
  * (1..C) for an update tx, or 0x80000000 | (snapshot - clock_begin) for a
  * read-only tx (linearised after that stamp); results[tx_id] = the

@@ -1,6 +1,7 @@
 // api.cu -- the C ABI (include/gstm.h) over the kernels in kernels.cu.
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <cuda_runtime.h>
 #include "../../include/gstm.h"
@@ -27,7 +28,16 @@ static void set_error(const char* fmt, ...)
         }                                                                                 \
     } while (0)
 
+static constexpr size_t kMetaBytes = 256 * 1024;  // metadata block (M_WORDS used) + g_clock candidates
+static constexpr int kClockCandidates = 64;        // candidate lines for g_clock after M_WORDS ...
+static constexpr int kClockStride = 288;           // ... 2304 B apart (crosses 256 B and 2 KiB address bits)
+
 struct gstm_handle {
+    char* block = nullptr;          // the single device allocation
+    char* block2 = nullptr;         // (layout experiments only)
+    char* meta_sep = nullptr;
+    unsigned long long* clock = nullptr;   // g_clock, on its own line inside the metadata block
+    int clock_slot = -1;
     uint32_t* own_heap = nullptr;
     uint32_t* heap = nullptr;
     uint64_t heap_words = 0, own_words = 0;
@@ -70,6 +80,7 @@ static gstm_params_t default_params(int workload)
     p.spin_cap = 1u << 16;
     p.timeout_ms = 60000;
     p.snapshot_reuse = 1;
+    p.lock_pipeline = 0;
     if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
     if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
     return p;
@@ -91,6 +102,31 @@ static WlParams wl_params(const gstm_params_t& p, uint64_t T, uint64_t K)
     w.T = T;
     w.K = K;
     return w;
+}
+
+static void fill_stats(gstm_stats_t* out, const unsigned long long* s, double ms, uint32_t err, int mode)
+{
+    memset(out, 0, sizeof(*out));
+    out->commits = s[S_COMMITS];
+    out->commits_ro = s[S_COMMITS_RO];
+    out->aborts_opacity = s[S_AB_OPACITY];
+    out->aborts_prevbv = s[S_AB_PREVBV];
+    out->aborts_tbv = s[S_AB_TBV];
+    out->aborts_commit_vbv = s[S_AB_COMMITVBV];
+    out->aborts_lock = s[S_AB_LOCK];
+    out->aborts = out->aborts_opacity + out->aborts_prevbv + out->aborts_tbv + out->aborts_commit_vbv + out->aborts_lock;
+    out->lock_retries = s[S_LOCK_RETRIES];
+    out->postvalidations = s[S_POSTVAL];
+    out->vbv_runs = s[S_VBV];
+    out->spins = s[S_SPINS];
+    out->attempts = s[S_ATTEMPTS];
+    out->errors = s[S_ERRORS];
+    out->elapsed_ms = ms;
+    const double done = static_cast<double>(out->commits + out->commits_ro);
+    out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
+    out->abort_ratio = (done + out->aborts) > 0 ? out->aborts / (done + out->aborts) : 0.0;
+    out->mode_used = mode;
+    out->status = (err & ERR_TIMEOUT) ? GSTM_ETIMEOUT : (err & (ERR_LOGOVF | ERR_INVALID)) ? GSTM_ELOGOVF : GSTM_OK;
 }
 
 extern "C" {
@@ -115,9 +151,41 @@ gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits)
     h->bits = lock_table_bits;
     h->params = default_params(GSTM_WL_RA);
     const size_t lock_bytes = sizeof(uint32_t) << lock_table_bits;
-    if (heap_words && cudaMalloc(&h->own_heap, heap_words * 4) != cudaSuccess) goto oom;
-    if (cudaMalloc(&h->locks, lock_bytes) != cudaSuccess) goto oom;
-    if (cudaMalloc(&h->meta, M_WORDS * 8) != cudaSuccess) goto oom;
+    // one allocation, fixed layout [metadata | lock table | heap]: where the
+    // hot words land must not depend on the caller's other allocations
+    const size_t heap_bytes = (heap_words * 4 + 255) & ~size_t(255);
+    {
+        const char* lay = getenv("GSTM_LAYOUT");
+        const int layout = lay ? atoi(lay) : 0;
+        const size_t P2 = 2u << 20;
+        auto up = [&](size_t x) { return (x + P2 - 1) & ~(P2 - 1); };
+        if (layout == 1 || layout == 3) {          // separate allocations
+            if (layout == 3 && cudaMalloc(&h->meta_sep, kMetaBytes) != cudaSuccess) goto oom;
+            if (cudaMalloc(&h->block, heap_bytes + 256) != cudaSuccess) goto oom;
+            if (cudaMalloc(&h->block2, lock_bytes) != cudaSuccess) goto oom;
+            if (layout == 1 && cudaMalloc(&h->meta_sep, kMetaBytes) != cudaSuccess) goto oom;
+            h->own_heap = reinterpret_cast<uint32_t*>(h->block);
+            h->locks = reinterpret_cast<uint32_t*>(h->block2);
+            h->meta = reinterpret_cast<unsigned long long*>(h->meta_sep);
+        } else if (layout == 2) {                   // [meta | locks | heap], 2 MiB aligned
+            if (cudaMalloc(&h->block, P2 + up(lock_bytes) + up(heap_bytes)) != cudaSuccess) goto oom;
+            h->meta = reinterpret_cast<unsigned long long*>(h->block);
+            h->locks = reinterpret_cast<uint32_t*>(h->block + P2);
+            h->own_heap = reinterpret_cast<uint32_t*>(h->block + P2 + up(lock_bytes));
+        } else if (layout == 4) {                   // [heap | locks | meta], 2 MiB aligned
+            if (cudaMalloc(&h->block, up(heap_bytes) + up(lock_bytes) + kMetaBytes) != cudaSuccess) goto oom;
+            h->own_heap = reinterpret_cast<uint32_t*>(h->block);
+            h->locks = reinterpret_cast<uint32_t*>(h->block + up(heap_bytes));
+            h->meta = reinterpret_cast<unsigned long long*>(h->block + up(heap_bytes) + up(lock_bytes));
+        } else {                                    // [meta | locks | heap]
+            if (cudaMalloc(&h->block, kMetaBytes + lock_bytes + heap_bytes) != cudaSuccess) goto oom;
+            h->meta = reinterpret_cast<unsigned long long*>(h->block);
+            h->locks = reinterpret_cast<uint32_t*>(h->block + kMetaBytes);
+            h->own_heap = reinterpret_cast<uint32_t*>(h->block + kMetaBytes + lock_bytes);
+        }
+        if (!heap_words) h->own_heap = nullptr;
+        h->clock = h->meta + M_CLOCK;
+    }
     if (cudaStreamCreateWithFlags(&h->own_stream, cudaStreamNonBlocking) != cudaSuccess) goto cuerr;
     if (cudaEventCreate(&h->ev0) != cudaSuccess || cudaEventCreate(&h->ev1) != cudaSuccess) goto cuerr;
     h->stream = h->own_stream;
@@ -125,8 +193,30 @@ gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits)
     h->heap_words = h->own_words = heap_words;
     if (heap_words && cudaMemsetAsync(h->own_heap, 0, heap_words * 4, h->stream) != cudaSuccess) goto cuerr;
     if (cudaMemsetAsync(h->locks, 0, lock_bytes, h->stream) != cudaSuccess) goto cuerr;
-    if (cudaMemsetAsync(h->meta, 0, M_WORDS * 8, h->stream) != cudaSuccess) goto cuerr;
+    if (cudaMemsetAsync(h->meta, 0, kMetaBytes, h->stream) != cudaSuccess) goto cuerr;
     if (cudaStreamSynchronize(h->stream) != cudaSuccess) goto cuerr;
+    {
+        // place g_clock on the candidate line with the fastest hot-spot
+        // atomic rate; GSTM_CLOCK_SLOT=k forces candidate
+        // k, GSTM_CLOCK_SLOT=-1 the fixed word M_CLOCK
+        const char* cs = getenv("GSTM_CLOCK_SLOT");
+        int slot;
+        if (cs) {
+            slot = atoi(cs);
+        } else if (lock_table_bits < 14) {
+            slot = -1;          // small tables: the hot-slice effect is negligible, skip the probe
+        } else {
+            uint64_t hw = 1;
+            while (hw * 2 <= heap_words) hw *= 2;
+            uint32_t* hp = heap_words ? h->own_heap : h->locks;
+            const uint32_t hmask = heap_words ? static_cast<uint32_t>(hw - 1) : static_cast<uint32_t>((1ull << lock_table_bits) - 1);
+            slot = clock_calibrate_mix(h->meta + M_WORDS, kClockCandidates, kClockStride, h->locks,
+                                       static_cast<uint32_t>((1ull << lock_table_bits) - 1), hp, hmask, h->stream);
+        }
+        if (slot >= kClockCandidates) slot = kClockCandidates - 1;
+        h->clock_slot = slot;
+        h->clock = slot < 0 ? h->meta + M_CLOCK : h->meta + M_WORDS + static_cast<size_t>(slot) * kClockStride;
+    }
     return h;
 oom:
     set_error("gstm_create: out of device memory (heap %llu words, 2^%u locks)", (unsigned long long)heap_words,
@@ -143,9 +233,9 @@ void gstm_destroy(gstm_t* h)
 {
     if (!h) return;
     if (h->stream) cudaStreamSynchronize(h->stream);
-    cudaFree(h->own_heap);
-    cudaFree(h->locks);
-    cudaFree(h->meta);
+    cudaFree(h->block);
+    cudaFree(h->block2);
+    cudaFree(h->meta_sep);
     cudaFree(h->tx_stamp);
     cudaFree(h->tx_result);
     if (h->ev0) cudaEventDestroy(h->ev0);
@@ -240,7 +330,7 @@ int gstm_read_clock(gstm_t* h, uint64_t* out)
 {
     if (!h || !out) { set_error("gstm_read_clock: NULL"); return GSTM_EINVAL; }
     unsigned long long c = 0;
-    CUDA_TRY(cudaMemcpyAsync(&c, h->meta + M_CLOCK, 8, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(&c, h->clock, 8, cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     *out = c;
     return GSTM_OK;
@@ -250,7 +340,7 @@ int gstm_reset_meta(gstm_t* h)
 {
     if (!h) { set_error("gstm_reset_meta: NULL"); return GSTM_EINVAL; }
     CUDA_TRY(cudaMemsetAsync(h->locks, 0, sizeof(uint32_t) << h->bits, h->stream));
-    CUDA_TRY(cudaMemsetAsync(h->meta + M_CLOCK, 0, 8, h->stream));
+    CUDA_TRY(cudaMemsetAsync(h->clock, 0, 8, h->stream));
     h->clock_bound = 0;
     return GSTM_OK;
 }
@@ -259,7 +349,7 @@ int gstm_set_clock(gstm_t* h, uint64_t value)
 {
     if (!h || value >= (1ull << 31)) { set_error("gstm_set_clock: bad argument"); return GSTM_EINVAL; }
     unsigned long long v = value;
-    CUDA_TRY(cudaMemcpyAsync(h->meta + M_CLOCK, &v, 8, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(h->clock, &v, 8, cudaMemcpyHostToDevice, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     if (value > h->clock_bound) h->clock_bound = value;
     return GSTM_OK;
@@ -315,7 +405,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.m.heap = h->heap;
     kp.m.locks = h->locks;
     kp.m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
-    kp.m.clock = h->meta + M_CLOCK;
+    kp.m.clock = h->clock;
     kp.m.spin_cap = P.spin_cap ? P.spin_cap : (1u << 16);
     kp.w = w;
     kp.meta = h->meta;
@@ -328,11 +418,12 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.k_lock = P.k_lock;
     kp.backoff_ns = P.backoff_ns;
     kp.snapshot_reuse = P.snapshot_reuse;
+    kp.lock_pipeline = P.lock_pipeline;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
-    CUDA_TRY(launch_prepare(h->meta, timeout_ns, h->stream));
+    CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));
     CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
-    CUDA_TRY(launch_finish(h->meta, h->stream));
+    CUDA_TRY(launch_finish(h->meta, h->clock, h->stream));
     CUDA_TRY(cudaEventRecord(h->ev1, h->stream));
     h->clock_bound += n_tx;
     h->launched = true;
@@ -351,33 +442,33 @@ int gstm_stats(gstm_t* h, gstm_stats_t* out)
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     float ms = 0.f;
     CUDA_TRY(cudaEventElapsedTime(&ms, h->ev0, h->ev1));
-    memset(out, 0, sizeof(*out));
-    const unsigned long long* s = m + M_STATS;
-    out->commits = s[S_COMMITS];
-    out->commits_ro = s[S_COMMITS_RO];
-    out->aborts_opacity = s[S_AB_OPACITY];
-    out->aborts_prevbv = s[S_AB_PREVBV];
-    out->aborts_tbv = s[S_AB_TBV];
-    out->aborts_commit_vbv = s[S_AB_COMMITVBV];
-    out->aborts_lock = s[S_AB_LOCK];
-    out->aborts = out->aborts_opacity + out->aborts_prevbv + out->aborts_tbv + out->aborts_commit_vbv + out->aborts_lock;
-    out->lock_retries = s[S_LOCK_RETRIES];
-    out->postvalidations = s[S_POSTVAL];
-    out->vbv_runs = s[S_VBV];
-    out->spins = s[S_SPINS];
-    out->attempts = s[S_ATTEMPTS];
-    out->errors = s[S_ERRORS];
+    fill_stats(out, m + M_STATS, ms, static_cast<uint32_t>(m[M_ERR]), h->last_mode);
+    out->clock_slot = h->clock_slot;
     out->clock_begin = m[M_CLOCK_BEGIN];
     out->clock_end = m[M_CLOCK_END];
-    out->elapsed_ms = ms;
-    const double done = static_cast<double>(out->commits + out->commits_ro);
-    out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
-    out->abort_ratio = (done + out->aborts) > 0 ? out->aborts / (done + out->aborts) : 0.0;
-    out->mode_used = h->last_mode;
-    const uint32_t err = static_cast<uint32_t>(m[M_ERR]);
-    out->status = (err & ERR_TIMEOUT) ? GSTM_ETIMEOUT : (err & (ERR_LOGOVF | ERR_INVALID)) ? GSTM_ELOGOVF : GSTM_OK;
     if (out->status) set_error("gstm_stats: launch reported %s", out->status == GSTM_ETIMEOUT ? "watchdog timeout" : "log overflow");
     return out->status;
+}
+
+int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches)
+{
+    if (!h || !out) { set_error("gstm_stats_total: NULL"); return GSTM_EINVAL; }
+    unsigned long long m[M_WORDS];
+    CUDA_TRY(cudaMemcpyAsync(m, h->meta, sizeof(m), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    fill_stats(out, m + M_TOTALS, m[M_T_NS] * 1e-6, static_cast<uint32_t>(m[M_T_ERR]), h->last_mode);
+    out->clock_slot = h->clock_slot;
+    out->clock_end = m[M_CLOCK_END];
+    if (launches) *launches = m[M_T_LAUNCHES];
+    if (out->status) set_error("gstm_stats_total: a launch reported %s", out->status == GSTM_ETIMEOUT ? "watchdog timeout" : "log overflow");
+    return out->status;
+}
+
+int gstm_reset_stats_total(gstm_t* h)
+{
+    if (!h) { set_error("gstm_reset_stats_total: NULL"); return GSTM_EINVAL; }
+    CUDA_TRY(cudaMemsetAsync(h->meta + M_TOTALS, 0, (M_T_ERR + 1 - M_TOTALS) * 8, h->stream));
+    return GSTM_OK;
 }
 
 int gstm_read_tx_log(gstm_t* h, uint32_t* stamps, uint32_t* results, uint64_t n)
@@ -463,7 +554,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
     m.heap = h->heap;
     m.locks = h->locks;
     m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
-    m.clock = h->meta + M_CLOCK;
+    m.clock = h->clock;
     m.spin_cap = 64;
     if (e == cudaSuccess) e = cudaMemcpyAsync(dops, ops, n_ops * 16, cudaMemcpyHostToDevice, h->stream);
     if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, h->stream);

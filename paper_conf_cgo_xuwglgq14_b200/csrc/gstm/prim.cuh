@@ -113,6 +113,13 @@ __device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t v)
     return old;
 }
 
+__device__ __forceinline__ uint32_t atom_or_relaxed(uint32_t* p, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.relaxed.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
 __device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, uint32_t v)
 {
     uint32_t old;

@@ -347,14 +347,52 @@ struct Tx {
         return ok;                                                   // l.52
     }
 
+    // Pipelined variant for a transaction's FIRST acquisition round (DESIGN.md
+    // §6.4): all atom.or are issued back to back (one memory round trip
+    // instead of n), then checked in ascending id.  On any conflict every
+    // lock this attempt set is restored and the next rounds fall back to the
+    // sequential sorted acquisition above, which carries the livelock-freedom
+    // argument.  Register-resident logs only.
+    __device__ __forceinline__ bool get_locks_and_tbv_pipelined(const Meta& m)
+    {
+        static_assert(kUnroll, "pipelined acquisition needs register-resident logs");
+        uint32_t vl[LCAP];
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) vl[k] = prim::atom_or_relaxed(m.locks + (l_ent[k] >> 2), 1u);   // l.45, all at once
+        prim::fence_acquire();
+        bool ok = true;
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (vl[k] & 1u)) ok = false;                  // l.46
+        if (!ok) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)                           // l.47: undo what we set
+                if (k < nl && !(vl[k] & 1u)) prim::st_relaxed(m.locks + (l_ent[k] >> 2), vl[k]);
+            n_acq = 0;
+            return false;
+        }
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) {
+                l_old[k] = vl[k];
+                if ((l_ent[k] & 1u) && (vl[k] >> 1) > snapshot) passTBV = false;   // l.49-51
+            }
+        n_acq = nl;
+        return true;
+    }
+
     // Commit steps up to the write-back (A3.l67-78).  Returns C_OK when all
     // locks are held and the read-set is valid, C_LOCK on a lock conflict
     // (nothing held; retry, l.73-74), or an abort cause (nothing held).
-    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv)
+    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
-        if (!get_locks_and_tbv(m)) return C_LOCK;                    // l.73
+        bool got;
+        if constexpr (kUnroll) got = pipelined ? get_locks_and_tbv_pipelined(m) : get_locks_and_tbv(m);
+        else got = get_locks_and_tbv(m);
+        if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18
             if (!vbv(m)) { release_locks(m); return C_COMMITVBV; }   // l.76-78

@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         for (uint32_t round = 0; __any_sync(FULL, pending); ++round) {
             bool got = false;
             if (pending) {
-                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0);
+                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, p.lock_pipeline && round == 0);
                 if (r == C_OK) {
                     got = true;
                     tx.writeback(m);                                  // l.79-82
@@ -338,16 +338,27 @@ __global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
     }
 }
 
-__global__ void prepare_kernel(unsigned long long* meta, uint64_t timeout_ns)
+__global__ void prepare_kernel(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns)
 {
-    meta[M_CLOCK_BEGIN] = meta[M_CLOCK];
-    meta[M_DEADLINE] = globaltimer() + timeout_ns;
+    const unsigned long long now = globaltimer();
+    meta[M_CLOCK_BEGIN] = *clock;
+    meta[M_DEADLINE] = now + timeout_ns;
+    meta[M_T_START] = now;
     for (int k = 0; k < S_NSTATS; ++k) meta[M_STATS + k] = 0;
     *reinterpret_cast<uint32_t*>(meta + M_ERR) = 0;
     *reinterpret_cast<uint32_t*>(meta + M_CGL_LOCK) = 0;
 }
 
-__global__ void finish_kernel(unsigned long long* meta) { meta[M_CLOCK_END] = meta[M_CLOCK]; }
+// end of a launch: record the clock and fold this launch's counters into the
+// running totals (so callers can enqueue many launches without syncing)
+__global__ void finish_kernel(unsigned long long* meta, const unsigned long long* clock)
+{
+    meta[M_CLOCK_END] = *clock;
+    for (int k = 0; k < S_NSTATS; ++k) meta[M_TOTALS + k] += meta[M_STATS + k];
+    meta[M_T_LAUNCHES] += 1;
+    meta[M_T_NS] += globaltimer() - meta[M_T_START];
+    meta[M_T_ERR] |= meta[M_ERR] & 0xffffffffull;
+}
 
 // workload-defined initial heaps
 __global__ void init_heap_kernel(int workload, uint32_t* heap, uint64_t words)
@@ -364,15 +375,15 @@ __global__ void init_heap_kernel(int workload, uint32_t* heap, uint64_t words)
 // ---------------------------------------------------------------------------
 // host launchers
 // ---------------------------------------------------------------------------
-cudaError_t launch_prepare(unsigned long long* meta, uint64_t timeout_ns, cudaStream_t s)
+cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s)
 {
-    prepare_kernel<<<1, 1, 0, s>>>(meta, timeout_ns);
+    prepare_kernel<<<1, 1, 0, s>>>(meta, clock, timeout_ns);
     return cudaGetLastError();
 }
 
-cudaError_t launch_finish(unsigned long long* meta, cudaStream_t s)
+cudaError_t launch_finish(unsigned long long* meta, const unsigned long long* clock, cudaStream_t s)
 {
-    finish_kernel<<<1, 1, 0, s>>>(meta);
+    finish_kernel<<<1, 1, 0, s>>>(meta, clock);
     return cudaGetLastError();
 }
 

@@ -21,8 +21,13 @@ enum {
     M_CLOCK_END = 18,
     M_STATS = 32,          // S_NSTATS counters
     M_CGL_LOCK = 64,       // coarse-grain lock word (uint32)
-    M_ERR = 80,            // sticky error bits (uint32)
-    M_WORDS = 96
+    M_ERR = 80,            // error bits of the last launch (uint32)
+    M_T_START = 81,        // %globaltimer at the start of the last launch
+    M_TOTALS = 96,         // S_NSTATS counters summed over launches since reset
+    M_T_LAUNCHES = 96 + S_NSTATS,      // launches since reset
+    M_T_NS = 97 + S_NSTATS,            // device ns (globaltimer) since reset
+    M_T_ERR = 98 + S_NSTATS,           // OR of the error bits since reset
+    M_WORDS = 128
 };
 
 enum { ERR_LOGOVF = 1, ERR_TIMEOUT = 2, ERR_INVALID = 4 };
@@ -39,11 +44,11 @@ struct KParams {
     uint64_t T;
     uint32_t K;
     uint64_t seed;
-    uint32_t prelock_vbv, k_lock, backoff_ns, snapshot_reuse;
+    uint32_t prelock_vbv, k_lock, backoff_ns, snapshot_reuse, lock_pipeline;
 };
 
-cudaError_t launch_prepare(unsigned long long* meta, uint64_t timeout_ns, cudaStream_t s);
-cudaError_t launch_finish(unsigned long long* meta, cudaStream_t s);
+cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);
+cudaError_t launch_finish(unsigned long long* meta, const unsigned long long* clock, cudaStream_t s);
 cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cudaStream_t s);
 cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt, cudaStream_t s);
 bool workload_check(int workload, const WlParams& w, uint64_t* footprint, int* descr_words);
@@ -52,5 +57,8 @@ cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* 
                           cudaStream_t s);
 cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s);
 int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
+int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s);
+int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_words, uint32_t* locks, uint32_t lmask,
+                        uint32_t* heap, uint32_t hmask, cudaStream_t s);
 
 }  // namespace gstm

@@ -9,6 +9,8 @@
 //   4  dependent chain of random atom.or (one per thread in flight): latency
 //   5  same-address atom.add.u64 issued by one lane per warp      (aggregated clock)
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <cuda_runtime.h>
 #include "kernels.cuh"
 
@@ -61,6 +63,107 @@ __global__ void ubench_kernel(int kind, uint32_t* table, uint32_t mask, unsigned
         break;
     }
     if (acc == 0xdeadbeefu) sink[0] = acc;
+}
+
+// Hot-spot probe for placing g_clock: every warp of a full-chip grid does
+// `n` warp-aggregated atom.add on one candidate word, like the commit path.
+__global__ void clock_probe_kernel(unsigned long long* word, uint32_t n, uint32_t* sink)
+{
+    // dependent chain: each increment waits for the previous one (latency
+    // under load, as on the commit path), not a pipelined throughput test
+    unsigned long long acc = 0;
+    if (prim::lane_id() == 0)
+        for (uint32_t k = 0; k < n; ++k) acc += prim::atom_add_acquire64(word, 8ull + (acc & 0x100000000000ull));
+    if (acc == 1ull) sink[0] = 1;
+}
+
+// Probe with the commit path's traffic mix: per warp round, 2 random
+// atom.or per lane on the lock table, 2 random loads per lane on the heap,
+// then one warp-aggregated increment of the candidate clock word.
+__global__ void clock_mix_probe_kernel(unsigned long long* word, uint32_t* locks, uint32_t lmask, uint32_t* heap,
+                                       uint32_t hmask, uint32_t n, uint32_t* sink)
+{
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    uint32_t acc = 0;
+    for (uint32_t k = 0; k < n; ++k) {
+        const uint32_t h1 = ub_hash(t, 2 * k), h2 = ub_hash(t, 2 * k + 1);
+        acc += prim::ld_relaxed(heap + ((h1 + acc) & hmask)) + prim::ld_relaxed(heap + ((h2 + acc) & hmask));
+        acc += prim::atom_or_relaxed(locks + ((h1 + acc) & lmask), 0u);
+        acc += prim::atom_or_relaxed(locks + ((h2 + acc) & lmask), 0u);
+        __syncwarp();
+        unsigned long long b = 0;
+        if (prim::lane_id() == 0) b = prim::atom_add_acquire64(word, 8ull + (acc & 0x40000000u));
+        acc += static_cast<uint32_t>(__shfl_sync(0xffffffffu, b, 0)) & 1u;
+    }
+    if (acc == 0xdeadbeefu) sink[0] = 1;
+}
+
+// Returns the index of the candidate (word = base + k*stride_words) with
+// the fastest probe, or -1 on error.  The L2 slice that owns g_clock is
+// decided by its physical address, and on B200 the per-slice load of a
+// 4 MiB table is uneven (ncu: max/avg lts requests 1.4), so the slice the
+// hot clock lands on changes commit throughput by ~25%.
+// The handle measures candidate lines once, with the commit path's mix of
+// lock-table atomics, heap loads and clock increments, and keeps the fastest.
+int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_words, uint32_t* locks, uint32_t lmask,
+                        uint32_t* heap, uint32_t hmask, cudaStream_t s)
+{
+    uint32_t* sink = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    int best = -1;
+    float best_ms = 1e30f;
+    if (cudaMalloc(&sink, 64) != cudaSuccess) return -1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    clock_mix_probe_kernel<<<148 * 8, 256, 0, s>>>(base, locks, lmask, heap, hmask, 16, sink);   // warm-up
+    for (int k = 0; k < n_candidates; ++k) {
+        unsigned long long* w = base + static_cast<size_t>(k) * stride_words;
+        cudaEventRecord(e0, s);
+        clock_mix_probe_kernel<<<148 * 8, 256, 0, s>>>(w, locks, lmask, heap, hmask, 16, sink);
+        cudaEventRecord(e1, s);
+        if (cudaEventSynchronize(e1) != cudaSuccess) { best = -1; goto out; }
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (getenv("GSTM_CALIB_VERBOSE")) fprintf(stderr, "clock candidate %d (mix): %.4f ms\n", k, ms);
+        if (ms < best_ms) { best_ms = ms; best = k; }
+    }
+    cudaMemsetAsync(base, 0, static_cast<size_t>(n_candidates) * stride_words * 8, s);
+    cudaStreamSynchronize(s);
+out:
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    return best;
+}
+
+int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s)
+{
+    uint32_t* sink = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    int best = -1;
+    float best_ms = 1e30f;
+    if (cudaMalloc(&sink, 64) != cudaSuccess) return -1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    for (int rep = 0; rep < 2; ++rep)
+        for (int k = 0; k < n_candidates; ++k) {
+            unsigned long long* w = base + static_cast<size_t>(k) * stride_words;
+            cudaEventRecord(e0, s);
+            clock_probe_kernel<<<148 * 4, 256, 0, s>>>(w, 32, sink);
+            cudaEventRecord(e1, s);
+            if (cudaEventSynchronize(e1) != cudaSuccess) { best = -1; goto out; }
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, e0, e1);
+            if (rep == 1 && getenv("GSTM_CALIB_VERBOSE")) fprintf(stderr, "clock candidate %d: %.4f ms\n", k, ms);
+            if (rep == 1 && ms < best_ms) { best_ms = ms; best = k; }
+        }
+    cudaMemsetAsync(base, 0, static_cast<size_t>(n_candidates) * stride_words * 8, s);
+    cudaStreamSynchronize(s);
+out:
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    return best;
 }
 
 // Runs `kind` over a table of table_bytes (power of two) with `threads`

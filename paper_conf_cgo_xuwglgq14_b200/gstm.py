@@ -34,6 +34,7 @@ EXPORTS = [
     "gstm_set_params", "gstm_get_params", "gstm_set_mode", "gstm_set_stream", "gstm_attach_heap",
     "gstm_heap_words", "gstm_heap_ptr", "gstm_init_heap", "gstm_write_heap", "gstm_read_heap",
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
+    "gstm_stats_total", "gstm_reset_stats_total",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
     "gstm_lock_log", "gstm_ubench",
 ]
@@ -51,6 +52,7 @@ class gstm_params_t(C.Structure):
         ("km_dims", C.c_uint32), ("prelock_vbv", C.c_uint32), ("k_lock", C.c_uint32),
         ("backoff_ns", C.c_uint32), ("verify", C.c_uint32), ("block_threads", C.c_uint32),
         ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32), ("snapshot_reuse", C.c_uint32),
+        ("lock_pipeline", C.c_uint32),
     ]
 
 
@@ -63,6 +65,7 @@ class gstm_stats_t(C.Structure):
         ("attempts", C.c_uint64), ("errors", C.c_uint64), ("clock_begin", C.c_uint64),
         ("clock_end", C.c_uint64), ("elapsed_ms", C.c_double), ("tx_per_s", C.c_double),
         ("abort_ratio", C.c_double), ("status", C.c_int32), ("mode_used", C.c_int32),
+        ("clock_slot", C.c_int32),
     ]
 
     def as_dict(self) -> dict:
@@ -104,6 +107,8 @@ def lib():
             "gstm_set_clock": (i32, [V, u64]),
             "gstm_launch": (i32, [V, i32, u64, u32, u64]),
             "gstm_stats": (i32, [V, P(gstm_stats_t)]),
+            "gstm_stats_total": (i32, [V, P(gstm_stats_t), P(u64)]),
+            "gstm_reset_stats_total": (i32, [V]),
             "gstm_read_tx_log": (i32, [V, V, V, u64]),
             "gstm_run_host": (i32, [V, i32, V, V, u64, u64, u32, u64, P(gstm_stats_t)]),
             "gstm_descr_words": (i32, [V, i32]),
@@ -290,6 +295,18 @@ class Gstm:
 
     def stats(self, check: bool = True) -> gstm_stats_t:
         return gstm_stats(self.h, check)
+
+    def stats_total(self, check: bool = True):
+        """(stats summed since reset_stats_total, number of launches)"""
+        s = gstm_stats_t()
+        n = C.c_uint64(0)
+        rc = lib().gstm_stats_total(self.h, C.byref(s), C.byref(n))
+        if check:
+            _check(rc, "gstm_stats_total")
+        return s, n.value
+
+    def reset_stats_total(self) -> None:
+        _check(lib().gstm_reset_stats_total(self.h), "gstm_reset_stats_total")
 
     def run(self, workload, n_threads: int, tx_per_thread: int, seed: int, check: bool = True) -> gstm_stats_t:
         self.launch(workload, n_threads, tx_per_thread, seed)

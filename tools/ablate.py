@@ -45,7 +45,26 @@ def main():
     ap.add_argument("--K", type=int, default=None)
     ap.add_argument("--bits", type=int, default=None)
     ap.add_argument("--variants", nargs="+", default=["mode=auto"])
+    ap.add_argument("--torch-heap", action="store_true", help="attach a torch tensor as the heap")
+    ap.add_argument("--sync", action="store_true", help="host sync after every step")
+    ap.add_argument("--seed-base", type=int, default=0)
+    ap.add_argument("--flush-first", action="store_true", help="allocate the L2-flush buffer before the handle")
+    ap.add_argument("--inproc", action="store_true",
+                    help="run all variants in this process (default: one fresh process per variant, so "
+                         "every variant sees the same allocation history)")
     a = ap.parse_args()
+
+    if len(a.variants) > 1 and not a.inproc:
+        import subprocess
+        argv = [x for x in sys.argv[1:]]
+        i = argv.index("--variants")
+        j = i + 1
+        while j < len(argv) and not argv[j].startswith("--"):
+            j += 1
+        base = argv[:i] + argv[j:]
+        for v in a.variants:
+            subprocess.run([sys.executable, os.path.abspath(__file__)] + base + ["--variants", v], check=False)
+        return
 
     import torch
     from paper_conf_cgo_xuwglgq14_b200 import build as B
@@ -59,34 +78,43 @@ def main():
     wl = WL_OF[a.wl]
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
-    flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
+    flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda") if a.flush_first else None
     for var in a.variants:
         kv = parse_variant(var)
         mode = kv.pop("mode", "auto")
+        pad_mb = int(kv.pop("pad_mb", 0))       # shift where the handle's buffers land
+        pad = torch.empty(pad_mb << 18, dtype=torch.float32, device="cuda") if pad_mb else None
         g = G.Gstm(shp["words"], bits)
+        if flush is None:
+            flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
         g.set_workload_defaults(wl, **shp["params"], **{k: int(v) for k, v in kv.items()})
         g.set_mode(mode)
         g.set_stream(stream)
+        theap = None
+        if a.torch_heap:
+            theap = torch.empty(shp["words"], dtype=torch.int32, device="cuda")
+            g.attach_heap(theap)
         g.init_heap(wl)
         for w in range(a.warmup):
             g.run(wl, T, K, 1000 + w)
-        tot_ms, done, ab = 0.0, 0, 0
-        agg = {}
+        torch.cuda.synchronize()
+        g.reset_stats_total()
+        evs = []
         for s in range(a.steps):
             flush.fill_(float(s))
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            g.launch(wl, T, K, s)
+            g.launch(wl, T, K, a.seed_base + s)
             e1.record(stream)
-            st = g.stats(check=False)
-            tot_ms += e0.elapsed_time(e1)
-            done += st.commits + st.commits_ro
-            ab += st.aborts
-            for k, v in st.as_dict().items():
-                if isinstance(v, int):
-                    agg[k] = agg.get(k, 0) + v
-            if st.status:
-                agg["status"] = st.status
+            evs.append((e0, e1))
+            if a.sync:
+                stream.synchronize()
+        torch.cuda.synchronize()
+        tot_ms = sum(e0.elapsed_time(e1) for e0, e1 in evs)
+        st, nl = g.stats_total(check=False)
+        assert nl == a.steps
+        done, ab = st.commits + st.commits_ro, st.aborts
+        agg = {k: v for k, v in st.as_dict().items() if isinstance(v, int)}
         line = {"wl": a.wl, "variant": var, "T": T, "K": K, "bits": bits, "mode_used": G.MODE_NAMES[st.mode_used],
                 "tx_per_s": done / (tot_ms * 1e-3), "ms_per_launch": tot_ms / a.steps,
                 "abort_ratio": ab / max(1, ab + done), "stats": agg}
