@@ -88,7 +88,7 @@ typedef struct {
                              /*    re-reading g_clock (A3.l4); default 1               */
     uint32_t lock_pipeline;  /* 1: a transaction's first lock-acquisition round issues */
                              /*    all atom.or at once; later rounds  */
-                             /*    are sequential in ascending id; default 0           */
+                             /*    are sequential in ascending id; default 1           */
 } gstm_params_t;
 
 typedef struct {

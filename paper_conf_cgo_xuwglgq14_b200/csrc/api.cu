@@ -80,7 +80,7 @@ static gstm_params_t default_params(int workload)
     p.spin_cap = 1u << 16;
     p.timeout_ms = 60000;
     p.snapshot_reuse = 1;
-    p.lock_pipeline = 0;
+    p.lock_pipeline = 1;
     if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
     if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
     return p;

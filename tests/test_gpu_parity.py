@@ -262,14 +262,29 @@ def test_eb_points_replay(mode, H, A, bits, T):
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("mode", ["hv", "tbv", "fgl"])
 @pytest.mark.parametrize("k_lock", [0, 1, 8])
-def test_livelock_freedom_two_words(mode, k_lock):
+@pytest.mark.parametrize("pipeline", [0, 1])
+def test_livelock_freedom_two_words(mode, k_lock, pipeline):
     """Every thread reads and writes the same 2 words in random order (the
     reverse-order pattern of P:63 and the r/w cross of P:184 inside every
-    warp); with sorted lock acquisition all 32K transactions commit."""
+    warp); with sorted lock acquisition all 4K transactions commit, with and
+    without the pipelined first acquisition round."""
     T, K = 512, 8
-    g, gp, op, init = U.make("ra", T, K, 10, mode=mode, n_reads=2, n_writes=2, n_words=2, k_lock=k_lock)
+    g, gp, op, init = U.make("ra", T, K, 10, mode=mode, n_reads=2, n_writes=2, n_words=2, k_lock=k_lock,
+                             lock_pipeline=pipeline)
     st, *_ = U.run_verified(g, "ra", op, init, T, K, 4)
     assert st.commits == T * K
+
+
+@pytest.mark.parametrize("pipeline,reuse,prelock", [(0, 0, 0), (0, 1, 1), (1, 0, 1), (1, 1, 0)])
+@pytest.mark.parametrize("mode", ["hv", "tbv"])
+def test_bank_knobs_replay(mode, pipeline, reuse, prelock):
+    """Every runtime knob of the commit path keeps the run serializable
+    (bank, 2^18 accounts, 2^18 threads x 4)."""
+    T, K = 1 << 18, 4
+    g, gp, op, init = U.make("bank", T, K, 18, mode=mode, n_words=1 << 18, lock_pipeline=pipeline,
+                             snapshot_reuse=reuse, prelock_vbv=prelock)
+    st, heap, *_ = U.run_verified(g, "bank", op, init, T, K, 13)
+    assert int(heap.astype(np.int64).sum()) == 1000 << 18
 
 
 def test_single_lock_table_degenerates_to_serial():
