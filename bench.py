@@ -53,6 +53,25 @@ def parse():
     return ap.parse_args()
 
 
+def shard_seed(rank: int) -> int:
+    """Key-partitioned bank: rank r owns its own 2^20 accounts (its own heap
+    on its own GPU) and generates shard-local transfers from this seed."""
+    return SEED + 1000003 * rank
+
+
+def reduce_over_ranks(stats_vec, balance, t_ms, wall, world, dist, device):
+    """The only collective of the run (after timing): SUM of the per-rank
+    stats vector and total balance, MAX of the timed milliseconds and wall
+    seconds.  float64 holds every count exactly (< 2^53)."""
+    import torch
+    vec = torch.tensor(list(stats_vec) + [balance], dtype=torch.float64, device=device)
+    tm = torch.tensor([t_ms, wall], dtype=torch.float64, device=device)
+    if world > 1:
+        dist.all_reduce(vec, op=dist.ReduceOp.SUM)
+        dist.all_reduce(tm, op=dist.ReduceOp.MAX)
+    return vec.cpu().numpy(), tm.cpu().tolist()
+
+
 def config(args, mode_used="tbv"):
     return {
         "workload": "bank transfer (BASELINE configs[1]): 2-account transfer tx, total-balance invariant",
@@ -180,12 +199,17 @@ class SM:
     # a random 4-byte word, i.e. one 32-byte sector moved between L2 and
     # the SM (and between HBM and L2 when not resident).
     UPD = {"ld": 4, "atom": 2, "st": 4}      # 2 values + 2 lock words; 2 lock atom.or; 2 write-back + 2 release
+    UPD_HV = {"ld": 6, "atom": 2, "st": 4}   # + the pre-lock VBV of the 2 values (A3.l71)
     RO = {"ld": 4, "atom": 0, "st": 0}       # skipped transfer: values + lock words
     SECTOR = 32
 
     @staticmethod
-    def roofline_bank(tot, t_ms, steps, peaks, peak_src, traffic=None):
-        acc_upd = sum(SM.UPD.values())
+    def upd(mode):
+        return SM.UPD_HV if mode == "hv" else SM.UPD
+
+    @staticmethod
+    def roofline_bank(tot, t_ms, steps, peaks, peak_src, mode, traffic=None):
+        acc_upd = sum(SM.upd(mode).values())
         acc_ro = sum(SM.RO.values())
         bytes_per_launch = (tot["commits"] * acc_upd + tot["commits_ro"] * acc_ro) * SM.SECTOR / steps
         dur_s = t_ms * 1e-3 / steps
@@ -198,7 +222,7 @@ class SM:
             except Exception:
                 traffic = None
         return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": "stm_kernel<BankWL, MODE_TBV>",
+                "traffic": traffic, "kernel": f"stm_kernel<BankWL, MODE_{mode.upper()}>",
                 "algorithmic_bytes_per_launch": bytes_per_launch,
                 "bytes_per_unit": {"update_tx": acc_upd * SM.SECTOR, "read_only_tx": acc_ro * SM.SECTOR},
                 "peak_source": peak_src,
@@ -206,23 +230,24 @@ class SM:
                         "launching stream, averaged over the timed steps"}
 
     @staticmethod
-    def roofline_l2_bank(G, tot, t_ms, steps):
+    def roofline_l2_bank(G, tot, t_ms, steps, mode):
         """L2-atomic roofline: the same PTX operations, measured on this box by
         gstm_ubench over a table of the heap's size (4 MiB, L2-resident)."""
+        upd = SM.upd(mode)
         threads = 148 * 2048
         A = G.gstm_ubench(0, 4 << 20, 1 << 26, threads)[0]      # random atom.or.b32
         L = G.gstm_ubench(2, 4 << 20, 1 << 26, threads)[0]      # random ld.relaxed.gpu
         S = G.gstm_ubench(3, 4 << 20, 1 << 26, threads)[0]      # random st.relaxed.gpu
         Cl = G.gstm_ubench(5, 256, 1 << 24, threads)[0]         # warp-aggregated clock increments
         per = lambda m: m["ld"] / L + m["atom"] / A + m["st"] / S
-        roof_s = (tot["commits"] * (per(SM.UPD) + 1.0 / Cl) + tot["commits_ro"] * per(SM.RO)) / steps
+        roof_s = (tot["commits"] * (per(upd) + 1.0 / Cl) + tot["commits_ro"] * per(SM.RO)) / steps
         dur_s = t_ms * 1e-3 / steps
         return {"bound": "l2_atomic", "frac": roof_s / dur_s,
                 "roof_tx_per_s": (tot["commits"] + tot["commits_ro"]) / steps / roof_s,
                 "achieved_tx_per_s": (tot["commits"] + tot["commits_ro"]) / steps / dur_s,
                 "peaks_ops_per_s": {"atom_or_random_4MiB": A, "ld_relaxed_random_4MiB": L,
                                     "st_relaxed_random_4MiB": S, "clock_increments_warp_aggregated": Cl},
-                "ops_per_update_tx": dict(SM.UPD, clock=1), "ops_per_read_only_tx": SM.RO,
+                "ops_per_update_tx": dict(upd, clock=1), "ops_per_read_only_tx": SM.RO,
                 "model": "time = sum over op classes of count / measured rate (one shared L2 request pipeline)"}
 
     @staticmethod
@@ -350,7 +375,7 @@ def run_native(args):
     g.attach_heap(heap)
     g.init_heap("bank")
     flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)    # 256 MiB > 126 MB L2
-    seed0 = SEED + 1000003 * rank
+    seed0 = shard_seed(rank)
 
     def step(k):
         g.launch("bank", T, K, seed0 + k)
@@ -389,13 +414,7 @@ def run_native(args):
 
     # NCCL: one all-reduce of the stats and invariants (SUM), one of the time (MAX)
     bal = float(heap.to(torch.int64).sum().item())
-    vec = torch.tensor(list(agg) + [bal], dtype=torch.float64, device=dev)
-    tmax = torch.tensor([t_ms, wall], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(vec, op=dist.ReduceOp.SUM)
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-    vec = vec.cpu().numpy()
-    t_ms, wall = tmax.cpu().tolist()
+    vec, (t_ms, wall) = reduce_over_ranks(agg, bal, t_ms, wall, world, dist, dev)
     tot = SM.from_vector(vec[:16])
     balance_ok = int(vec[16]) == world * ACCOUNTS * 1000
 
@@ -431,8 +450,8 @@ def run_native(args):
                                            [m for m in ("auto", "tbv", "hv", "fgl") if m != args.mode])
         # roofline of the dominant kernel (stm_kernel<BankWL, TBV>)
         peaks, peak_src = measured_peaks()
-        extra["roofline"] = SM.roofline_bank(tot, t_ms, args.steps, peaks, peak_src)
-        extra["roofline_l2"] = SM.roofline_l2_bank(G, tot, t_ms, args.steps)
+        extra["roofline"] = SM.roofline_bank(tot, t_ms, args.steps, peaks, peak_src, mode_used)
+        extra["roofline_l2"] = SM.roofline_l2_bank(G, tot, t_ms, args.steps, mode_used)
         if world == 1 and not args.no_cpu:
             extra["cpu_baseline"] = SM.cpu_baseline(ACCOUNTS, T, K, SEED)
 

@@ -1,0 +1,82 @@
+"""World-size-2 gloo tests of the multi-GPU host logic (-m "not gpu").
+
+bench.py at N > 1 runs a key-partitioned bank: every rank owns its own
+accounts and its own seed (shard-local transactions, no data-path
+collective), then ONE all-reduce sums the stats and the balance invariant
+and takes the max of the timings.  Here each rank stands in for its GPU with
+the CPU oracle's serial run of its shard and calls the same reduction
+function bench.py uses.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    accounts, T, K = 1024, 64, 4
+    p = O.params("bank", n_words=accounts)
+    heap = O.init_heap(p, accounts)
+    res, upd = O.serial(p, heap, T, K, bench.shard_seed(rank))
+    vec = np.zeros(16)
+    vec[0] = upd.sum()
+    vec[1] = (~upd).sum()
+    t_ms = 10.0 + rank
+    out, (tmax, wall) = bench.reduce_over_ranks(vec, float(heap.astype(np.int64).sum()), t_ms, 0.5 * rank,
+                                                world, dist, torch.device("cpu"))
+    q.put((rank, int(vec[0]), int(vec[1]), out.tolist(), tmax, wall, heap.tobytes()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_two_rank_reduction_gloo():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    got.sort()
+    commits = sum(g[1] for g in got)
+    ro = sum(g[2] for g in got)
+    for rank, c, r, out, tmax, wall, _ in got:
+        assert out[0] == commits and out[1] == ro                # SUM over shards
+        assert out[16] == world * 1024 * 1000                    # global balance invariant
+        assert tmax == 11.0 and wall == 0.5                      # MAX over ranks
+    assert commits + ro == world * 64 * 4
+    # shards use different seeds, so their transactions (and heaps) differ
+    assert got[0][6] != got[1][6]
+
+
+def test_shard_seeds_are_distinct():
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    seeds = {bench.shard_seed(r) for r in range(8)}
+    assert len(seeds) == 8
