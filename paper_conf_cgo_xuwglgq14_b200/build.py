@@ -51,6 +51,8 @@ def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = Fals
         obj = os.path.join(objdir, src.replace(".cu", ".o"))
         cmd = [nvcc()] + ARCH + FLAGS + ["-I", os.path.join(ROOT, "include"), "-I", CSRC, "-c",
                                          os.path.join(CSRC, src), "-o", obj]
+        # e.g. GSTM_DEFINES="-DGSTM_STRICT_FENCES=1" (ablation builds; use --force)
+        cmd += os.environ.get("GSTM_DEFINES", "").split()
         if ptxas_verbose:
             cmd += ["-Xptxas", "-v"]
         if verbose:
