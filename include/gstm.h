@@ -89,6 +89,10 @@ typedef struct {
     uint32_t lock_pipeline;  /* 1: a transaction's first lock-acquisition round issues */
                              /*    all atom.or at once; later rounds  */
                              /*    are sequential in ascending id; default 1           */
+    uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
+                             /*    n_threads STM threads (grid-stride); 0 = no cap     */
+    uint32_t lock_shift;     /* stripe size 2^lock_shift words per version lock      */
+                             /*    (lock = (word >> shift) mod 2^bits); default 0     */
 } gstm_params_t;
 
 typedef struct {

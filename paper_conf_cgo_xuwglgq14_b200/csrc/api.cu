@@ -407,6 +407,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
     kp.m.clock = h->clock;
     kp.m.spin_cap = P.spin_cap ? P.spin_cap : (1u << 16);
+    kp.m.lock_shift = P.lock_shift;
     kp.w = w;
     kp.meta = h->meta;
     kp.tx_stamp = P.verify ? h->tx_stamp : nullptr;
@@ -419,6 +420,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.backoff_ns = P.backoff_ns;
     kp.snapshot_reuse = P.snapshot_reuse;
     kp.lock_pipeline = P.lock_pipeline;
+    kp.max_threads = P.max_threads;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));
@@ -556,6 +558,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
     m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
     m.clock = h->clock;
     m.spin_cap = 64;
+    m.lock_shift = 0;
     if (e == cudaSuccess) e = cudaMemcpyAsync(dops, ops, n_ops * 16, cudaMemcpyHostToDevice, h->stream);
     if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, h->stream);
     if (e == cudaSuccess) e = cudaMemcpyAsync(out, dout, n_ops * 16, cudaMemcpyDeviceToHost, h->stream);

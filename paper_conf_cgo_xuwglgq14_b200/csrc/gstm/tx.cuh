@@ -31,9 +31,14 @@ enum { C_OK = 0, C_OPACITY = 1, C_PREVBV = 2, C_TBV = 3, C_COMMITVBV = 4, C_READ
 struct Meta {
     uint32_t* heap;
     uint32_t* locks;
-    uint32_t lock_mask;              // 2^bits - 1: hash(word) = word & mask (Q2)
+    uint32_t lock_mask;              // 2^bits - 1
+    uint32_t lock_shift;             // stripe = 2^shift words (0: one lock per word)
     unsigned long long* clock;       // g_clock
     uint32_t spin_cap;               // bound on the l.27-29 spin and on PostValidation restarts
+
+    // hash(addr) of P:113 (reading Q2): the version lock of a memory stripe
+    // of 2^lock_shift consecutive words, modulo the table size
+    __device__ __forceinline__ uint32_t lock_of(uint32_t w) const { return (w >> lock_shift) & lock_mask; }
 };
 
 // A3.l83 version <- Atomic_inc(g_clock) + 1, for n commits at once (the
@@ -52,9 +57,11 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
     return 1ull << ((static_cast<unsigned long long>(w) * 0x9E3779B97F4A7C15ull) >> 58);
 }
 
-template <int RCAP, int WCAP, int LCAP>
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false>
 struct Tx {
-    static constexpr bool kUnroll = (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
+    // register-resident (unrolled) logs for small capacities unless the
+    // workload asks for local memory (LOCAL: fewer registers, more warps)
+    static constexpr bool kUnroll = !LOCAL && (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
     static constexpr int kRcap = RCAP, kWcap = WCAP, kLcap = LCAP;
 
     uint32_t r_addr[RCAP], r_val[RCAP];   // read-set  <addr,val>
@@ -184,7 +191,7 @@ struct Tx {
                 uint32_t vl[RCAP];
 #pragma unroll
                 for (int k = 0; k < RCAP; ++k)                       // l.13
-                    if (k < nr) vl[k] = prim::ld_relaxed(m.locks + (r_addr[k] & m.lock_mask)); // l.14
+                    if (k < nr) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(r_addr[k])); // l.14
 #pragma unroll
                 for (int k = 0; k < RCAP; ++k)
                     if (k < nr && ((vl[k] & 1u) || (vl[k] >> 1) > snapshot)) {   // l.15-17
@@ -193,7 +200,7 @@ struct Tx {
                     }
             } else {
                 for (int k = 0; k < nr; ++k) {
-                    const uint32_t vl = prim::ld_relaxed(m.locks + (r_addr[k] & m.lock_mask));
+                    const uint32_t vl = prim::ld_relaxed(m.locks + m.lock_of(r_addr[k]));
                     if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
                 }
             }
@@ -211,7 +218,7 @@ struct Tx {
         while (vl & 1u) {                                            // l.29
             if (++spins > m.spin_cap) { opaque = false; break; }
             __nanosleep(32);
-            vl = prim::ld_relaxed(m.locks + (a & m.lock_mask));      // l.28
+            vl = prim::ld_relaxed(m.locks + m.lock_of(a));      // l.28
         }
         n_spin += spins;
         const uint32_t version = vl >> 1;                            // l.30
@@ -232,9 +239,9 @@ struct Tx {
         v = prim::ld_relaxed(m.heap + a);                            // l.24
         append_read(a, v);                                           // l.25
         prim::fence_acquire();                                       // l.26
-        const uint32_t vl = prim::ld_relaxed(m.locks + (a & m.lock_mask));
+        const uint32_t vl = prim::ld_relaxed(m.locks + m.lock_of(a));
         check_lock(m, a, vl, mode);                                  // l.27-33
-        insert_lock(((a & m.lock_mask) << 2) | 1u);                  // l.34
+        insert_lock((m.lock_of(a) << 2) | 1u);                  // l.34
         return v;                                                    // l.35
     }
 
@@ -261,12 +268,36 @@ struct Tx {
         prim::fence_acquire();                                       // l.26
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (need[k]) vl[k] = prim::ld_relaxed(m.locks + (a[k] & m.lock_mask));
+            if (need[k]) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(a[k]));
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) {
                 check_lock(m, a[k], vl[k], mode);                    // l.27-33
-                insert_lock(((a[k] & m.lock_mask) << 2) | 1u);       // l.34
+                insert_lock((m.lock_of(a[k]) << 2) | 1u);       // l.34
+            }
+    }
+
+    // Batched TXRead of n words (n only known at run time; arrays in local
+    // memory): the value loads go out 8 at a time, one acquire fence orders
+    // them before the lock-word loads, then l.27-34 per word.  skip[k] marks
+    // reads the caller serves from its own write-set later.
+    __device__ __forceinline__ void read_many(const Meta& m, const uint32_t* a, uint32_t* v, const bool* skip, int n,
+                                              int mode)
+    {
+        uint32_t vl[kRcap];
+#pragma unroll 8
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) v[k] = prim::ld_relaxed(m.heap + a[k]);   // l.24
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) append_read(a[k], v[k]);                    // l.25
+        prim::fence_acquire();                                        // l.26
+#pragma unroll 8
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(a[k]));
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) {
+                check_lock(m, a[k], vl[k], mode);                     // l.27-33
+                insert_lock((m.lock_of(a[k]) << 2) | 1u);             // l.34
             }
     }
 
@@ -296,7 +327,7 @@ struct Tx {
             ++nw;
             bloom |= bloom_bit(a);
         }
-        insert_lock(((a & m.lock_mask) << 2) | 2u);                  // l.38
+        insert_lock((m.lock_of(a) << 2) | 2u);                  // l.38
     }
 
     // ---- A3.l53-55 ReleaseLocks: restore the words this attempt acquired --

@@ -39,6 +39,10 @@ struct StmCtx {
     {
         tx.template read_batch<N>(m, a, v, n, mode);
     }
+    __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
+    {
+        tx.read_many(m, a, v, skip, n, mode);
+    }
     __device__ __forceinline__ void write(uint32_t a, uint32_t v) { tx.write(m, a, v); }
     __device__ __forceinline__ bool ok() const { return tx.opaque; }
     // the body found its own view inconsistent (e.g. a chain pointer out of
@@ -60,6 +64,11 @@ struct DirectCtx {
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (k < n) v[k] = prim::ld_relaxed(heap + a[k]);
+    }
+    __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
+    {
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) v[k] = prim::ld_relaxed(heap + a[k]);
     }
     __device__ __forceinline__ void write(uint32_t a, uint32_t v) { prim::st_relaxed(heap + a, v); ++nw; }
     __device__ __forceinline__ bool ok() const { return !bad; }
@@ -268,18 +277,33 @@ struct EbWL {
     static constexpr int DESCR = 2 * MAXA;
     __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
+    // All addresses are known up front, so the reads that are not
+    // read-after-write are issued as one batch (Tx::read_many, DESIGN.md
+    // §6.3); a read of a word this transaction wrote earlier is served from
+    // the write-set in program order (A3.l22-23).
     template <class Ctx>
     __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
     {
         const uint32_t A = p.n_accesses;
+        uint32_t addr[MAXA], ra[MAXA / 2], rv[MAXA / 2];
+        bool raw[MAXA / 2];
+        for (uint32_t j = 0; j < A; ++j) addr[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        const uint32_t R = (A + 1) / 2;
+        for (uint32_t r = 0; r < R; ++r) {
+            ra[r] = addr[2 * r];
+            bool hit = false;
+            for (uint32_t k = 1; k < 2 * r; k += 2) hit |= (addr[k] == ra[r]);
+            raw[r] = hit;
+        }
+        c.read_many(ra, rv, raw, static_cast<int>(R));
+        if (!c.ok()) return;
         uint32_t acc = 0;
         for (uint32_t j = 0; j < A; ++j) {
-            const uint32_t a = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
             if ((j & 1u) == 0) {
-                acc += c.read(a);
+                acc += raw[j / 2] ? c.read(addr[j]) : rv[j / 2];
                 if (!c.ok()) return;
             } else {
-                c.write(a, acc + lo32(gen::draw(x, A + j)));
+                c.write(addr[j], acc + lo32(gen::draw(x, A + j)));
             }
         }
         result = acc;
@@ -303,7 +327,11 @@ struct EbWL {
 struct KmWL {
     static constexpr int MAXD = 16;
     static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
-    static constexpr int kMinBlocks = 1;
+#ifndef GSTM_KM_LOCAL_LOGS
+#define GSTM_KM_LOCAL_LOGS 1     // local-memory logs: 122 vs 254 registers, 2.5x faster
+#endif
+    static constexpr bool kLocalLogs = GSTM_KM_LOCAL_LOGS;
+    static constexpr int kMinBlocks = GSTM_KM_LOCAL_LOGS ? 2 : 1;
     static constexpr int DESCR = MAXD + 1;
     __host__ static bool check(const WlParams& p) { return p.km_clusters > 0 && p.km_dims <= MAXD; }
     __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * (p.km_dims + 1); }

@@ -13,12 +13,20 @@
 //   * the committing lanes of a round take their commit stamps with ONE
 //     atomic on the global clock (A3.l83 aggregated over the warp);
 //   * the snapshot (A3.l4) is read once per warp and broadcast.
+#include <algorithm>
 #include <cstdint>
+#include <type_traits>
 #include "kernels.cuh"
 
 namespace gstm {
 
 using prim::FULL;
+
+// WL::kLocalLogs (optional): keep the logs in local memory even when small
+template <class WL, class = void>
+struct LocalLogs { static constexpr bool value = false; };
+template <class WL>
+struct LocalLogs<WL, std::void_t<decltype(WL::kLocalLogs)>> { static constexpr bool value = WL::kLocalLogs; };
 
 __device__ __forceinline__ unsigned long long globaltimer()
 {
@@ -105,9 +113,12 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
 template <class WL, int MODE>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
-    using TX = Tx<WL::RCAP, WL::WCAP, WL::LCAP>;
-    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    const bool valid = t < p.T;
+    using TX = Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>;
+    // physical thread -> logical STM threads t, t + P, t + 2P, ... (P = the
+    // grid's threads; P < T when the launch caps concurrency, p.max_threads)
+    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (p.K == 0) t = p.T;
     const Meta m = p.m;
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
@@ -115,11 +126,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     TX tx;
     tx.reset_stats();
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0;
-    bool timed_out = false, have_snap = false;
+    bool timed_out = false, have_snap = false, lock_aborted = false;
 
-    while (__any_sync(FULL, valid && i < p.K)) {
+    while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = valid && i < p.K;
+        const bool act = t < p.T;
         // TXBegin l.4-5: a fresh clock read, or the clock value right after
         // this warp's own last commit (p.snapshot_reuse)
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
@@ -151,13 +162,21 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         for (uint32_t round = 0; __any_sync(FULL, pending); ++round) {
             bool got = false;
             if (pending) {
-                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, p.lock_pipeline && round == 0);
+                // the pipelined round (§6.4) only for a transaction's first
+                // round of an execution that never lost its locks before, so
+                // every retry uses the sequential sorted acquisition
+                const bool pipelined = p.lock_pipeline && round == 0 && !lock_aborted;
+                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
                 if (r == C_OK) {
                     got = true;
                     tx.writeback(m);                                  // l.79-82
                 } else if (r == C_LOCK) {
                     ++cnt.c[S_LOCK_RETRIES];                          // l.73-74 retry next round
-                    if (p.k_lock && round + 1 >= p.k_lock) { pending = false; ++cnt.c[S_AB_LOCK]; }
+                    if (p.k_lock && round + 1 >= p.k_lock) {
+                        pending = false;
+                        lock_aborted = true;
+                        ++cnt.c[S_AB_LOCK];
+                    }
                 } else {
                     pending = false;
                     ++cnt.c[r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV)];
@@ -178,8 +197,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             }
         }
         if (done || skip) {
-            ++i;
+            if (++i >= p.K) { i = 0; t += P; }
             backoff = 0;
+            lock_aborted = false;
         } else if (p.backoff_ns) {
             // warp-uniform exponential backoff after an abort (all lanes sleep
             // together: per-lane delays cannot work under SIMT)
@@ -205,17 +225,18 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
 template <class WL>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams p)
 {
-    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    const bool valid = t < p.T;
+    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (p.K == 0) t = p.T;
     uint32_t* lock = reinterpret_cast<uint32_t*>(p.meta + M_CGL_LOCK);
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
     Counters cnt;
     uint32_t i = 0, iter = 0, backoff = 0;
     bool timed_out = false;
-    while (__any_sync(FULL, valid && i < p.K)) {
+    while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = valid && i < p.K;
+        const bool act = t < p.T;
         if (act) {
             ++cnt.c[S_ATTEMPTS];
             if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
@@ -236,7 +257,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams 
                 if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
                 prim::fence_release();
                 prim::st_relaxed(lock, 0u);                           // Scheme #3 l.15
-                ++i;
+                if (++i >= p.K) { i = 0; t += P; }
             } else {
                 ++cnt.c[S_LOCK_RETRIES];
                 // optional per-thread exponential backoff (test-and-test-and-set
@@ -264,8 +285,9 @@ template <class WL>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams p)
 {
     using TX = Tx<1, 1, WL::FGL_LCAP>;      // only the sorted lock log is used
-    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    const bool valid = t < p.T;
+    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (p.K == 0) t = p.T;
     const Meta m = p.m;
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
@@ -273,9 +295,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
     TX lk;
     uint32_t i = 0, iter = 0;
     bool timed_out = false;
-    while (__any_sync(FULL, valid && i < p.K)) {
+    while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = valid && i < p.K;
+        const bool act = t < p.T;
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
         bool got = false;
         int nw = 0;
@@ -284,7 +306,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
             ++cnt.c[S_ATTEMPTS];
             const uint64_t x = gen::tx_key(p.seed, t, i);
             lk.begin(0);
-            WL::fgl_words(p.w, x, t, i, [&](uint32_t w) { lk.insert_lock(((w & m.lock_mask) << 2) | 2u); });
+            WL::fgl_words(p.w, x, t, i, [&](uint32_t w) { lk.insert_lock((m.lock_of(w) << 2) | 2u); });
             if (lk.overflow) {
                 ++cnt.c[S_ERRORS];
             } else if (lk.get_locks_and_tbv(m)) {
@@ -314,8 +336,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
             if (GSTM_STRICT_FENCES) prim::fence_release();
             lk.release_locks(m);
         }
-        if (got || (act && lk.overflow)) ++i;
-        else if (act && p.backoff_ns) __nanosleep(p.backoff_ns);
+        if (got || (act && lk.overflow)) {
+            if (++i >= p.K) { i = 0; t += P; }
+        } else if (act && p.backoff_ns) {
+            __nanosleep(p.backoff_ns);
+        }
     }
     if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
     if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
@@ -399,7 +424,8 @@ cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, cudaS
 template <class WL>
 static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
 {
-    const uint64_t grid = (kp.T + block - 1) / block;
+    uint64_t grid = (kp.T + block - 1) / block;
+    if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
     if (grid == 0) return cudaSuccess;
     const dim3 g(static_cast<unsigned>(grid)), b(block);
     switch (kmode) {

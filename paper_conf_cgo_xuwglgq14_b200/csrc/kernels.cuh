@@ -45,6 +45,7 @@ struct KParams {
     uint32_t K;
     uint64_t seed;
     uint32_t prelock_vbv, k_lock, backoff_ns, snapshot_reuse, lock_pipeline;
+    uint64_t max_threads;          // 0: one CUDA thread per STM thread; else cap (grid-stride)
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);

@@ -52,7 +52,7 @@ class gstm_params_t(C.Structure):
         ("km_dims", C.c_uint32), ("prelock_vbv", C.c_uint32), ("k_lock", C.c_uint32),
         ("backoff_ns", C.c_uint32), ("verify", C.c_uint32), ("block_threads", C.c_uint32),
         ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32), ("snapshot_reuse", C.c_uint32),
-        ("lock_pipeline", C.c_uint32),
+        ("lock_pipeline", C.c_uint32), ("max_threads", C.c_uint32), ("lock_shift", C.c_uint32),
     ]
 
 

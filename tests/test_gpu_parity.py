@@ -275,6 +275,33 @@ def test_livelock_freedom_two_words(mode, k_lock, pipeline):
     assert st.commits == T * K
 
 
+@pytest.mark.parametrize("mode", ["hv", "tbv", "cgl", "fgl"])
+@pytest.mark.parametrize("wl,kw,T,K,cap", [
+    ("bank", dict(n_words=1 << 12), 1 << 16, 3, 2048),
+    ("km", dict(km_clusters=64, km_dims=16), 1 << 14, 2, 1024),
+    ("ra", dict(n_reads=4, n_writes=4, n_words=1024), 1000, 5, 96),
+])
+def test_concurrency_cap_replay(mode, wl, kw, T, K, cap):
+    """max_threads: fewer CUDA threads run the T STM threads grid-stride;
+    the run must stay serializable and respect each STM thread's order."""
+    g, gp, op, init = U.make(wl, T, K, 12, mode=mode, max_threads=cap, **kw)
+    st, *_ = U.run_verified(g, wl, op, init, T, K, 21)
+    assert st.commits + st.commits_ro == T * K
+
+
+@pytest.mark.parametrize("mode", ["hv", "tbv"])
+def test_k_lock_one_with_pipeline_progresses(mode):
+    """k_lock = 1 aborts on the first lost lock round; after such an abort a
+    transaction never uses the pipelined round again, so high contention
+    (RA configs[0]) still finishes (regression: pipelined-only retries
+    livelocked)."""
+    T, K = 256, 64
+    g, gp, op, init = U.make("ra", T, K, 10, mode=mode, n_reads=4, n_writes=4, n_words=1024, k_lock=1,
+                             lock_pipeline=1, timeout_ms=20000)
+    st, *_ = U.run_verified(g, "ra", op, init, T, K, 3)
+    assert st.aborts_lock > 0
+
+
 @pytest.mark.parametrize("pipeline,reuse,prelock", [(0, 0, 0), (0, 1, 1), (1, 0, 1), (1, 1, 0)])
 @pytest.mark.parametrize("mode", ["hv", "tbv"])
 def test_bank_knobs_replay(mode, pipeline, reuse, prelock):

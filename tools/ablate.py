@@ -49,6 +49,7 @@ def main():
     ap.add_argument("--sync", action="store_true", help="host sync after every step")
     ap.add_argument("--seed-base", type=int, default=0)
     ap.add_argument("--flush-first", action="store_true", help="allocate the L2-flush buffer before the handle")
+    ap.add_argument("--variant-timeout", type=int, default=240, help="seconds per variant process")
     ap.add_argument("--inproc", action="store_true",
                     help="run all variants in this process (default: one fresh process per variant, so "
                          "every variant sees the same allocation history)")
@@ -63,7 +64,11 @@ def main():
             j += 1
         base = argv[:i] + argv[j:]
         for v in a.variants:
-            subprocess.run([sys.executable, os.path.abspath(__file__)] + base + ["--variants", v], check=False)
+            try:
+                subprocess.run([sys.executable, os.path.abspath(__file__)] + base + ["--variants", v], check=False,
+                               timeout=a.variant_timeout)
+            except subprocess.TimeoutExpired:
+                print(json.dumps({"wl": a.wl, "variant": v, "error": f"timeout {a.variant_timeout}s"}), flush=True)
         return
 
     import torch
@@ -96,11 +101,15 @@ def main():
             g.attach_heap(theap)
         g.init_heap(wl)
         for w in range(a.warmup):
+            if wl == "ht":
+                g.init_heap("ht")
             g.run(wl, T, K, 1000 + w)
         torch.cuda.synchronize()
         g.reset_stats_total()
         evs = []
         for s in range(a.steps):
+            if wl == "ht":
+                g.init_heap("ht")       # HT node ids are per launch: every step starts from an empty table
             flush.fill_(float(s))
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
