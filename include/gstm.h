@@ -125,6 +125,18 @@ typedef struct {
  * 2^lock_table_bits version locks (0 <= bits <= 30, zeroed), the global clock
  * (0) and statistics.  Returns NULL on error (gstm_last_error). */
 gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits);
+/* flags for gstm_create_ex */
+#define GSTM_CREATE_PAIRED 1u
+/* As gstm_create, with layout flags.  GSTM_CREATE_PAIRED stores word w and
+ * its version lock w side by side in one 8-byte slot (value low half, lock
+ * high half) so a read, a lock acquisition (which also
+ * returns the value) and a write-back + unlock are one memory access each.
+ * Requires 1 <= heap_words <= 2^lock_table_bits (one lock per word, stripe
+ * 1).  The heap is still addressed by word index through every call below;
+ * gstm_attach_heap is not available in this layout.  flags = 0 is
+ * gstm_create (the paper's separate lock table). */
+gstm_t* gstm_create_ex(uint64_t heap_words, uint32_t lock_table_bits, uint32_t flags);
+uint32_t gstm_flags(const gstm_t* h);
 /* Frees everything the handle owns (not an attached heap).  NULL is a no-op. */
 void gstm_destroy(gstm_t* h);
 /* Message of the last failure on this thread ("" if none).  Static storage. */

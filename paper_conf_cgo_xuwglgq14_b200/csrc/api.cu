@@ -34,8 +34,9 @@ static constexpr int kClockStride = 288;           // ... 2304 B apart (crosses 
 
 struct gstm_handle {
     char* block = nullptr;          // the single device allocation
-    char* block2 = nullptr;         // (layout experiments only)
-    char* meta_sep = nullptr;
+    bool paired = false;            // GSTM_CREATE_PAIRED layout
+    uint32_t* scratch = nullptr;    // paired layout: plain word buffer for copies
+    uint64_t scratch_words = 0;
     unsigned long long* clock = nullptr;   // g_clock, on its own line inside the metadata block
     int clock_slot = -1;
     uint32_t* own_heap = nullptr;
@@ -143,62 +144,51 @@ int gstm_default_params(int workload, gstm_params_t* out)
 
 gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits)
 {
+    return gstm_create_ex(heap_words, lock_table_bits, 0);
+}
+
+gstm_t* gstm_create_ex(uint64_t heap_words, uint32_t lock_table_bits, uint32_t flags)
+{
     g_err[0] = 0;
     if (lock_table_bits > 30) { set_error("gstm_create: lock_table_bits %u > 30", lock_table_bits); return nullptr; }
+    if (flags & ~uint32_t(GSTM_CREATE_PAIRED)) { set_error("gstm_create_ex: unknown flags 0x%x", flags); return nullptr; }
+    const bool paired = (flags & GSTM_CREATE_PAIRED) != 0;
+    if (paired && (heap_words == 0 || heap_words > (1ull << lock_table_bits))) {
+        set_error("gstm_create_ex: the paired layout needs 1 <= heap_words <= 2^lock_table_bits (one lock per word)");
+        return nullptr;
+    }
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) { set_error("gstm_create: no CUDA device"); return nullptr; }
     gstm_t* h = new gstm_t();
     h->bits = lock_table_bits;
+    h->paired = paired;
     h->params = default_params(GSTM_WL_RA);
-    const size_t lock_bytes = sizeof(uint32_t) << lock_table_bits;
-    // one allocation, fixed layout [metadata | lock table | heap]: where the
-    // hot words land must not depend on the caller's other allocations
-    const size_t heap_bytes = (heap_words * 4 + 255) & ~size_t(255);
-    {
-        const char* lay = getenv("GSTM_LAYOUT");
-        const int layout = lay ? atoi(lay) : 0;
-        const size_t P2 = 2u << 20;
-        auto up = [&](size_t x) { return (x + P2 - 1) & ~(P2 - 1); };
-        if (layout == 1 || layout == 3) {          // separate allocations
-            if (layout == 3 && cudaMalloc(&h->meta_sep, kMetaBytes) != cudaSuccess) goto oom;
-            if (cudaMalloc(&h->block, heap_bytes + 256) != cudaSuccess) goto oom;
-            if (cudaMalloc(&h->block2, lock_bytes) != cudaSuccess) goto oom;
-            if (layout == 1 && cudaMalloc(&h->meta_sep, kMetaBytes) != cudaSuccess) goto oom;
-            h->own_heap = reinterpret_cast<uint32_t*>(h->block);
-            h->locks = reinterpret_cast<uint32_t*>(h->block2);
-            h->meta = reinterpret_cast<unsigned long long*>(h->meta_sep);
-        } else if (layout == 2) {                   // [meta | locks | heap], 2 MiB aligned
-            if (cudaMalloc(&h->block, P2 + up(lock_bytes) + up(heap_bytes)) != cudaSuccess) goto oom;
-            h->meta = reinterpret_cast<unsigned long long*>(h->block);
-            h->locks = reinterpret_cast<uint32_t*>(h->block + P2);
-            h->own_heap = reinterpret_cast<uint32_t*>(h->block + P2 + up(lock_bytes));
-        } else if (layout == 4) {                   // [heap | locks | meta], 2 MiB aligned
-            if (cudaMalloc(&h->block, up(heap_bytes) + up(lock_bytes) + kMetaBytes) != cudaSuccess) goto oom;
-            h->own_heap = reinterpret_cast<uint32_t*>(h->block);
-            h->locks = reinterpret_cast<uint32_t*>(h->block + up(heap_bytes));
-            h->meta = reinterpret_cast<unsigned long long*>(h->block + up(heap_bytes) + up(lock_bytes));
-        } else {                                    // [meta | locks | heap]
-            if (cudaMalloc(&h->block, kMetaBytes + lock_bytes + heap_bytes) != cudaSuccess) goto oom;
-            h->meta = reinterpret_cast<unsigned long long*>(h->block);
-            h->locks = reinterpret_cast<uint32_t*>(h->block + kMetaBytes);
-            h->own_heap = reinterpret_cast<uint32_t*>(h->block + kMetaBytes + lock_bytes);
-        }
-        if (!heap_words) h->own_heap = nullptr;
-        h->clock = h->meta + M_CLOCK;
+    // one allocation, fixed layout: where the hot words land must not depend
+    // on the caller's other allocations.  Split (the paper's): [metadata |
+    // lock table | heap].  Paired: [metadata | heap_words x (value, lock)].
+    const size_t lock_bytes = paired ? 0 : (sizeof(uint32_t) << lock_table_bits);
+    const size_t heap_bytes = ((paired ? heap_words * 8 : heap_words * 4) + 255) & ~size_t(255);
+    if (cudaMalloc(&h->block, kMetaBytes + lock_bytes + heap_bytes) != cudaSuccess) goto oom;
+    h->meta = reinterpret_cast<unsigned long long*>(h->block);
+    if (paired) {
+        h->own_heap = reinterpret_cast<uint32_t*>(h->block + kMetaBytes);
+        h->locks = h->own_heap + 1;
+    } else {
+        h->locks = reinterpret_cast<uint32_t*>(h->block + kMetaBytes);
+        h->own_heap = heap_words ? reinterpret_cast<uint32_t*>(h->block + kMetaBytes + lock_bytes) : nullptr;
     }
+    h->clock = h->meta + M_CLOCK;
     if (cudaStreamCreateWithFlags(&h->own_stream, cudaStreamNonBlocking) != cudaSuccess) goto cuerr;
     if (cudaEventCreate(&h->ev0) != cudaSuccess || cudaEventCreate(&h->ev1) != cudaSuccess) goto cuerr;
     h->stream = h->own_stream;
     h->heap = h->own_heap;
     h->heap_words = h->own_words = heap_words;
-    if (heap_words && cudaMemsetAsync(h->own_heap, 0, heap_words * 4, h->stream) != cudaSuccess) goto cuerr;
-    if (cudaMemsetAsync(h->locks, 0, lock_bytes, h->stream) != cudaSuccess) goto cuerr;
-    if (cudaMemsetAsync(h->meta, 0, kMetaBytes, h->stream) != cudaSuccess) goto cuerr;
+    if (cudaMemsetAsync(h->block, 0, kMetaBytes + lock_bytes + heap_bytes, h->stream) != cudaSuccess) goto cuerr;
     if (cudaStreamSynchronize(h->stream) != cudaSuccess) goto cuerr;
     {
-        // place g_clock on the candidate line with the fastest hot-spot
-        // atomic rate; GSTM_CLOCK_SLOT=k forces candidate
-        // k, GSTM_CLOCK_SLOT=-1 the fixed word M_CLOCK
+        // place g_clock on the candidate line with the fastest probe
+        // (DESIGN.md §6.5); GSTM_CLOCK_SLOT=k forces candidate k,
+        // GSTM_CLOCK_SLOT=-1 the fixed word M_CLOCK
         const char* cs = getenv("GSTM_CLOCK_SLOT");
         int slot;
         if (cs) {
@@ -206,12 +196,17 @@ gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits)
         } else if (lock_table_bits < 14) {
             slot = -1;          // small tables: the hot-slice effect is negligible, skip the probe
         } else {
-            uint64_t hw = 1;
-            while (hw * 2 <= heap_words) hw *= 2;
-            uint32_t* hp = heap_words ? h->own_heap : h->locks;
-            const uint32_t hmask = heap_words ? static_cast<uint32_t>(hw - 1) : static_cast<uint32_t>((1ull << lock_table_bits) - 1);
-            slot = clock_calibrate_mix(h->meta + M_WORDS, kClockCandidates, kClockStride, h->locks,
-                                       static_cast<uint32_t>((1ull << lock_table_bits) - 1), hp, hmask, h->stream);
+            // the probe's random lock-table and heap traffic goes over the
+            // handle's own tables (for the paired layout: the pair array)
+            uint32_t* tbl = paired ? h->own_heap : h->locks;
+            const uint64_t tbl_words = paired ? 2 * heap_words : (1ull << lock_table_bits);
+            uint32_t* hp = paired ? h->own_heap : (heap_words ? h->own_heap : h->locks);
+            const uint64_t hp_words = paired ? 2 * heap_words : (heap_words ? heap_words : tbl_words);
+            uint64_t t2 = 1, h2 = 1;
+            while (t2 * 2 <= tbl_words) t2 *= 2;
+            while (h2 * 2 <= hp_words) h2 *= 2;
+            slot = clock_calibrate_mix(h->meta + M_WORDS, kClockCandidates, kClockStride, tbl,
+                                       static_cast<uint32_t>(t2 - 1), hp, static_cast<uint32_t>(h2 - 1), h->stream);
         }
         if (slot >= kClockCandidates) slot = kClockCandidates - 1;
         h->clock_slot = slot;
@@ -229,13 +224,14 @@ cuerr:
     return nullptr;
 }
 
+uint32_t gstm_flags(const gstm_t* h) { return h && h->paired ? GSTM_CREATE_PAIRED : 0u; }
+
 void gstm_destroy(gstm_t* h)
 {
     if (!h) return;
     if (h->stream) cudaStreamSynchronize(h->stream);
     cudaFree(h->block);
-    cudaFree(h->block2);
-    cudaFree(h->meta_sep);
+    cudaFree(h->scratch);
     cudaFree(h->tx_stamp);
     cudaFree(h->tx_result);
     if (h->ev0) cudaEventDestroy(h->ev0);
@@ -284,6 +280,7 @@ int gstm_attach_heap(gstm_t* h, void* dev_ptr, uint64_t words)
         h->heap_words = h->own_words;
         return GSTM_OK;
     }
+    if (h->paired) { set_error("gstm_attach_heap: not available with the paired layout"); return GSTM_EINVAL; }
     if (reinterpret_cast<uintptr_t>(dev_ptr) & 3) { set_error("gstm_attach_heap: unaligned pointer"); return GSTM_EINVAL; }
     h->heap = static_cast<uint32_t*>(dev_ptr);
     h->heap_words = words;
@@ -293,18 +290,59 @@ int gstm_attach_heap(gstm_t* h, void* dev_ptr, uint64_t words)
 uint64_t gstm_heap_words(const gstm_t* h) { return h ? h->heap_words : 0; }
 void* gstm_heap_ptr(const gstm_t* h) { return h ? h->heap : nullptr; }
 
+// paired layout: a plain device buffer of `words` words for packing
+static int ensure_scratch(gstm_t* h, uint64_t words)
+{
+    if (h->scratch_words >= words) return GSTM_OK;
+    cudaFree(h->scratch);
+    h->scratch = nullptr;
+    h->scratch_words = 0;
+    if (cudaMalloc(&h->scratch, words * 4) != cudaSuccess) { set_error("out of device memory (scratch)"); return GSTM_ENOMEM; }
+    h->scratch_words = words;
+    return GSTM_OK;
+}
+
 int gstm_init_heap(gstm_t* h, int workload)
 {
     if (!h || workload < 0 || workload > 4) { set_error("gstm_init_heap: bad argument"); return GSTM_EINVAL; }
-    CUDA_TRY(launch_init_heap(workload, h->heap, h->heap_words, h->stream));
+    CUDA_TRY(launch_init_heap(workload, h->heap, h->heap_words, h->paired ? 1 : 0, h->stream));
+    return GSTM_OK;
+}
+
+// host -> heap words [offset, offset+words), asynchronous on the handle's stream
+static int copy_in(gstm_t* h, const uint32_t* src, uint64_t offset, uint64_t words)
+{
+    if (!words) return GSTM_OK;
+    if (!h->paired) {
+        CUDA_TRY(cudaMemcpyAsync(h->heap + offset, src, words * 4, cudaMemcpyHostToDevice, h->stream));
+        return GSTM_OK;
+    }
+    int rc = ensure_scratch(h, words);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(h->scratch, src, words * 4, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(launch_pack(h->scratch, h->heap + 2 * offset, words, 1, h->stream));
+    return GSTM_OK;
+}
+
+static int copy_out(gstm_t* h, uint32_t* dst, uint64_t offset, uint64_t words)
+{
+    if (!words) return GSTM_OK;
+    if (!h->paired) {
+        CUDA_TRY(cudaMemcpyAsync(dst, h->heap + offset, words * 4, cudaMemcpyDeviceToHost, h->stream));
+        return GSTM_OK;
+    }
+    int rc = ensure_scratch(h, words);
+    if (rc) return rc;
+    CUDA_TRY(launch_pack(h->scratch, h->heap + 2 * offset, words, 0, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(dst, h->scratch, words * 4, cudaMemcpyDeviceToHost, h->stream));
     return GSTM_OK;
 }
 
 int gstm_write_heap(gstm_t* h, const uint32_t* src, uint64_t offset, uint64_t words)
 {
     if (!h || (!src && words) || offset + words > h->heap_words) { set_error("gstm_write_heap: bad range"); return GSTM_EINVAL; }
-    if (!words) return GSTM_OK;
-    CUDA_TRY(cudaMemcpyAsync(h->heap + offset, src, words * 4, cudaMemcpyHostToDevice, h->stream));
+    int rc = copy_in(h, src, offset, words);
+    if (rc) return rc;
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     return GSTM_OK;
 }
@@ -312,8 +350,8 @@ int gstm_write_heap(gstm_t* h, const uint32_t* src, uint64_t offset, uint64_t wo
 int gstm_read_heap(gstm_t* h, uint32_t* dst, uint64_t offset, uint64_t words)
 {
     if (!h || (!dst && words) || offset + words > h->heap_words) { set_error("gstm_read_heap: bad range"); return GSTM_EINVAL; }
-    if (!words) return GSTM_OK;
-    CUDA_TRY(cudaMemcpyAsync(dst, h->heap + offset, words * 4, cudaMemcpyDeviceToHost, h->stream));
+    int rc = copy_out(h, dst, offset, words);
+    if (rc) return rc;
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     return GSTM_OK;
 }
@@ -321,7 +359,17 @@ int gstm_read_heap(gstm_t* h, uint32_t* dst, uint64_t offset, uint64_t words)
 int gstm_read_locks(gstm_t* h, uint32_t* dst, uint64_t n)
 {
     if (!h || !dst || n > (1ull << h->bits)) { set_error("gstm_read_locks: bad range"); return GSTM_EINVAL; }
-    CUDA_TRY(cudaMemcpyAsync(dst, h->locks, n * 4, cudaMemcpyDeviceToHost, h->stream));
+    if (!h->paired) {
+        CUDA_TRY(cudaMemcpyAsync(dst, h->locks, n * 4, cudaMemcpyDeviceToHost, h->stream));
+    } else {
+        // lock i lives next to word i; locks of ids >= heap_words are never used
+        const uint64_t m = n < h->own_words ? n : h->own_words;
+        int rc = ensure_scratch(h, m ? m : 1);
+        if (rc) return rc;
+        CUDA_TRY(launch_lock_halves(h->own_heap, m, h->scratch, h->stream));
+        if (m) CUDA_TRY(cudaMemcpyAsync(dst, h->scratch, m * 4, cudaMemcpyDeviceToHost, h->stream));
+        for (uint64_t k = m; k < n; ++k) dst[k] = 0;
+    }
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     return GSTM_OK;
 }
@@ -339,7 +387,8 @@ int gstm_read_clock(gstm_t* h, uint64_t* out)
 int gstm_reset_meta(gstm_t* h)
 {
     if (!h) { set_error("gstm_reset_meta: NULL"); return GSTM_EINVAL; }
-    CUDA_TRY(cudaMemsetAsync(h->locks, 0, sizeof(uint32_t) << h->bits, h->stream));
+    if (h->paired) CUDA_TRY(launch_lock_halves(h->own_heap, h->own_words, nullptr, h->stream));
+    else CUDA_TRY(cudaMemsetAsync(h->locks, 0, sizeof(uint32_t) << h->bits, h->stream));
     CUDA_TRY(cudaMemsetAsync(h->clock, 0, 8, h->stream));
     h->clock_bound = 0;
     return GSTM_OK;
@@ -379,6 +428,8 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
         return GSTM_EINVAL;
     }
     if (n_threads > (1ull << 32)) { set_error("gstm_launch: n_threads > 2^32"); return GSTM_EINVAL; }
+    if (h->paired && P.lock_shift) { set_error("gstm_launch: the paired layout has one lock per word (lock_shift 0)"); return GSTM_EINVAL; }
+    if (P.lock_shift > 31) { set_error("gstm_launch: lock_shift > 31"); return GSTM_EINVAL; }
     const uint64_t n_tx = n_threads * tx_per_thread;
     if (n_tx >= (1ull << 31) - 2) { set_error("gstm_launch: %llu transactions >= 2^31", (unsigned long long)n_tx); return GSTM_EOVERFLOW; }
     // 31-bit versions: start a new version epoch before they can wrap
@@ -408,6 +459,8 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.m.clock = h->clock;
     kp.m.spin_cap = P.spin_cap ? P.spin_cap : (1u << 16);
     kp.m.lock_shift = P.lock_shift;
+    kp.m.vshift = kp.m.lshift = h->paired ? 1u : 0u;
+    kp.paired = h->paired ? 1u : 0u;
     kp.w = w;
     kp.meta = h->meta;
     kp.tx_stamp = P.verify ? h->tx_stamp : nullptr;
@@ -487,10 +540,12 @@ int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* he
                   uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed, gstm_stats_t* stats)
 {
     if (!h || words > h->heap_words || (words && (!heap_in || !heap_out))) { set_error("gstm_run_host: bad buffers"); return GSTM_EINVAL; }
-    if (words) CUDA_TRY(cudaMemcpyAsync(h->heap, heap_in, words * 4, cudaMemcpyHostToDevice, h->stream));
-    int rc = gstm_launch(h, workload, n_threads, tx_per_thread, seed);
+    int rc = copy_in(h, heap_in, 0, words);
     if (rc) return rc;
-    if (words) CUDA_TRY(cudaMemcpyAsync(heap_out, h->heap, words * 4, cudaMemcpyDeviceToHost, h->stream));
+    rc = gstm_launch(h, workload, n_threads, tx_per_thread, seed);
+    if (rc) return rc;
+    rc = copy_out(h, heap_out, 0, words);
+    if (rc) return rc;
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     gstm_stats_t local;
     return gstm_stats(h, stats ? stats : &local);
@@ -559,6 +614,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
     m.clock = h->clock;
     m.spin_cap = 64;
     m.lock_shift = 0;
+    m.vshift = m.lshift = h->paired ? 1u : 0u;
     if (e == cudaSuccess) e = cudaMemcpyAsync(dops, ops, n_ops * 16, cudaMemcpyHostToDevice, h->stream);
     if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, h->stream);
     if (e == cudaSuccess) e = cudaMemcpyAsync(out, dout, n_ops * 16, cudaMemcpyDeviceToHost, h->stream);

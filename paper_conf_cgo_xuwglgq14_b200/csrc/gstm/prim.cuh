@@ -113,6 +113,34 @@ __device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t v)
     return old;
 }
 
+// 8-byte accesses for the paired layout (value | version lock in one
+// naturally aligned u64: single-copy atomic, one L2 request)
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long atom_or_acquire_u64(unsigned long long* p, unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.acquire.gpu.global.or.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ unsigned long long atom_or_relaxed_u64(unsigned long long* p, unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.relaxed.gpu.global.or.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+
 __device__ __forceinline__ uint32_t atom_or_relaxed(uint32_t* p, uint32_t v)
 {
     uint32_t old;

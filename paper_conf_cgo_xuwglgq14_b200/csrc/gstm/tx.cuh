@@ -29,16 +29,24 @@ enum { MODE_HV = 1, MODE_TBV = 2 };
 enum { C_OK = 0, C_OPACITY = 1, C_PREVBV = 2, C_TBV = 3, C_COMMITVBV = 4, C_READONLY = 5, C_LOCK = 6 };
 
 struct Meta {
-    uint32_t* heap;
-    uint32_t* locks;
+    uint32_t* heap;                  // word w at heap[w << vshift]
+    uint32_t* locks;                 // version lock i at locks[i << lshift]
     uint32_t lock_mask;              // 2^bits - 1
     uint32_t lock_shift;             // stripe = 2^shift words (0: one lock per word)
+    uint32_t vshift, lshift;         // 0,0: the paper's separate lock table; 1,1: paired layout
     unsigned long long* clock;       // g_clock
     uint32_t spin_cap;               // bound on the l.27-29 spin and on PostValidation restarts
 
     // hash(addr) of P:113 (reading Q2): the version lock of a memory stripe
     // of 2^lock_shift consecutive words, modulo the table size
     __device__ __forceinline__ uint32_t lock_of(uint32_t w) const { return (w >> lock_shift) & lock_mask; }
+    __device__ __forceinline__ uint32_t* val_ptr(uint32_t w) const { return heap + (static_cast<uint64_t>(w) << vshift); }
+    __device__ __forceinline__ uint32_t* lock_ptr(uint32_t id) const { return locks + (static_cast<uint64_t>(id) << lshift); }
+    // paired layout: word w and its version lock in one u64 (value low, lock high)
+    __device__ __forceinline__ unsigned long long* pair_ptr(uint32_t w) const
+    {
+        return reinterpret_cast<unsigned long long*>(heap) + w;
+    }
 };
 
 // A3.l83 version <- Atomic_inc(g_clock) + 1, for n commits at once (the
@@ -164,13 +172,13 @@ struct Tx {
             uint32_t cur[RCAP];
 #pragma unroll
             for (int k = 0; k < RCAP; ++k)
-                if (k < nr) cur[k] = prim::ld_relaxed(m.heap + r_addr[k]);
+                if (k < nr) cur[k] = prim::ld_relaxed(m.val_ptr(r_addr[k]));
 #pragma unroll
             for (int k = 0; k < RCAP; ++k)
                 if (k < nr) ok &= (cur[k] == r_val[k]);
         } else {
             for (int k = 0; k < nr; ++k)
-                ok &= (prim::ld_relaxed(m.heap + r_addr[k]) == r_val[k]);
+                ok &= (prim::ld_relaxed(m.val_ptr(r_addr[k])) == r_val[k]);
         }
         return ok;
     }
@@ -191,7 +199,7 @@ struct Tx {
                 uint32_t vl[RCAP];
 #pragma unroll
                 for (int k = 0; k < RCAP; ++k)                       // l.13
-                    if (k < nr) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(r_addr[k])); // l.14
+                    if (k < nr) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(r_addr[k]))); // l.14
 #pragma unroll
                 for (int k = 0; k < RCAP; ++k)
                     if (k < nr && ((vl[k] & 1u) || (vl[k] >> 1) > snapshot)) {   // l.15-17
@@ -200,7 +208,7 @@ struct Tx {
                     }
             } else {
                 for (int k = 0; k < nr; ++k) {
-                    const uint32_t vl = prim::ld_relaxed(m.locks + m.lock_of(r_addr[k]));
+                    const uint32_t vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(r_addr[k])));
                     if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
                 }
             }
@@ -218,7 +226,7 @@ struct Tx {
         while (vl & 1u) {                                            // l.29
             if (++spins > m.spin_cap) { opaque = false; break; }
             __nanosleep(32);
-            vl = prim::ld_relaxed(m.locks + m.lock_of(a));      // l.28
+            vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));      // l.28
         }
         n_spin += spins;
         const uint32_t version = vl >> 1;                            // l.30
@@ -236,10 +244,10 @@ struct Tx {
     {
         uint32_t v;
         if (raw_lookup(a, v)) return v;                              // l.22-23
-        v = prim::ld_relaxed(m.heap + a);                            // l.24
+        v = prim::ld_relaxed(m.val_ptr(a));                            // l.24
         append_read(a, v);                                           // l.25
         prim::fence_acquire();                                       // l.26
-        const uint32_t vl = prim::ld_relaxed(m.locks + m.lock_of(a));
+        const uint32_t vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));
         check_lock(m, a, vl, mode);                                  // l.27-33
         insert_lock((m.lock_of(a) << 2) | 1u);                  // l.34
         return v;                                                    // l.35
@@ -261,14 +269,14 @@ struct Tx {
         for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (need[k]) v[k] = prim::ld_relaxed(m.heap + a[k]);    // l.24
+            if (need[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));    // l.24
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) append_read(a[k], v[k]);                    // l.25
         prim::fence_acquire();                                       // l.26
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (need[k]) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(a[k]));
+            if (need[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) {
@@ -287,13 +295,13 @@ struct Tx {
         uint32_t vl[kRcap];
 #pragma unroll 8
         for (int k = 0; k < n; ++k)
-            if (!skip[k]) v[k] = prim::ld_relaxed(m.heap + a[k]);   // l.24
+            if (!skip[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));   // l.24
         for (int k = 0; k < n; ++k)
             if (!skip[k]) append_read(a[k], v[k]);                    // l.25
         prim::fence_acquire();                                        // l.26
 #pragma unroll 8
         for (int k = 0; k < n; ++k)
-            if (!skip[k]) vl[k] = prim::ld_relaxed(m.locks + m.lock_of(a[k]));
+            if (!skip[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
         for (int k = 0; k < n; ++k)
             if (!skip[k]) {
                 check_lock(m, a[k], vl[k], mode);                     // l.27-33
@@ -336,9 +344,9 @@ struct Tx {
         if constexpr (kUnroll) {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k)
-                if (k < n_acq) prim::st_relaxed(m.locks + (l_ent[k] >> 2), l_old[k]);
+                if (k < n_acq) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]);
         } else {
-            for (int k = 0; k < n_acq; ++k) prim::st_relaxed(m.locks + (l_ent[k] >> 2), l_old[k]);
+            for (int k = 0; k < n_acq; ++k) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]);
         }
         n_acq = 0;
     }
@@ -355,7 +363,7 @@ struct Tx {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k) {
                 if (ok && k < nl) {
-                    const uint32_t vl = prim::atom_or_acquire(m.locks + (l_ent[k] >> 2), 1u);  // l.45
+                    const uint32_t vl = prim::atom_or_acquire(m.lock_ptr(l_ent[k] >> 2), 1u);  // l.45
                     if (vl & 1u) {
                         ok = false;                                  // l.46-48
                     } else {
@@ -367,7 +375,7 @@ struct Tx {
             }
         } else {
             for (int k = 0; k < nl; ++k) {
-                const uint32_t vl = prim::atom_or_acquire(m.locks + (l_ent[k] >> 2), 1u);
+                const uint32_t vl = prim::atom_or_acquire(m.lock_ptr(l_ent[k] >> 2), 1u);
                 if (vl & 1u) { ok = false; break; }
                 l_old[k] = vl;
                 n_acq = k + 1;
@@ -390,7 +398,7 @@ struct Tx {
         uint32_t vl[LCAP];
 #pragma unroll
         for (int k = 0; k < LCAP; ++k)
-            if (k < nl) vl[k] = prim::atom_or_relaxed(m.locks + (l_ent[k] >> 2), 1u);   // l.45, all at once
+            if (k < nl) vl[k] = prim::atom_or_relaxed(m.lock_ptr(l_ent[k] >> 2), 1u);   // l.45, all at once
         prim::fence_acquire();
         bool ok = true;
 #pragma unroll
@@ -399,7 +407,7 @@ struct Tx {
         if (!ok) {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k)                           // l.47: undo what we set
-                if (k < nl && !(vl[k] & 1u)) prim::st_relaxed(m.locks + (l_ent[k] >> 2), vl[k]);
+                if (k < nl && !(vl[k] & 1u)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), vl[k]);
             n_acq = 0;
             return false;
         }
@@ -444,9 +452,9 @@ struct Tx {
         if constexpr (kUnroll) {
 #pragma unroll
             for (int k = 0; k < WCAP; ++k)
-                if (k < nw) prim::st_relaxed(m.heap + w_addr[k], w_val[k]);
+                if (k < nw) prim::st_relaxed(m.val_ptr(w_addr[k]), w_val[k]);
         } else {
-            for (int k = 0; k < nw; ++k) prim::st_relaxed(m.heap + w_addr[k], w_val[k]);
+            for (int k = 0; k < nw; ++k) prim::st_relaxed(m.val_ptr(w_addr[k]), w_val[k]);
         }
         prim::fence_release();                                       // l.82
     }
@@ -460,10 +468,10 @@ struct Tx {
         if constexpr (kUnroll) {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k)
-                if (k < nl) prim::st_relaxed(m.locks + (l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
+                if (k < nl) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
         } else {
             for (int k = 0; k < nl; ++k)
-                prim::st_relaxed(m.locks + (l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
+                prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
         }
         n_acq = 0;
     }

@@ -1,0 +1,355 @@
+// tx_pair.cuh -- GPU-STM on the PAIRED layout.
+//
+// The paper keeps a global table of version locks apart from the data and
+// maps word w to lock hash(w).  When the table has one lock
+// per word (2^bits >= heap words, stripe 1 -- the regime where P:252 picks
+// TBV), the same logical structure can be laid out B200-first: word w and its
+// version lock share one naturally aligned u64 (value in the low half, lock
+// word in the high half).  Then
+//   * TXRead is ONE 8-byte strong load: value and version lock read
+//     atomically together (A3.l24 and l.28 at one instant, no fence l.26);
+//   * PostValidation checks value and lock of each read word in one pass;
+//   * lock acquisition `atom.or.b64` returns the word's current value with
+//     the old lock, so the VBV under locks (A3.l76) needs no memory access;
+//   * write-back and lock release of a written word are one 8-byte store
+//     (value, stamp<<1), issued after the stamp: a reader that sees the word
+//     still locked waits (A3.l27-29), so publishing the value with the
+//     unlock is equivalent to l.80-84 and needs no release fence (l.82).
+// Per bank transaction: 2 + 2 + 2 (+ clock) L2 requests instead of 14.
+#pragma once
+#include "tx.cuh"
+
+namespace gstm {
+
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL>;
+    using B::kUnroll;
+    using B::r_addr;
+    using B::r_val;
+    using B::w_addr;
+    using B::w_val;
+    using B::l_ent;
+    using B::l_old;
+    using B::nr;
+    using B::nw;
+    using B::nl;
+    using B::n_acq;
+    using B::snapshot;
+    using B::opaque;
+    using B::passTBV;
+    using B::n_postval;
+    using B::n_vbv;
+    using B::n_spin;
+    using B::raw_lookup;
+    using B::append_read;
+    using B::insert_lock;
+
+    uint32_t l_val[LCAP];   // value each acquiring atom.or.b64 returned
+
+    static __device__ __forceinline__ uint32_t lo(unsigned long long p) { return static_cast<uint32_t>(p); }
+    static __device__ __forceinline__ uint32_t hi(unsigned long long p) { return static_cast<uint32_t>(p >> 32); }
+    static __device__ __forceinline__ unsigned long long mk(uint32_t val, uint32_t lock)
+    {
+        return (static_cast<unsigned long long>(lock) << 32) | val;
+    }
+
+    // ---- A3.l6-20 PostValidation: value and lock of every read word from
+    //      one atomic 8-byte load (l.9-11 and l.13-19 in one pass) --------
+    __device__ __forceinline__ bool post_validation(const Meta& m, uint32_t version)
+    {
+        ++n_postval;
+        ++n_vbv;
+        if (version > snapshot) snapshot = version;                  // l.7 (Q9)
+        for (uint32_t restart = 0; restart <= m.spin_cap; ++restart) {  // l.8
+            bool again = false, ok = true;
+            uint32_t newsnap = snapshot;
+            if constexpr (kUnroll) {
+                unsigned long long pv[RCAP];
+#pragma unroll
+                for (int k = 0; k < RCAP; ++k)
+                    if (k < nr) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]));
+#pragma unroll
+                for (int k = 0; k < RCAP; ++k)
+                    if (k < nr) {
+                        ok &= (lo(pv[k]) == r_val[k]);                  // l.10
+                        const uint32_t vl = hi(pv[k]);
+                        if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                    }
+            } else {
+                for (int k = 0; k < nr; ++k) {
+                    const unsigned long long pv = prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]));
+                    ok &= (lo(pv) == r_val[k]);
+                    const uint32_t vl = hi(pv);
+                    if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                }
+            }
+            if (!ok) return false;                                   // l.11
+            snapshot = newsnap;                                      // l.18
+            if (!again) return true;                                 // l.20
+            if (restart) __nanosleep(64);
+        }
+        return false;
+    }
+
+    // A3.l27-29: while the word is locked re-read the pair (value and lock),
+    // so the logged value is the one that goes with the version checked
+    __device__ __forceinline__ unsigned long long settle(const Meta& m, uint32_t a, unsigned long long pv)
+    {
+        uint32_t spins = 0;
+        while (hi(pv) & 1u) {
+            if (++spins > m.spin_cap) { opaque = false; break; }
+            __nanosleep(32);
+            pv = prim::ld_relaxed_u64(m.pair_ptr(a));
+        }
+        n_spin += spins;
+        return pv;
+    }
+
+    // A3.l30-33
+    __device__ __forceinline__ void check_version(const Meta& m, uint32_t vl, int mode)
+    {
+        const uint32_t version = vl >> 1;
+        if (opaque && version > snapshot) {
+            if (mode == MODE_HV) {
+                if (!post_validation(m, version)) opaque = false;
+            } else {
+                opaque = false;
+            }
+        }
+    }
+
+    __device__ __forceinline__ uint32_t read(const Meta& m, uint32_t a, int mode)
+    {
+        uint32_t v;
+        if (raw_lookup(a, v)) return v;                              // l.22-23
+        const unsigned long long pv = settle(m, a, prim::ld_relaxed_u64(m.pair_ptr(a)));   // l.24, l.27-29
+        v = lo(pv);
+        append_read(a, v);                                           // l.25
+        check_version(m, hi(pv), mode);                              // l.30-33
+        insert_lock((a << 2) | 1u);                                  // l.34 (lock id = word)
+        return v;
+    }
+
+    template <int N>
+    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode)
+    {
+        bool need[N];
+        unsigned long long pv[N];
+#pragma unroll
+        for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) {
+                pv[k] = settle(m, a[k], pv[k]);
+                v[k] = lo(pv[k]);
+                append_read(a[k], v[k]);
+            }
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) {
+                check_version(m, hi(pv[k]), mode);
+                insert_lock((a[k] << 2) | 1u);
+            }
+    }
+
+    __device__ __forceinline__ void read_many(const Meta& m, const uint32_t* a, uint32_t* v, const bool* skip, int n,
+                                              int mode)
+    {
+        uint32_t vl[RCAP];
+#pragma unroll 8
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) {
+                const unsigned long long pv = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
+                v[k] = lo(pv);
+                vl[k] = hi(pv);
+            }
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) {
+                if (vl[k] & 1u) {
+                    const unsigned long long pv = settle(m, a[k], mk(v[k], vl[k]));
+                    v[k] = lo(pv);
+                    vl[k] = hi(pv);
+                }
+                append_read(a[k], v[k]);
+            }
+        for (int k = 0; k < n; ++k)
+            if (!skip[k]) {
+                check_version(m, vl[k], mode);
+                insert_lock((a[k] << 2) | 1u);
+            }
+    }
+
+    // ---- A3.l62-66 VBV from the values in memory --------------------------
+    __device__ __forceinline__ bool vbv(const Meta& m)
+    {
+        ++n_vbv;
+        bool ok = true;
+        if constexpr (kUnroll) {
+            unsigned long long pv[RCAP];
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+                if (k < nr) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]));
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+                if (k < nr) ok &= (lo(pv[k]) == r_val[k]);
+        } else {
+            for (int k = 0; k < nr; ++k) ok &= (lo(prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]))) == r_val[k]);
+        }
+        return ok;
+    }
+
+    // ---- A3.l76 VBV under locks, from the values the atomics returned ----
+    __device__ __forceinline__ bool vbv_locked()
+    {
+        ++n_vbv;
+        bool ok = true;
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < RCAP; ++k)
+#pragma unroll
+                for (int j = 0; j < LCAP; ++j)
+                    if (k < nr && j < nl && (l_ent[j] >> 2) == r_addr[k]) ok &= (l_val[j] == r_val[k]);
+        } else {
+            for (int k = 0; k < nr; ++k)
+                for (int j = 0; j < nl; ++j)
+                    if ((l_ent[j] >> 2) == r_addr[k]) { ok &= (l_val[j] == r_val[k]); break; }
+        }
+        return ok;
+    }
+
+    // ---- A3.l53-55 ReleaseLocks: put back the exact pairs we locked -------
+    __device__ __forceinline__ void release_locks(const Meta& m)
+    {
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k < n_acq) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), mk(l_val[k], l_old[k]));
+        } else {
+            for (int k = 0; k < n_acq; ++k) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), mk(l_val[k], l_old[k]));
+        }
+        n_acq = 0;
+    }
+
+    // ---- A3.l43-52 GetLocksAndTBV, sequential in ascending id -------------
+    __device__ __forceinline__ bool get_locks_and_tbv(const Meta& m)
+    {
+        n_acq = 0;
+        bool ok = true;
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k) {
+                if (ok && k < nl) {
+                    const unsigned long long old = prim::atom_or_acquire_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);  // l.45
+                    if (hi(old) & 1u) {
+                        ok = false;                                  // l.46-48
+                    } else {
+                        l_old[k] = hi(old);
+                        l_val[k] = lo(old);
+                        n_acq = k + 1;
+                        if ((l_ent[k] & 1u) && (hi(old) >> 1) > snapshot) passTBV = false;  // l.49-51
+                    }
+                }
+            }
+        } else {
+            for (int k = 0; k < nl; ++k) {
+                const unsigned long long old = prim::atom_or_acquire_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);
+                if (hi(old) & 1u) { ok = false; break; }
+                l_old[k] = hi(old);
+                l_val[k] = lo(old);
+                n_acq = k + 1;
+                if ((l_ent[k] & 1u) && (hi(old) >> 1) > snapshot) passTBV = false;
+            }
+        }
+        if (!ok) release_locks(m);                                   // l.47
+        return ok;
+    }
+
+    // first round of a fresh execution: all atom.or.b64 at once (§6.4)
+    __device__ __forceinline__ bool get_locks_and_tbv_pipelined(const Meta& m)
+    {
+        static_assert(kUnroll, "pipelined acquisition needs register-resident logs");
+        unsigned long long old[LCAP];
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) old[k] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);
+        prim::fence_acquire();
+        bool ok = true;
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (hi(old[k]) & 1u)) ok = false;
+        if (!ok) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k < nl && !(hi(old[k]) & 1u)) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), old[k]);
+            n_acq = 0;
+            return false;
+        }
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) {
+                l_old[k] = hi(old[k]);
+                l_val[k] = lo(old[k]);
+                if ((l_ent[k] & 1u) && (hi(old[k]) >> 1) > snapshot) passTBV = false;
+            }
+        n_acq = nl;
+        return true;
+    }
+
+    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
+    {
+        if (mode == MODE_HV && prelock_vbv)
+            if (!vbv(m)) return C_PREVBV;                            // l.71-72
+        bool got;
+        if constexpr (kUnroll) got = pipelined ? get_locks_and_tbv_pipelined(m) : get_locks_and_tbv(m);
+        else got = get_locks_and_tbv(m);
+        if (!got) return C_LOCK;                                     // l.73
+        if (!passTBV) {                                              // l.75
+            if (mode != MODE_HV) { release_locks(m); return C_TBV; }
+            if (!vbv_locked()) { release_locks(m); return C_COMMITVBV; }   // l.76-78
+        }
+        return C_OK;
+    }
+
+    // l.79-82: nothing to do here -- each written value is published
+    // together with its unlock in release_and_update
+    __device__ __forceinline__ void writeback(const Meta&) {}
+
+    // ---- A3.l80-84: written pairs get (new value, stamp<<1); read-only
+    //      pairs get back exactly what the atomic returned --------------------
+    __device__ __forceinline__ void release_and_update(const Meta& m, uint32_t version)
+    {
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)
+                if (k < nl) {
+                    const uint32_t id = l_ent[k] >> 2;
+                    uint32_t val = l_val[k], lock = l_old[k];
+                    if (l_ent[k] & 2u) {
+                        lock = version << 1;
+#pragma unroll
+                        for (int j = 0; j < WCAP; ++j)
+                            if (j < nw && w_addr[j] == id) val = w_val[j];
+                    }
+                    prim::st_relaxed_u64(m.pair_ptr(id), mk(val, lock));
+                }
+        } else {
+            for (int k = 0; k < nl; ++k) {
+                const uint32_t id = l_ent[k] >> 2;
+                uint32_t val = l_val[k], lock = l_old[k];
+                if (l_ent[k] & 2u) {
+                    lock = version << 1;
+                    for (int j = 0; j < nw; ++j)
+                        if (w_addr[j] == id) { val = w_val[j]; break; }
+                }
+                prim::st_relaxed_u64(m.pair_ptr(id), mk(val, lock));
+            }
+        }
+        n_acq = 0;
+    }
+};
+
+}  // namespace gstm

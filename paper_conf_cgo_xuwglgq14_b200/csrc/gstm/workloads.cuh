@@ -54,23 +54,23 @@ struct StmCtx {
 };
 
 struct DirectCtx {
-    uint32_t* heap;
+    const Meta& m;
     int nw;
     bool bad;
-    __device__ __forceinline__ uint32_t read(uint32_t a) { return prim::ld_relaxed(heap + a); }
+    __device__ __forceinline__ uint32_t read(uint32_t a) { return prim::ld_relaxed(m.val_ptr(a)); }
     template <int N>
     __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n)
     {
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (k < n) v[k] = prim::ld_relaxed(heap + a[k]);
+            if (k < n) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
     }
     __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
     {
         for (int k = 0; k < n; ++k)
-            if (!skip[k]) v[k] = prim::ld_relaxed(heap + a[k]);
+            if (!skip[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
     }
-    __device__ __forceinline__ void write(uint32_t a, uint32_t v) { prim::st_relaxed(heap + a, v); ++nw; }
+    __device__ __forceinline__ void write(uint32_t a, uint32_t v) { prim::st_relaxed(m.val_ptr(a), v); ++nw; }
     __device__ __forceinline__ bool ok() const { return !bad; }
     __device__ __forceinline__ void invalid() { bad = true; }
     __device__ __forceinline__ void overflow() { bad = true; }

@@ -60,7 +60,11 @@ __device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool g
     unsigned long long base = 0;
     if (gm) {
         const int leader = __ffs(gm) - 1;
+#if GSTM_EXPERIMENT_NO_CLOCK   // measurement only: fake stamps, NOT serializable
+        base = (static_cast<unsigned long long>(blockIdx.x) << 20) + threadIdx.x;
+#else
         if (static_cast<int>(prim::lane_id()) == leader) base = clock_fetch_add(clock, __popc(gm));
+#endif
         base = __shfl_sync(FULL, base, leader);
         __syncwarp();
         next_snap = static_cast<uint32_t>(base) + __popc(gm);
@@ -110,10 +114,11 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
 // STM kernel: GPU-STM with hierarchical validation (MODE_HV, "STM-HV-Sorting")
 // or timestamp-only validation (MODE_TBV, "STM-TBV-Sorting").
 // ---------------------------------------------------------------------------
-template <class WL, int MODE>
+template <class WL, int MODE, bool PAIR>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
-    using TX = Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>;
+    using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>,
+                                  Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>>;
     // physical thread -> logical STM threads t, t + P, t + 2P, ... (P = the
     // grid's threads; P < T when the launch caps concurrency, p.max_threads)
     const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
@@ -242,7 +247,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams 
             if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
                 backoff = 0;
                 const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-                DirectCtx ctx{p.m.heap, 0, false};
+                DirectCtx ctx{p.m, 0, false};
                 uint32_t result = 0;
                 WL::body(ctx, p.w, gen::tx_key(p.seed, t, i), t, i, result);   // critical section
                 uint32_t s;
@@ -311,7 +316,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
                 ++cnt.c[S_ERRORS];
             } else if (lk.get_locks_and_tbv(m)) {
                 got = true;
-                DirectCtx ctx{m.heap, 0, false};
+                DirectCtx ctx{m, 0, false};
                 WL::body(ctx, p.w, x, t, i, result);
                 nw = ctx.nw;
                 if (ctx.bad) ++cnt.c[S_ERRORS];
@@ -386,15 +391,56 @@ __global__ void finish_kernel(unsigned long long* meta, const unsigned long long
 }
 
 // workload-defined initial heaps
-__global__ void init_heap_kernel(int workload, uint32_t* heap, uint64_t words)
+__global__ void init_heap_kernel(int workload, uint32_t* heap, uint64_t words, int vshift)
 {
     for (uint64_t k = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k < words;
          k += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
         uint32_t v = 0;
         if (workload == WL_RA || workload == WL_EB) v = static_cast<uint32_t>(k);
         else if (workload == WL_BANK) v = 1000u;
-        heap[k] = v;
+        heap[k << vshift] = v;
     }
+}
+
+// paired layout <-> plain word array (values only; lock halves untouched)
+__global__ void pack_kernel(uint32_t* plain, uint32_t* pairs, uint64_t words, int to_pairs)
+{
+    for (uint64_t k = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k < words;
+         k += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+        if (to_pairs) pairs[2 * k] = plain[k];
+        else plain[k] = pairs[2 * k];
+    }
+}
+
+// lock halves of the paired layout: zero them, or copy them out
+__global__ void lock_halves_kernel(uint32_t* pairs, uint64_t words, uint32_t* out)
+{
+    for (uint64_t k = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k < words;
+         k += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+        if (out) out[k] = pairs[2 * k + 1];
+        else pairs[2 * k + 1] = 0u;
+    }
+}
+
+static unsigned grid_for(uint64_t n)
+{
+    uint64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 32) blocks = 148 * 32;
+    return static_cast<unsigned>(blocks ? blocks : 1);
+}
+
+cudaError_t launch_pack(uint32_t* plain, uint32_t* pairs, uint64_t words, int to_pairs, cudaStream_t s)
+{
+    if (!words) return cudaSuccess;
+    pack_kernel<<<grid_for(words), 256, 0, s>>>(plain, pairs, words, to_pairs);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_lock_halves(uint32_t* pairs, uint64_t words, uint32_t* out, cudaStream_t s)
+{
+    if (!words) return cudaSuccess;
+    lock_halves_kernel<<<grid_for(words), 256, 0, s>>>(pairs, words, out);
+    return cudaGetLastError();
 }
 
 // ---------------------------------------------------------------------------
@@ -412,12 +458,10 @@ cudaError_t launch_finish(unsigned long long* meta, const unsigned long long* cl
     return cudaGetLastError();
 }
 
-cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, cudaStream_t s)
+cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, int vshift, cudaStream_t s)
 {
     if (!words) return cudaSuccess;
-    uint64_t blocks = (words + 255) / 256;
-    if (blocks > 148 * 32) blocks = 148 * 32;
-    init_heap_kernel<<<static_cast<unsigned>(blocks), 256, 0, s>>>(workload, heap, words);
+    init_heap_kernel<<<grid_for(words), 256, 0, s>>>(workload, heap, words, vshift);
     return cudaGetLastError();
 }
 
@@ -429,8 +473,14 @@ static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream
     if (grid == 0) return cudaSuccess;
     const dim3 g(static_cast<unsigned>(grid)), b(block);
     switch (kmode) {
-    case KMODE_HV: stm_kernel<WL, MODE_HV><<<g, b, 0, s>>>(kp); break;
-    case KMODE_TBV: stm_kernel<WL, MODE_TBV><<<g, b, 0, s>>>(kp); break;
+    case KMODE_HV:
+        if (kp.paired) stm_kernel<WL, MODE_HV, true><<<g, b, 0, s>>>(kp);
+        else stm_kernel<WL, MODE_HV, false><<<g, b, 0, s>>>(kp);
+        break;
+    case KMODE_TBV:
+        if (kp.paired) stm_kernel<WL, MODE_TBV, true><<<g, b, 0, s>>>(kp);
+        else stm_kernel<WL, MODE_TBV, false><<<g, b, 0, s>>>(kp);
+        break;
     case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     default: return cudaErrorInvalidValue;

@@ -3,6 +3,7 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 #include "gstm/tx.cuh"
+#include "gstm/tx_pair.cuh"
 #include "gstm/workloads.cuh"
 
 namespace gstm {
@@ -46,6 +47,7 @@ struct KParams {
     uint64_t seed;
     uint32_t prelock_vbv, k_lock, backoff_ns, snapshot_reuse, lock_pipeline;
     uint64_t max_threads;          // 0: one CUDA thread per STM thread; else cap (grid-stride)
+    uint32_t paired;               // paired layout (value | lock per u64, tx_pair.cuh)
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);
@@ -53,7 +55,9 @@ cudaError_t launch_finish(unsigned long long* meta, const unsigned long long* cl
 cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cudaStream_t s);
 cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt, cudaStream_t s);
 bool workload_check(int workload, const WlParams& w, uint64_t* footprint, int* descr_words);
-cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, cudaStream_t s);
+cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, int vshift, cudaStream_t s);
+cudaError_t launch_pack(uint32_t* plain, uint32_t* pairs, uint64_t words, int to_pairs, cudaStream_t s);
+cudaError_t launch_lock_halves(uint32_t* pairs, uint64_t words, uint32_t* out, cudaStream_t s);
 cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
                           cudaStream_t s);
 cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s);

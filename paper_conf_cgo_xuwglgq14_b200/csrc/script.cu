@@ -12,9 +12,9 @@
 
 namespace gstm {
 
-using ScriptTx = Tx<64, 64, 128>;
 constexpr int kMaxScriptTx = 8;
 
+template <class ScriptTx>
 __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out,
                               int n_tx)
 {
@@ -91,7 +91,8 @@ cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* 
                           cudaStream_t s)
 {
     if (n_tx > kMaxScriptTx) return cudaErrorInvalidValue;
-    script_kernel<<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    if (m.vshift) script_kernel<TxPair<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    else script_kernel<Tx<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
     return cudaGetLastError();
 }
 

@@ -30,7 +30,7 @@ STATUS = {0: "GSTM_OK", -1: "GSTM_EINVAL", -2: "GSTM_ENOMEM", -3: "GSTM_ECUDA", 
 
 # every symbol include/gstm.h declares (checked by tests/test_abi.py)
 EXPORTS = [
-    "gstm_create", "gstm_destroy", "gstm_last_error", "gstm_api_version", "gstm_default_params",
+    "gstm_create", "gstm_create_ex", "gstm_flags", "gstm_destroy", "gstm_last_error", "gstm_api_version", "gstm_default_params",
     "gstm_set_params", "gstm_get_params", "gstm_set_mode", "gstm_set_stream", "gstm_attach_heap",
     "gstm_heap_words", "gstm_heap_ptr", "gstm_init_heap", "gstm_write_heap", "gstm_read_heap",
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
@@ -87,6 +87,8 @@ def lib():
         u32, u64, i32 = C.c_uint32, C.c_uint64, C.c_int
         sig = {
             "gstm_create": (V, [u64, u32]),
+            "gstm_create_ex": (V, [u64, u32, u32]),
+            "gstm_flags": (u32, [V]),
             "gstm_destroy": (None, [V]),
             "gstm_last_error": (C.c_char_p, []),
             "gstm_api_version": (i32, []),
@@ -141,8 +143,12 @@ def _ptr(a: np.ndarray):
 
 
 # ---- function-style API with the C names --------------------------------
-def gstm_create(heap_words: int, lock_table_bits: int):
-    h = lib().gstm_create(heap_words, lock_table_bits)
+CREATE_PAIRED = 1
+
+
+def gstm_create(heap_words: int, lock_table_bits: int, flags: int = 0):
+    h = lib().gstm_create_ex(heap_words, lock_table_bits, flags) if flags else lib().gstm_create(heap_words,
+                                                                                                 lock_table_bits)
     if not h:
         raise GstmError(f"gstm_create: {last_error()}")
     return h
@@ -189,9 +195,13 @@ def _mode(m) -> int:
 class Gstm:
     """Owning wrapper of a gstm_t handle."""
 
-    def __init__(self, heap_words: int, lock_table_bits: int):
-        self.h = gstm_create(heap_words, lock_table_bits)
+    def __init__(self, heap_words: int, lock_table_bits: int, paired: bool = False):
+        """paired=True: GSTM_CREATE_PAIRED layout (each word next to its
+        version lock; needs heap_words <= 2^lock_table_bits)."""
+        self.h = None
+        self.h = gstm_create(heap_words, lock_table_bits, CREATE_PAIRED if paired else 0)
         self.bits = lock_table_bits
+        self.paired = paired
         self._attached = None
 
     def close(self) -> None:

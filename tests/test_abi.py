@@ -37,10 +37,15 @@ def test_library_is_sm100a_and_self_contained(so):
     assert "sm_100a" in out
     deps = subprocess.check_output(["ldd", so], text=True)
     assert "libcudart" not in deps          # static cudart: nothing to resolve on the GPU box
-    sass = subprocess.check_output(["cuobjdump", "-sass", "-fun", "_ZN4gstm10stm_kernelINS_6BankWLELi2EEEvNS_7KParamsE", so],
-                                   text=True)
+    sass = subprocess.check_output(["cuobjdump", "-sass", so], text=True)
+    funcs = dict(re.findall(r"Function : (\S+)\n(.*?)(?=\n\s*Function : |\Z)", sass, flags=re.S))
+    split = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb0EEEvNS_7KParamsE"]    # HV, paper layout
+    paired = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb1EEEvNS_7KParamsE"]   # HV, paired layout
     # the hot path is made of L2 atomics / strong gpu-scope accesses
-    assert "ATOMG.E.OR.STRONG.GPU" in sass and "LDG.E.STRONG.GPU" in sass
+    assert "ATOMG.E.OR.STRONG.GPU" in split and "LDG.E.STRONG.GPU" in split
+    assert "ATOMG.E.OR.64.STRONG.GPU" in paired and "LDG.E.64.STRONG.GPU" in paired
+    # one MEMBAR (the l.82 release fence) in the paper layout, none paired
+    assert split.count("MEMBAR") == 1 and paired.count("MEMBAR") == 0
 
 
 def test_loads_and_host_only_calls(so):

@@ -89,7 +89,8 @@ def main():
         mode = kv.pop("mode", "auto")
         pad_mb = int(kv.pop("pad_mb", 0))       # shift where the handle's buffers land
         pad = torch.empty(pad_mb << 18, dtype=torch.float32, device="cuda") if pad_mb else None
-        g = G.Gstm(shp["words"], bits)
+        paired = bool(int(kv.pop("paired", 0)))
+        g = G.Gstm(shp["words"], bits, paired=paired)
         if flush is None:
             flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
         g.set_workload_defaults(wl, **shp["params"], **{k: int(v) for k, v in kv.items()})
