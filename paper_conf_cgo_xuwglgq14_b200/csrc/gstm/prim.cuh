@@ -29,6 +29,11 @@
 #define GSTM_STRICT_FENCES 0
 #endif
 
+// nanoseconds a reader sleeps between re-reads of a locked word (A3.l27-29)
+#ifndef GSTM_SPIN_NS
+#define GSTM_SPIN_NS 32
+#endif
+
 namespace gstm {
 namespace prim {
 

@@ -225,7 +225,7 @@ struct Tx {
         uint32_t spins = 0;
         while (vl & 1u) {                                            // l.29
             if (++spins > m.spin_cap) { opaque = false; break; }
-            __nanosleep(32);
+            if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
             vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));      // l.28
         }
         n_spin += spins;

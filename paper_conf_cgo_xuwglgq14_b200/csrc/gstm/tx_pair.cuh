@@ -99,7 +99,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL> {
         uint32_t spins = 0;
         while (hi(pv) & 1u) {
             if (++spins > m.spin_cap) { opaque = false; break; }
-            __nanosleep(32);
+            if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
             pv = prim::ld_relaxed_u64(m.pair_ptr(a));
         }
         n_spin += spins;

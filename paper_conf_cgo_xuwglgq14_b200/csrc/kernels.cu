@@ -119,18 +119,26 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
 {
     using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>,
                                   Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>>;
-    // physical thread -> logical STM threads t, t + P, t + 2P, ... (P = the
-    // grid's threads; P < T when the launch caps concurrency, p.max_threads)
+    // The grid is persistent (host sizes it to what fits on the chip, or to
+    // p.max_threads): lane g starts with STM thread t = g; a lane that has run
+    // all K transactions of its thread takes the next unstarted thread from a
+    // global counter (one warp-aggregated atomic), so no lane idles while
+    // work remains and the program order of each STM thread is kept.
     const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
     uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
     if (p.K == 0) t = p.T;
     const Meta m = p.m;
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
+    unsigned long long* work = p.meta + M_WORK;
     Counters cnt;
     TX tx;
     tx.reset_stats();
-    uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0;
+    uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
+    // stage 0: start (or re-execute) transaction (t, i); stage 1: its body
+    // ran and it waits for its locks (a lost lock round is retried in the
+    // warp's next iteration, after the winners committed)
+    int stage = 0;
     bool timed_out = false, have_snap = false, lock_aborted = false;
 
     while (__any_sync(FULL, t < p.T)) {
@@ -141,76 +149,92 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
         have_snap = false;
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-        uint32_t result = 0;
-        if (act) {
+        bool done = false, skip = false;
+        if (act && stage == 0) {
             ++cnt.c[S_ATTEMPTS];
+            result = 0;
             const uint64_t x = gen::tx_key(p.seed, t, i);
             tx.begin(snap);                                           // TXBegin l.2-3
             StmCtx<TX> ctx{tx, m, MODE};
             WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
-        }
-        bool done = false, skip = false;
-        bool pending = act && tx.opaque && !tx.read_only();
-        if (act && !tx.opaque) {
-            if (tx.overflow) { ++cnt.c[S_ERRORS]; skip = true; }    // sticky ELOGOVF, give up this tx
-            else ++cnt.c[S_AB_OPACITY];                              // Figure 1 / Q11
-        }
-        if (act && tx.opaque && tx.read_only()) {                     // l.68: linearized at snapshot
-            if (p.tx_stamp) {
-                p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
-                p.tx_result[tx_id] = result;
-            }
-            ++cnt.c[S_COMMITS_RO];
-            done = true;
-        }
-        // warp-collective TXCommit (l.67-85)
-        for (uint32_t round = 0; __any_sync(FULL, pending); ++round) {
-            bool got = false;
-            if (pending) {
-                // the pipelined round (§6.4) only for a transaction's first
-                // round of an execution that never lost its locks before, so
-                // every retry uses the sequential sorted acquisition
-                const bool pipelined = p.lock_pipeline && round == 0 && !lock_aborted;
-                const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
-                if (r == C_OK) {
-                    got = true;
-                    tx.writeback(m);                                  // l.79-82
-                } else if (r == C_LOCK) {
-                    ++cnt.c[S_LOCK_RETRIES];                          // l.73-74 retry next round
-                    if (p.k_lock && round + 1 >= p.k_lock) {
-                        pending = false;
-                        lock_aborted = true;
-                        ++cnt.c[S_AB_LOCK];
-                    }
-                } else {
-                    pending = false;
-                    ++cnt.c[r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV)];
-                }
-            }
-            unsigned gm;
-            const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
-            if (gm) have_snap = true;
-            if (got) {
-                tx.release_and_update(m, stamp);                      // l.84
+            if (!tx.opaque) {
+                if (tx.overflow) { ++cnt.c[S_ERRORS]; skip = true; }  // sticky ELOGOVF, give up this tx
+                else ++cnt.c[S_AB_OPACITY];                          // Figure 1 / Q11
+            } else if (tx.read_only()) {                              // l.68: linearized at snapshot
                 if (p.tx_stamp) {
-                    p.tx_stamp[tx_id] = stamp - clock_begin;
+                    p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
                     p.tx_result[tx_id] = result;
                 }
-                ++cnt.c[S_COMMITS];
-                pending = false;
+                ++cnt.c[S_COMMITS_RO];
                 done = true;
+            } else {
+                stage = 1;
+                tries = 0;
             }
         }
+        // No lane may take a lock while another lane of its warp can still be
+        // spinning on a lock in its read phase (A3.l27-29): under independent
+        // thread scheduling the locker would then wait for the spinner at the
+        // warp barrier in warp_stamp while the spinner waits for its lock.
+        __syncwarp();
+        // one warp-collective TXCommit round per iteration (l.67-85)
+        bool got = false;
+        if (act && stage == 1) {
+            // the pipelined round (§6.4) only for the first round of an
+            // execution that never lost its locks before: every retry uses the
+            // sequential sorted acquisition
+            const bool pipelined = p.lock_pipeline && tries == 0 && !lock_aborted;
+            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
+            if (r == C_OK) {
+                got = true;
+                tx.writeback(m);                                      // l.79-82
+            } else if (r == C_LOCK) {
+                ++cnt.c[S_LOCK_RETRIES];                              // l.73-74: retry next iteration
+                if (p.k_lock && ++tries >= p.k_lock) {
+                    stage = 0;
+                    lock_aborted = true;
+                    ++cnt.c[S_AB_LOCK];
+                }
+            } else {
+                stage = 0;
+                ++cnt.c[r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV)];
+            }
+        }
+        unsigned gm;
+        const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
+        if (gm) have_snap = true;
+        if (got) {
+            tx.release_and_update(m, stamp);                          // l.84
+            if (p.tx_stamp) {
+                p.tx_stamp[tx_id] = stamp - clock_begin;
+                p.tx_result[tx_id] = result;
+            }
+            ++cnt.c[S_COMMITS];
+            done = true;
+        }
         if (done || skip) {
-            if (++i >= p.K) { i = 0; t += P; }
+            stage = 0;
+            ++i;
             backoff = 0;
             lock_aborted = false;
-        } else if (p.backoff_ns) {
-            // warp-uniform exponential backoff after an abort (all lanes sleep
-            // together: per-lane delays cannot work under SIMT)
-            if (__any_sync(FULL, act)) {
-                backoff = backoff ? min(backoff * 2u, 64u * p.backoff_ns) : p.backoff_ns;
-                __nanosleep(backoff);
+        } else if (p.backoff_ns && act && stage == 0) {
+            // exponential backoff after an abort (P:111 argues per-lane
+            // delays cannot work under SIMT; lanes here sleep independently
+            // under independent thread scheduling)
+            backoff = backoff ? min(backoff * 2u, 64u * p.backoff_ns) : p.backoff_ns;
+            __nanosleep(backoff);
+        }
+        // refill: lanes whose STM thread ran all K transactions take the next one
+        const bool need = t < p.T && i >= p.K;
+        const unsigned nm = __ballot_sync(FULL, need);
+        if (nm) {
+            const int leader = __ffs(nm) - 1;
+            unsigned long long base = 0;
+            if (static_cast<int>(prim::lane_id()) == leader) base = atomicAdd(work, static_cast<unsigned long long>(__popc(nm)));
+            base = __shfl_sync(FULL, base, leader);
+            if (need) {
+                t = P + base + __popc(nm & prim::lanemask_lt());
+                i = 0;
             }
         }
     }
@@ -374,6 +398,7 @@ __global__ void prepare_kernel(unsigned long long* meta, const unsigned long lon
     meta[M_CLOCK_BEGIN] = *clock;
     meta[M_DEADLINE] = now + timeout_ns;
     meta[M_T_START] = now;
+    meta[M_WORK] = 0;
     for (int k = 0; k < S_NSTATS; ++k) meta[M_STATS + k] = 0;
     *reinterpret_cast<uint32_t*>(meta + M_ERR) = 0;
     *reinterpret_cast<uint32_t*>(meta + M_CGL_LOCK) = 0;
@@ -465,6 +490,32 @@ cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, int v
     return cudaGetLastError();
 }
 
+// persistent grid for a kernel: the blocks that fit on the chip at once
+template <class K>
+static uint64_t resident_blocks(K kernel, int block)
+{
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, 0) != cudaSuccess || per_sm < 1) per_sm = 1;
+    return static_cast<uint64_t>(per_sm) * (sms > 0 ? sms : 148);
+}
+
+template <class K>
+static cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s)
+{
+    uint64_t grid = (kp.T + block - 1) / block;
+    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block));
+    if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
+    if (grid == 0) return cudaSuccess;
+    kernel<<<static_cast<unsigned>(grid), block, 0, s>>>(kp);
+    return cudaGetLastError();
+}
+
 template <class WL>
 static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
 {
@@ -474,13 +525,11 @@ static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream
     const dim3 g(static_cast<unsigned>(grid)), b(block);
     switch (kmode) {
     case KMODE_HV:
-        if (kp.paired) stm_kernel<WL, MODE_HV, true><<<g, b, 0, s>>>(kp);
-        else stm_kernel<WL, MODE_HV, false><<<g, b, 0, s>>>(kp);
-        break;
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s)
+                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s);
     case KMODE_TBV:
-        if (kp.paired) stm_kernel<WL, MODE_TBV, true><<<g, b, 0, s>>>(kp);
-        else stm_kernel<WL, MODE_TBV, false><<<g, b, 0, s>>>(kp);
-        break;
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s)
+                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s);
     case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     default: return cudaErrorInvalidValue;
