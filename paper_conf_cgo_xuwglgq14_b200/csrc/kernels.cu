@@ -72,28 +72,30 @@ __device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool g
     return static_cast<uint32_t>(base) + __popc(gm & prim::lanemask_lt()) + 1u;
 }
 
+// Statistics counters: one block-shared array (shared-memory atomics on the
+// rare events), flushed to the launch's counters with one global atomic per
+// counter per block.  Kept out of registers (they cost occupancy).
 struct Counters {
-    uint32_t c[S_NSTATS];
-    __device__ __forceinline__ Counters()
+    unsigned long long* sh;
+    bool error = false;
+    __device__ __forceinline__ void inc(int k, uint32_t v = 1u)
     {
-#pragma unroll
-        for (int k = 0; k < S_NSTATS; ++k) c[k] = 0;
+        if (v) atomicAdd(&sh[k], static_cast<unsigned long long>(v));
+        if (k == S_ERRORS) error = true;
     }
 };
 
-// warp reduce -> shared -> one global atomic per counter per block
-__device__ __forceinline__ void flush_counters(const Counters& cnt, unsigned long long* stats)
+#define GSTM_COUNTERS(name)                                                 \
+    __shared__ unsigned long long name##_sh[S_NSTATS];                      \
+    if (threadIdx.x < S_NSTATS) name##_sh[threadIdx.x] = 0;                 \
+    __syncthreads();                                                        \
+    Counters name{name##_sh}
+
+// block totals -> one global atomic per counter per block
+__device__ __forceinline__ void flush_counters(Counters& cnt, unsigned long long* stats)
 {
-    __shared__ unsigned long long sh[S_NSTATS];
-    if (threadIdx.x < S_NSTATS) sh[threadIdx.x] = 0;
     __syncthreads();
-#pragma unroll
-    for (int k = 0; k < S_NSTATS; ++k) {
-        const uint32_t v = __reduce_add_sync(FULL, cnt.c[k]);
-        if (prim::lane_id() == 0 && v) atomicAdd(&sh[k], static_cast<unsigned long long>(v));
-    }
-    __syncthreads();
-    if (threadIdx.x < S_NSTATS && sh[threadIdx.x]) atomicAdd(stats + threadIdx.x, sh[threadIdx.x]);
+    if (threadIdx.x < S_NSTATS && cnt.sh[threadIdx.x]) atomicAdd(stats + threadIdx.x, cnt.sh[threadIdx.x]);
 }
 
 __device__ __forceinline__ void set_err(unsigned long long* meta, uint32_t bits)
@@ -131,7 +133,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
     unsigned long long* work = p.meta + M_WORK;
-    Counters cnt;
+    GSTM_COUNTERS(cnt);
     TX tx;
     tx.reset_stats();
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
@@ -151,21 +153,21 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
         bool done = false, skip = false;
         if (act && stage == 0) {
-            ++cnt.c[S_ATTEMPTS];
+            cnt.inc(S_ATTEMPTS);
             result = 0;
             const uint64_t x = gen::tx_key(p.seed, t, i);
             tx.begin(snap);                                           // TXBegin l.2-3
             StmCtx<TX> ctx{tx, m, MODE};
             WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
             if (!tx.opaque) {
-                if (tx.overflow) { ++cnt.c[S_ERRORS]; skip = true; }  // sticky ELOGOVF, give up this tx
-                else ++cnt.c[S_AB_OPACITY];                          // Figure 1 / Q11
+                if (tx.overflow) { cnt.inc(S_ERRORS); skip = true; }  // sticky ELOGOVF, give up this tx
+                else cnt.inc(S_AB_OPACITY);                          // Figure 1 / Q11
             } else if (tx.read_only()) {                              // l.68: linearized at snapshot
                 if (p.tx_stamp) {
                     p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
                     p.tx_result[tx_id] = result;
                 }
-                ++cnt.c[S_COMMITS_RO];
+                cnt.inc(S_COMMITS_RO);
                 done = true;
             } else {
                 stage = 1;
@@ -189,15 +191,15 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 got = true;
                 tx.writeback(m);                                      // l.79-82
             } else if (r == C_LOCK) {
-                ++cnt.c[S_LOCK_RETRIES];                              // l.73-74: retry next iteration
+                cnt.inc(S_LOCK_RETRIES);                              // l.73-74: retry next iteration
                 if (p.k_lock && ++tries >= p.k_lock) {
                     stage = 0;
                     lock_aborted = true;
-                    ++cnt.c[S_AB_LOCK];
+                    cnt.inc(S_AB_LOCK);
                 }
             } else {
                 stage = 0;
-                ++cnt.c[r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV)];
+                cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
             }
         }
         unsigned gm;
@@ -209,7 +211,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 p.tx_stamp[tx_id] = stamp - clock_begin;
                 p.tx_result[tx_id] = result;
             }
-            ++cnt.c[S_COMMITS];
+            cnt.inc(S_COMMITS);
             done = true;
         }
         if (done || skip) {
@@ -238,11 +240,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             }
         }
     }
-    cnt.c[S_POSTVAL] = tx.n_postval;
-    cnt.c[S_VBV] = tx.n_vbv;
-    cnt.c[S_SPINS] = tx.n_spin;
+    cnt.inc(S_POSTVAL, tx.n_postval);
+    cnt.inc(S_VBV, tx.n_vbv);
+    cnt.inc(S_SPINS, tx.n_spin);
     if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
+    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
     flush_counters(cnt, p.meta + M_STATS);
 }
 
@@ -260,14 +262,14 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams 
     uint32_t* lock = reinterpret_cast<uint32_t*>(p.meta + M_CGL_LOCK);
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
-    Counters cnt;
+    GSTM_COUNTERS(cnt);
     uint32_t i = 0, iter = 0, backoff = 0;
     bool timed_out = false;
     while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
         const bool act = t < p.T;
         if (act) {
-            ++cnt.c[S_ATTEMPTS];
+            cnt.inc(S_ATTEMPTS);
             if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
                 backoff = 0;
                 const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
@@ -277,18 +279,18 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams 
                 uint32_t s;
                 if (ctx.nw) {
                     s = static_cast<uint32_t>(prim::atom_add_relaxed64(p.m.clock, 1ull)) + 1u - clock_begin;
-                    ++cnt.c[S_COMMITS];
+                    cnt.inc(S_COMMITS);
                 } else {
                     s = 0x80000000u | (static_cast<uint32_t>(prim::ld_relaxed64(p.m.clock)) - clock_begin);
-                    ++cnt.c[S_COMMITS_RO];
+                    cnt.inc(S_COMMITS_RO);
                 }
-                if (ctx.bad) ++cnt.c[S_ERRORS];
+                if (ctx.bad) cnt.inc(S_ERRORS);
                 if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
                 prim::fence_release();
                 prim::st_relaxed(lock, 0u);                           // Scheme #3 l.15
                 if (++i >= p.K) { i = 0; t += P; }
             } else {
-                ++cnt.c[S_LOCK_RETRIES];
+                cnt.inc(S_LOCK_RETRIES);
                 // optional per-thread exponential backoff (test-and-test-and-set
                 // with backoff; the paper's Scheme #3 has none: backoff_ns = 0)
                 if (p.backoff_ns) {
@@ -299,7 +301,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams 
         }
     }
     if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_INVALID);
+    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_INVALID);
     flush_counters(cnt, p.meta + M_STATS);
 }
 
@@ -320,7 +322,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
     const Meta m = p.m;
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
-    Counters cnt;
+    GSTM_COUNTERS(cnt);
     TX lk;
     uint32_t i = 0, iter = 0;
     bool timed_out = false;
@@ -332,21 +334,21 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
         int nw = 0;
         uint32_t result = 0;
         if (act) {
-            ++cnt.c[S_ATTEMPTS];
+            cnt.inc(S_ATTEMPTS);
             const uint64_t x = gen::tx_key(p.seed, t, i);
             lk.begin(0);
             WL::fgl_words(p.w, x, t, i, [&](uint32_t w) { lk.insert_lock((m.lock_of(w) << 2) | 2u); });
             if (lk.overflow) {
-                ++cnt.c[S_ERRORS];
+                cnt.inc(S_ERRORS);
             } else if (lk.get_locks_and_tbv(m)) {
                 got = true;
                 DirectCtx ctx{m, 0, false};
                 WL::body(ctx, p.w, x, t, i, result);
                 nw = ctx.nw;
-                if (ctx.bad) ++cnt.c[S_ERRORS];
+                if (ctx.bad) cnt.inc(S_ERRORS);
                 prim::fence_release();          // in-place writes before stamp and unlock
             } else {
-                ++cnt.c[S_LOCK_RETRIES];
+                cnt.inc(S_LOCK_RETRIES);
             }
         }
         unsigned gm;
@@ -356,10 +358,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
             uint32_t s;
             if (nw > 0) {
                 s = stamp - clock_begin;
-                ++cnt.c[S_COMMITS];
+                cnt.inc(S_COMMITS);
             } else {
                 s = 0x80000000u | (static_cast<uint32_t>(prim::ld_acquire64(m.clock)) - clock_begin);
-                ++cnt.c[S_COMMITS_RO];
+                cnt.inc(S_COMMITS_RO);
             }
             if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
             if (GSTM_STRICT_FENCES) prim::fence_release();
@@ -372,7 +374,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams 
         }
     }
     if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.c[S_ERRORS] != 0) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
+    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
     flush_counters(cnt, p.meta + M_STATS);
 }
 
