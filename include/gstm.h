@@ -192,6 +192,13 @@ int gstm_stats(gstm_t* h, gstm_stats_t* out);
  * the first error any of them reported. */
 int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches);
 int gstm_reset_stats_total(gstm_t* h);
+/* Per-phase time breakdown of the STM loop since gstm_reset_stats_total
+ * (the paper's Figure 5 study): SM cycles summed over warps for
+ * out[0] TXBegin/snapshot, [1] transaction body (reads, PostValidation, lock
+ * spins), [2] lock acquisition + validation, [3] commit stamp, [4] write-back
+ * and release, [5] loop/refill.  Non-zero only in a library built with
+ * -DGSTM_PHASE_TIMING=1 (GSTM_DEFINES); writes min(n, 8) entries. */
+int gstm_phase_cycles(gstm_t* h, uint64_t* out, int n);
 /* Verify mode (params.verify = 1): stamps[tx_id] = commit stamp - clock_begin
  * (1..C) for an update tx, or 0x80000000 | (snapshot - clock_begin) for a
  * read-only tx (linearised after that stamp); results[tx_id] = the

@@ -522,7 +522,17 @@ int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches)
 int gstm_reset_stats_total(gstm_t* h)
 {
     if (!h) { set_error("gstm_reset_stats_total: NULL"); return GSTM_EINVAL; }
-    CUDA_TRY(cudaMemsetAsync(h->meta + M_TOTALS, 0, (M_T_ERR + 1 - M_TOTALS) * 8, h->stream));
+    CUDA_TRY(cudaMemsetAsync(h->meta + M_TOTALS, 0, (M_PHASE + 8 - M_TOTALS) * 8, h->stream));
+    return GSTM_OK;
+}
+
+int gstm_phase_cycles(gstm_t* h, uint64_t* out, int n)
+{
+    if (!h || !out || n < 0) { set_error("gstm_phase_cycles: bad argument"); return GSTM_EINVAL; }
+    unsigned long long ph[8];
+    CUDA_TRY(cudaMemcpyAsync(ph, h->meta + M_PHASE, sizeof(ph), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    for (int k = 0; k < n && k < 8; ++k) out[k] = ph[k];
     return GSTM_OK;
 }
 

@@ -112,6 +112,34 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
     return __shfl_sync(FULL, late, 0);
 }
 
+// Per-phase time breakdown of the transaction loop (the Figure 5 study of
+// P:329-333): build with -DGSTM_PHASE_TIMING=1; lane 0 of every
+// warp adds the SM cycles each phase of each iteration took (after a warp
+// barrier, so the time is the warp's) to meta[M_PHASE + k].
+#ifndef GSTM_PHASE_TIMING
+#define GSTM_PHASE_TIMING 0
+#endif
+enum { PH_BEGIN = 0, PH_BODY, PH_LOCK, PH_STAMP, PH_RELEASE, PH_LOOP, PH_N };
+#if GSTM_PHASE_TIMING
+#define PHASE_DECL() unsigned long long ph_[PH_N] = {0, 0, 0, 0, 0, 0}; long long ph_t_ = clock64()
+#define PHASE_MARK(k)                                                        \
+    do {                                                                     \
+        __syncwarp();                                                        \
+        const long long now_ = clock64();                                    \
+        ph_[k] += static_cast<unsigned long long>(now_ - ph_t_);            \
+        ph_t_ = now_;                                                        \
+    } while (0)
+#define PHASE_FLUSH(dst)                                                     \
+    do {                                                                     \
+        if (prim::lane_id() == 0)                                            \
+            for (int k_ = 0; k_ < PH_N; ++k_) atomicAdd((dst) + k_, ph_[k_]); \
+    } while (0)
+#else
+#define PHASE_DECL() do {} while (0)
+#define PHASE_MARK(k) do {} while (0)
+#define PHASE_FLUSH(dst) do {} while (0)
+#endif
+
 // ---------------------------------------------------------------------------
 // STM kernel: GPU-STM with hierarchical validation (MODE_HV, "STM-HV-Sorting")
 // or timestamp-only validation (MODE_TBV, "STM-TBV-Sorting").
@@ -142,6 +170,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     // warp's next iteration, after the winners committed)
     int stage = 0;
     bool timed_out = false, have_snap = false, lock_aborted = false;
+    PHASE_DECL();
 
     while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
@@ -150,6 +179,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         // this warp's own last commit (p.snapshot_reuse)
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
         have_snap = false;
+        PHASE_MARK(PH_BEGIN);
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
         bool done = false, skip = false;
         if (act && stage == 0) {
@@ -174,6 +204,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 tries = 0;
             }
         }
+        PHASE_MARK(PH_BODY);
         // No lane may take a lock while another lane of its warp can still be
         // spinning on a lock in its read phase (A3.l27-29): under independent
         // thread scheduling the locker would then wait for the spinner at the
@@ -202,9 +233,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
             }
         }
+        PHASE_MARK(PH_LOCK);
         unsigned gm;
         const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
         if (gm) have_snap = true;
+        PHASE_MARK(PH_STAMP);
         if (got) {
             tx.release_and_update(m, stamp);                          // l.84
             if (p.tx_stamp) {
@@ -214,6 +247,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             cnt.inc(S_COMMITS);
             done = true;
         }
+        PHASE_MARK(PH_RELEASE);
         if (done || skip) {
             stage = 0;
             ++i;
@@ -239,7 +273,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 i = 0;
             }
         }
+        PHASE_MARK(PH_LOOP);
     }
+    PHASE_FLUSH(p.meta + M_PHASE);
     cnt.inc(S_POSTVAL, tx.n_postval);
     cnt.inc(S_VBV, tx.n_vbv);
     cnt.inc(S_SPINS, tx.n_spin);

@@ -28,6 +28,7 @@ enum {
     M_T_LAUNCHES = 96 + S_NSTATS,      // launches since reset
     M_T_NS = 97 + S_NSTATS,            // device ns (globaltimer) since reset
     M_T_ERR = 98 + S_NSTATS,           // OR of the error bits since reset
+    M_PHASE = 112,                     // 8 phase-cycle accumulators (GSTM_PHASE_TIMING builds)
     M_WORK = 120,                      // next unstarted STM thread (persistent grid), own line
     M_WORDS = 128
 };

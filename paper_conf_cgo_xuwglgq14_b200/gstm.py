@@ -34,7 +34,7 @@ EXPORTS = [
     "gstm_set_params", "gstm_get_params", "gstm_set_mode", "gstm_set_stream", "gstm_attach_heap",
     "gstm_heap_words", "gstm_heap_ptr", "gstm_init_heap", "gstm_write_heap", "gstm_read_heap",
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
-    "gstm_stats_total", "gstm_reset_stats_total",
+    "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
     "gstm_lock_log", "gstm_ubench",
 ]
@@ -111,6 +111,7 @@ def lib():
             "gstm_stats": (i32, [V, P(gstm_stats_t)]),
             "gstm_stats_total": (i32, [V, P(gstm_stats_t), P(u64)]),
             "gstm_reset_stats_total": (i32, [V]),
+            "gstm_phase_cycles": (i32, [V, V, i32]),
             "gstm_read_tx_log": (i32, [V, V, V, u64]),
             "gstm_run_host": (i32, [V, i32, V, V, u64, u64, u32, u64, P(gstm_stats_t)]),
             "gstm_descr_words": (i32, [V, i32]),
@@ -314,6 +315,14 @@ class Gstm:
         if check:
             _check(rc, "gstm_stats_total")
         return s, n.value
+
+    PHASES = ["begin", "body", "lock", "stamp", "release", "loop"]
+
+    def phase_cycles(self) -> dict:
+        """Figure-5-style breakdown (needs a GSTM_PHASE_TIMING build)."""
+        out = np.zeros(8, dtype=np.uint64)
+        _check(lib().gstm_phase_cycles(self.h, _ptr(out), 8), "gstm_phase_cycles")
+        return {k: int(out[i]) for i, k in enumerate(self.PHASES)}
 
     def reset_stats_total(self) -> None:
         _check(lib().gstm_reset_stats_total(self.h), "gstm_reset_stats_total")

@@ -128,6 +128,11 @@ def main():
         line = {"wl": a.wl, "variant": var, "T": T, "K": K, "bits": bits, "mode_used": G.MODE_NAMES[st.mode_used],
                 "tx_per_s": done / (tot_ms * 1e-3), "ms_per_launch": tot_ms / a.steps,
                 "abort_ratio": ab / max(1, ab + done), "stats": agg}
+        ph = g.phase_cycles()
+        if any(ph.values()):
+            tot = sum(ph.values())
+            line["phases_frac"] = {k: v / tot for k, v in ph.items()}
+            line["phase_cycles"] = ph
         print(json.dumps(line), flush=True)
         g.close()
 
