@@ -50,6 +50,7 @@ def parse(argv=None):
     ap.add_argument("--layout", default="paired", choices=["paired", "split"])
     ap.add_argument("--prelock", type=int, default=None,
                     help="pre-lock VBV (A3.l71); default 0 on the paired layout, 1 on the split one")
+    ap.add_argument("--k-lock", type=int, default=1, help="lock rounds before a transaction re-executes")
     ap.add_argument("--threads", type=int, default=THREADS)
     ap.add_argument("--tx-per-thread", type=int, default=TX_PER_THREAD)
     ap.add_argument("--no-cgl", action="store_true", help="skip the CGL/FGL baselines and the variant table")
@@ -89,6 +90,8 @@ class Variant:
         s = f"{self.mode}/{self.layout}"
         if self.mode in ("hv", "auto") and self.prelock != (0 if self.layout == "paired" else 1):
             s += f"/prelock={self.prelock}"
+        for k, v in sorted(self.params.items()):
+            s += f"/{k}={v}"
         return s
 
     def handle(self, G, stream):
@@ -117,7 +120,10 @@ class Variant:
 
 
 def headline_variant(args) -> Variant:
-    return Variant(args.mode, args.layout, args.prelock)
+    # k_lock = 1: a transaction that loses a lock round re-executes with fresh
+    # reads instead of retrying the commit with stale ones (P:325 leaves the
+    # number of attempts open; DESIGN.md §7.3 ablation)
+    return Variant(args.mode, args.layout, args.prelock, k_lock=args.k_lock)
 
 
 def config(args, label="hv/paired"):
