@@ -46,7 +46,7 @@ def parse(argv=None):
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
-    ap.add_argument("--mode", default="hv", choices=["auto", "hv", "tbv", "fgl", "cgl"])
+    ap.add_argument("--mode", default="hv", choices=["auto", "hv", "tbv", "fgl", "cgl", "hv_backoff", "vbv"])
     ap.add_argument("--layout", default="paired", choices=["paired", "split"])
     ap.add_argument("--prelock", type=int, default=None,
                     help="pre-lock VBV (A3.l71); default 0 on the paired layout, 1 on the split one")
@@ -88,7 +88,7 @@ class Variant:
     @property
     def name(self) -> str:
         s = f"{self.mode}/{self.layout}"
-        if self.mode in ("hv", "auto") and self.prelock != (0 if self.layout == "paired" else 1):
+        if self.mode in ("hv", "auto", "hv_backoff") and self.prelock != (0 if self.layout == "paired" else 1):
             s += f"/prelock={self.prelock}"
         for k, v in sorted(self.params.items()):
             s += f"/{k}={v}"
@@ -109,12 +109,12 @@ class Variant:
         if self.layout == "paired":
             upd = {"ld": 2, "atom": 2, "st": 2}      # 2 pair loads; 2 atom.or.b64 (lock + value); 2 pair stores
             ro = {"ld": 2, "atom": 0, "st": 0}
-            if mode_used == "hv" and self.prelock:
+            if mode_used in ("hv", "hv_backoff") and self.prelock:
                 upd = dict(upd, ld=4)
         else:
             upd = {"ld": 4, "atom": 2, "st": 4}      # 2 values + 2 lock words; 2 atom.or; 2 write-back + 2 release
             ro = {"ld": 4, "atom": 0, "st": 0}
-            if mode_used == "hv" and self.prelock:
+            if mode_used in ("hv", "hv_backoff") and self.prelock:
                 upd = dict(upd, ld=6)                 # + pre-lock VBV of the 2 values (A3.l71)
         return upd, ro
 
@@ -318,16 +318,18 @@ def roofline_l2(G, var: Variant, mode_used, tot, t_ms, steps):
             "model": "time = sum over op classes of count / measured rate (one shared L2 request pipeline)"}
 
 
-def cgl_baseline(G, stream, T, seed):
+def cgl_baseline(G, stream, T, seed, mode="cgl"):
     """CGL serialises every transaction, so its rate depends on how many
     threads fight for the one lock, not on the batch size.  Probe the paper's
     Scheme #3 (backoff 0) and test-and-test-and-set with exponential backoff
     at several thread counts and divide by the FASTEST (the most favourable
-    baseline), then time it on a bounded sample of ~0.5 s."""
-    g = Variant("cgl").handle(G, stream)
+    baseline), then time it on a bounded sample of ~0.5 s.  mode="vbv": the
+    same for STM-VBV, whose writers are serialised by one sequence lock
+    (backoff does not apply)."""
+    g = Variant(mode).handle(G, stream)
     probes = {}
     for Tc in (148 * 32, 1 << 14, 1 << 16, 1 << 18):
-        for bo in (0, 256):
+        for bo in ((0, 256) if mode == "cgl" else (0,)):
             g.set_params(backoff_ns=bo)
             probes[(Tc, bo)] = g.run("bank", Tc, max(1, (1 << 14) // Tc), seed + 11 + bo).tx_per_s
     (Tc, bo) = max(probes, key=probes.get)
@@ -338,7 +340,7 @@ def cgl_baseline(G, stream, T, seed):
     return {"value": st.tx_per_s, "unit": UNIT, "threads": Tc, "tx_per_thread": Kc, "backoff_ns": bo,
             "probe_tx_per_s": {f"T={k[0]},backoff={k[1]}": v for k, v in probes.items()},
             "sample": f"{Tc} threads x {Kc} tx at the fastest probed CGL configuration",
-            "elapsed_ms": st.elapsed_ms, "kernel": "cgl_kernel<BankWL>"}
+            "elapsed_ms": st.elapsed_ms, "abort_ratio": st.abort_ratio, "kernel": f"{mode}_kernel<BankWL>"}
 
 
 def variant_table(G, stream, flush, T, K, seed, variants, steps=8, warmup=3):
@@ -439,9 +441,11 @@ def run_native(args):
         g2.close()
         if not args.no_cgl:
             extra["cgl"] = cgl_baseline(G, stream, T, seed0)
+            extra["stm_vbv"] = cgl_baseline(G, stream, T, seed0, mode="vbv")
             table = [Variant("auto", "split"), Variant("tbv", "split"), Variant("hv", "split"),
-                     Variant("tbv", "paired"), Variant("hv", "paired", prelock=1), Variant("fgl", "split"),
-                     Variant("fgl", "paired")]
+                     Variant("tbv", "paired"), Variant("hv", "paired", prelock=1),
+                     Variant("hv_backoff", "split"), Variant("hv_backoff", "paired", k_lock=1),
+                     Variant("fgl", "split"), Variant("fgl", "paired")]
             extra["variants"] = variant_table(G, stream, flush, T, K, seed0,
                                               [v for v in table if v.name != var.name])
             fgl = [v for k, v in extra["variants"].items() if k.startswith("fgl")]

@@ -60,8 +60,19 @@ enum gstm_workload { GSTM_WL_RA = 0, GSTM_WL_BANK = 1, GSTM_WL_HT = 2, GSTM_WL_E
  *   TBV  = STM-TBV-Sorting (timestamp validation only);
  *   CGL  = coarse-grain lock baseline, Scheme #3 of Algorithm 1;
  *   FGL  = fine-grain lock baseline (sorted per-stripe locks; P:288 notes the
- *          paper did not implement it). */
-enum gstm_mode { GSTM_MODE_AUTO = 0, GSTM_MODE_HV = 1, GSTM_MODE_TBV = 2, GSTM_MODE_CGL = 3, GSTM_MODE_FGL = 4 };
+ *          paper did not implement it);
+ *   HV_BACKOFF = STM-HV-Backoff: HV with locks in encounter order;
+ *          the first lock attempt is made by all lanes of a warp in parallel,
+ *          lanes that failed retry one at a time while the others wait;
+ *   VBV  = STM-VBV: NOrec-like value-based validation behind
+ *          one global sequence lock, writers serialised (no lock table);
+ *   HV_UNSORTED = ablation: HV with locks in encounter order and the parallel
+ *          retry of HV -- exposed to the intra-warp livelock of P:63 (ends in
+ *          GSTM_ETIMEOUT when it happens; for demonstrations only). */
+enum gstm_mode {
+    GSTM_MODE_AUTO = 0, GSTM_MODE_HV = 1, GSTM_MODE_TBV = 2, GSTM_MODE_CGL = 3, GSTM_MODE_FGL = 4,
+    GSTM_MODE_HV_BACKOFF = 5, GSTM_MODE_VBV = 6, GSTM_MODE_HV_UNSORTED = 7
+};
 
 typedef struct {
     /* workload shape (which fields apply: DESIGN.md §3.3) */
@@ -223,8 +234,10 @@ int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per
  * DESIGN.md §5.3).  mode: GSTM_MODE_HV or GSTM_MODE_TBV. */
 int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx);
 /* Insert entries (id<<2 | wr<<1 | rd) into a device lock log (variant 0:
- * register-resident, capacity 16; 1: local memory, capacity 256) and return
- * the resulting log in out; returns its length or a negative error. */
+ * register-resident, capacity 16; 1: local memory, capacity 256; both sorted
+ * by id.  Variants 2 and 3: the same capacities in encounter
+ * order, the lock order of GSTM_MODE_HV_BACKOFF / GSTM_MODE_HV_UNSORTED) and
+ * return the resulting log in out; returns its length or a negative error. */
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant);
 /* Roofline microbenchmark: kind 0 random atom.or, 1
  * same-address atom.add.u64, 2 random ld.relaxed, 3 random st.relaxed, 4

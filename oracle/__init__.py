@@ -107,6 +107,8 @@ def lib():
                                      P(u32), i32]
         L.or_lock_log.restype = i32
         L.or_lock_log.argtypes = [P(u32), i32, P(u32), i32]
+        L.or_lock_log_encounter.restype = i32
+        L.or_lock_log_encounter.argtypes = [P(u32), i32, P(u32), i32]
         L.or_brute.restype = i64
         L.or_brute.argtypes = [P(Params), P(u32), u64, u64, u64, u64, P(u32), P(u32), P(i32),
                                P(i64)]
@@ -217,10 +219,12 @@ def alg3_script(mode: int, bits: int, heap: np.ndarray, lock_tab: np.ndarray, cl
     return out, clk.value
 
 
-def lock_log(entries) -> np.ndarray:
+def lock_log(entries, sorted_log: bool = True) -> np.ndarray:
+    """Sorted lock log, or the encounter-order log (Q32)."""
     e = np.ascontiguousarray(np.asarray(entries, dtype=np.uint32))
     out = np.zeros(max(e.size, 1), dtype=np.uint32)
-    n = lib().or_lock_log(_p(e, C.c_uint32), e.size, _p(out, C.c_uint32), out.size)
+    fn = lib().or_lock_log if sorted_log else lib().or_lock_log_encounter
+    n = fn(_p(e, C.c_uint32), e.size, _p(out, C.c_uint32), out.size)
     return out[:n].copy()
 
 

@@ -77,6 +77,23 @@ int or_lock_log(const uint32_t* entries, int n, uint32_t* out, int cap)
     return m;
 }
 
+/* Encounter-order lock log (Q32): the lock order of STM-HV-Backoff
+ * (P:250), which does not sort -- each lock id appears once, at the position
+ * of its first access, carrying the OR of the rd/wr bits of all its accesses. */
+int or_lock_log_encounter(const uint32_t* entries, int n, uint32_t* out, int cap)
+{
+    int m = 0;
+    for (int k = 0; k < n; ++k) {
+        const uint32_t id = entries[k] >> 2;
+        int j = 0;
+        while (j < m && (out[j] >> 2) != id) ++j;
+        if (j < m) { out[j] |= entries[k] & 3u; continue; }
+        if (m >= cap) return -1;
+        out[m++] = entries[k];
+    }
+    return m;
+}
+
 /* 1: TXBegin */
 static void TXBegin(stm_t* g, tx_t* tx)
 {

@@ -115,6 +115,9 @@ int or_alg3_script(int mode, int prelock_vbv, uint32_t bits,
 /* Encounter-time sorted lock log: insert the given entries
  * (lock_id<<2 | wr<<1 | rd) in order, return the resulting log. */
 int or_lock_log(const uint32_t* entries, int n, uint32_t* out, int cap);
+/* Encounter-order variant (STM-HV-Backoff; Q32): first
+ * occurrence order, duplicates merged.  Returns the length or -1 (cap). */
+int or_lock_log_encounter(const uint32_t* entries, int n, uint32_t* out, int cap);
 
 /* ---------------- brute.c: every serial order of a tiny tx set ----------- */
 /* Enumerate all interleavings of the T per-thread sequences of K txs

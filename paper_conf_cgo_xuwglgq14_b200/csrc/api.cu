@@ -31,6 +31,8 @@ static void set_error(const char* fmt, ...)
 static constexpr size_t kMetaBytes = 256 * 1024;  // metadata block (M_WORDS used) + g_clock candidates
 static constexpr int kClockCandidates = 64;        // candidate lines for g_clock after M_WORDS ...
 static constexpr int kClockStride = 288;           // ... 2304 B apart (crosses 256 B and 2 KiB address bits)
+static_assert(gstm::M_SEQ >= gstm::M_WORDS + kClockCandidates * kClockStride + 16 && gstm::M_SEQ * 8 + 128 <= kMetaBytes,
+              "STM-VBV sequence lock must sit on its own line after the clock candidates");
 
 struct gstm_handle {
     char* block = nullptr;          // the single device allocation
@@ -260,7 +262,7 @@ int gstm_get_params(const gstm_t* h, gstm_params_t* out)
 
 int gstm_set_mode(gstm_t* h, int mode)
 {
-    if (!h || mode < GSTM_MODE_AUTO || mode > GSTM_MODE_FGL) { set_error("gstm_set_mode: bad mode %d", mode); return GSTM_EINVAL; }
+    if (!h || mode < GSTM_MODE_AUTO || mode > GSTM_MODE_HV_UNSORTED) { set_error("gstm_set_mode: bad mode %d", mode); return GSTM_EINVAL; }
     h->mode = mode;
     return GSTM_OK;
 }
@@ -637,7 +639,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
 
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant)
 {
-    if (!entries || !out || n < 0 || n > 4096 || (variant != 0 && variant != 1)) { set_error("gstm_lock_log: bad argument"); return GSTM_EINVAL; }
+    if (!entries || !out || n < 0 || n > 4096 || variant < 0 || variant > 3) { set_error("gstm_lock_log: bad argument"); return GSTM_EINVAL; }
     uint32_t *de = nullptr, *dout = nullptr;
     int* dn = nullptr;
     CUDA_TRY(cudaMalloc(&de, (n + 1) * 4));

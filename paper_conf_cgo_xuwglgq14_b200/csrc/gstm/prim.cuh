@@ -161,6 +161,15 @@ __device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, 
     return old;
 }
 
+__device__ __forceinline__ unsigned long long atom_cas_acquire64(unsigned long long* p, unsigned long long cmp,
+                                                                 unsigned long long v)
+{
+    unsigned long long old;
+    asm volatile("atom.acquire.gpu.global.cas.b64 %0, [%1], %2, %3;"
+                 : "=l"(old) : "l"(p), "l"(cmp), "l"(v) : "memory");
+    return old;
+}
+
 __device__ __forceinline__ unsigned long long atom_add_acq_rel64(unsigned long long* p, unsigned long long v)
 {
     unsigned long long old;

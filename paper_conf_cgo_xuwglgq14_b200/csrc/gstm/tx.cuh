@@ -65,7 +65,10 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
     return 1ull << ((static_cast<unsigned long long>(w) * 0x9E3779B97F4A7C15ull) >> 58);
 }
 
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false>
+// SORTED = false: the lock log keeps encounter order (duplicates still
+// merged) -- the lock order of STM-HV-Backoff and of the unsorted
+// ablation; the paper's GPU-STM sorts.
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true>
 struct Tx {
     // register-resident (unrolled) logs for small capacities unless the
     // workload asks for local memory (LOCAL: fewer registers, more warps)
@@ -145,6 +148,7 @@ struct Tx {
             }
             if (dup) return;
             if (nl >= LCAP) { overflow = true; opaque = false; return; }
+            if constexpr (!SORTED) pos = nl;                         // encounter order: append
 #pragma unroll
             for (int k = LCAP - 1; k > 0; --k)
                 if (k <= nl && k > pos) l_ent[k] = l_ent[k - 1];
@@ -154,7 +158,11 @@ struct Tx {
             ++nl;
         } else {
             int pos = 0;
-            while (pos < nl && (l_ent[pos] >> 2) < id) ++pos;
+            if constexpr (SORTED) {
+                while (pos < nl && (l_ent[pos] >> 2) < id) ++pos;
+            } else {
+                while (pos < nl && (l_ent[pos] >> 2) != id) ++pos;   // encounter order: find or append
+            }
             if (pos < nl && (l_ent[pos] >> 2) == id) { l_ent[pos] |= (e & 3u); return; }
             if (nl >= LCAP) { overflow = true; opaque = false; return; }
             for (int k = nl; k > pos; --k) l_ent[k] = l_ent[k - 1];

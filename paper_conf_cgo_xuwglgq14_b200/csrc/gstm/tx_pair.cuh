@@ -21,9 +21,9 @@
 
 namespace gstm {
 
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false>
-struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL> {
-    using B = Tx<RCAP, WCAP, LCAP, LOCAL>;
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED>;
     using B::kUnroll;
     using B::r_addr;
     using B::r_val;

@@ -1,442 +1,31 @@
-// kernels.cu -- the transaction kernels (STM-HV, STM-TBV, CGL, FGL) and
-// their helpers.
-//
-// One CUDA thread = one STM thread t (Figure 1) that runs K
-// transactions i = 0..K-1 (tx_id = i*T + t).  The loop is warp-uniform:
-// every iteration the 32 lanes each attempt their current transaction
-// together (lanes whose transaction committed move on to the next one, the
-// others re-execute theirs), and commit is a warp-collective phase:
-//   * lock acquisition rounds: lanes that fail to get a lock retry only
-//     after the lanes of the same warp that got theirs finished committing
-//     ("On locking failure, it retries after transactions within the same
-//     warp finish committing"), for at most k_lock rounds;
-//   * the committing lanes of a round take their commit stamps with ONE
-//     atomic on the global clock (A3.l83 aggregated over the warp);
-//   * the snapshot (A3.l4) is read once per warp and broadcast.
+// kernels.cu -- the non-template kernels (launch prologue/epilogue, heap
+// initialisation, paired-layout packing) and the per-workload dispatch; the
+// transaction kernels are in stm_kernels.cuh, instantiated in wl_*.cu.
 #include <algorithm>
 #include <cstdint>
-#include <type_traits>
 #include "kernels.cuh"
 
 namespace gstm {
 
-using prim::FULL;
-
-// WL::kLocalLogs (optional): keep the logs in local memory even when small
-template <class WL, class = void>
-struct LocalLogs { static constexpr bool value = false; };
-template <class WL>
-struct LocalLogs<WL, std::void_t<decltype(WL::kLocalLogs)>> { static constexpr bool value = WL::kLocalLogs; };
-
-__device__ __forceinline__ unsigned long long globaltimer()
+__device__ __forceinline__ unsigned long long globaltimer_ns()
 {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
 
-// A3.l4-5: snapshot <- g_clock; threadfence.  One acquire load per warp; the
-// __syncwarp orders every lane's later accesses after it.
-__device__ __forceinline__ uint32_t warp_snapshot(unsigned long long* clock)
-{
-    unsigned long long s = 0;
-    if (prim::lane_id() == 0) s = prim::ld_acquire64(clock);
-    s = __shfl_sync(FULL, s, 0);
-    __syncwarp();
-    return static_cast<uint32_t>(s);
-}
-
-// warp-aggregated commit stamp (A3.l83): lanes in `got` each receive a
-// distinct stamp; one atom.add per warp round.  Every committing lane has
-// drained its write-back with a release fence (l.82, in Tx::writeback); the
-// __syncwarp orders those fences before the leader's atomic, and the one
-// after orders the leader's acquire before every lane's lock release.  If
-// any lane committed, *next_snap = base + n is the clock value right after
-// the warp's own commits, a valid snapshot for its next transactions.
-__device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool got, unsigned& gm, uint32_t& next_snap)
-{
-    __syncwarp();
-    gm = __ballot_sync(FULL, got);
-    unsigned long long base = 0;
-    if (gm) {
-        const int leader = __ffs(gm) - 1;
-#if GSTM_EXPERIMENT_NO_CLOCK   // measurement only: fake stamps, NOT serializable
-        base = (static_cast<unsigned long long>(blockIdx.x) << 20) + threadIdx.x;
-#else
-        if (static_cast<int>(prim::lane_id()) == leader) base = clock_fetch_add(clock, __popc(gm));
-#endif
-        base = __shfl_sync(FULL, base, leader);
-        __syncwarp();
-        next_snap = static_cast<uint32_t>(base) + __popc(gm);
-    }
-    return static_cast<uint32_t>(base) + __popc(gm & prim::lanemask_lt()) + 1u;
-}
-
-// Statistics counters: one block-shared array (shared-memory atomics on the
-// rare events), flushed to the launch's counters with one global atomic per
-// counter per block.  Kept out of registers (they cost occupancy).
-struct Counters {
-    unsigned long long* sh;
-    bool error = false;
-    __device__ __forceinline__ void inc(int k, uint32_t v = 1u)
-    {
-        if (v) atomicAdd(&sh[k], static_cast<unsigned long long>(v));
-        if (k == S_ERRORS) error = true;
-    }
-};
-
-#define GSTM_COUNTERS(name)                                                 \
-    __shared__ unsigned long long name##_sh[S_NSTATS];                      \
-    if (threadIdx.x < S_NSTATS) name##_sh[threadIdx.x] = 0;                 \
-    __syncthreads();                                                        \
-    Counters name{name##_sh}
-
-// block totals -> one global atomic per counter per block
-__device__ __forceinline__ void flush_counters(Counters& cnt, unsigned long long* stats)
-{
-    __syncthreads();
-    if (threadIdx.x < S_NSTATS && cnt.sh[threadIdx.x]) atomicAdd(stats + threadIdx.x, cnt.sh[threadIdx.x]);
-}
-
-__device__ __forceinline__ void set_err(unsigned long long* meta, uint32_t bits)
-{
-    atomicOr(reinterpret_cast<unsigned int*>(meta + M_ERR), bits);
-}
-
-// warp-uniform watchdog check (every 16 iterations)
-__device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long deadline)
-{
-    if (iter & 15u) return false;
-    bool late = false;
-    if (prim::lane_id() == 0) late = globaltimer() > deadline;
-    return __shfl_sync(FULL, late, 0);
-}
-
-// Per-phase time breakdown of the transaction loop (the Figure 5 study of
-// P:329-333): build with -DGSTM_PHASE_TIMING=1; lane 0 of every
-// warp adds the SM cycles each phase of each iteration took (after a warp
-// barrier, so the time is the warp's) to meta[M_PHASE + k].
-#ifndef GSTM_PHASE_TIMING
-#define GSTM_PHASE_TIMING 0
-#endif
-enum { PH_BEGIN = 0, PH_BODY, PH_LOCK, PH_STAMP, PH_RELEASE, PH_LOOP, PH_N };
-#if GSTM_PHASE_TIMING
-#define PHASE_DECL() unsigned long long ph_[PH_N] = {0, 0, 0, 0, 0, 0}; long long ph_t_ = clock64()
-#define PHASE_MARK(k)                                                        \
-    do {                                                                     \
-        __syncwarp();                                                        \
-        const long long now_ = clock64();                                    \
-        ph_[k] += static_cast<unsigned long long>(now_ - ph_t_);            \
-        ph_t_ = now_;                                                        \
-    } while (0)
-#define PHASE_FLUSH(dst)                                                     \
-    do {                                                                     \
-        if (prim::lane_id() == 0)                                            \
-            for (int k_ = 0; k_ < PH_N; ++k_) atomicAdd((dst) + k_, ph_[k_]); \
-    } while (0)
-#else
-#define PHASE_DECL() do {} while (0)
-#define PHASE_MARK(k) do {} while (0)
-#define PHASE_FLUSH(dst) do {} while (0)
-#endif
-
-// ---------------------------------------------------------------------------
-// STM kernel: GPU-STM with hierarchical validation (MODE_HV, "STM-HV-Sorting")
-// or timestamp-only validation (MODE_TBV, "STM-TBV-Sorting").
-// ---------------------------------------------------------------------------
-template <class WL, int MODE, bool PAIR>
-__global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
-{
-    using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>,
-                                  Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value>>;
-    // The grid is persistent (host sizes it to what fits on the chip, or to
-    // p.max_threads): lane g starts with STM thread t = g; a lane that has run
-    // all K transactions of its thread takes the next unstarted thread from a
-    // global counter (one warp-aggregated atomic), so no lane idles while
-    // work remains and the program order of each STM thread is kept.
-    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (p.K == 0) t = p.T;
-    const Meta m = p.m;
-    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
-    const unsigned long long deadline = p.meta[M_DEADLINE];
-    unsigned long long* work = p.meta + M_WORK;
-    GSTM_COUNTERS(cnt);
-    TX tx;
-    tx.reset_stats();
-    uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
-    // stage 0: start (or re-execute) transaction (t, i); stage 1: its body
-    // ran and it waits for its locks (a lost lock round is retried in the
-    // warp's next iteration, after the winners committed)
-    int stage = 0;
-    bool timed_out = false, have_snap = false, lock_aborted = false;
-    PHASE_DECL();
-
-    while (__any_sync(FULL, t < p.T)) {
-        if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = t < p.T;
-        // TXBegin l.4-5: a fresh clock read, or the clock value right after
-        // this warp's own last commit (p.snapshot_reuse)
-        const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
-        have_snap = false;
-        PHASE_MARK(PH_BEGIN);
-        const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-        bool done = false, skip = false;
-        if (act && stage == 0) {
-            cnt.inc(S_ATTEMPTS);
-            result = 0;
-            const uint64_t x = gen::tx_key(p.seed, t, i);
-            tx.begin(snap);                                           // TXBegin l.2-3
-            StmCtx<TX> ctx{tx, m, MODE};
-            WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
-            if (!tx.opaque) {
-                if (tx.overflow) { cnt.inc(S_ERRORS); skip = true; }  // sticky ELOGOVF, give up this tx
-                else cnt.inc(S_AB_OPACITY);                          // Figure 1 / Q11
-            } else if (tx.read_only()) {                              // l.68: linearized at snapshot
-                if (p.tx_stamp) {
-                    p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
-                    p.tx_result[tx_id] = result;
-                }
-                cnt.inc(S_COMMITS_RO);
-                done = true;
-            } else {
-                stage = 1;
-                tries = 0;
-            }
-        }
-        PHASE_MARK(PH_BODY);
-        // No lane may take a lock while another lane of its warp can still be
-        // spinning on a lock in its read phase (A3.l27-29): under independent
-        // thread scheduling the locker would then wait for the spinner at the
-        // warp barrier in warp_stamp while the spinner waits for its lock.
-        __syncwarp();
-        // one warp-collective TXCommit round per iteration (l.67-85)
-        bool got = false;
-        if (act && stage == 1) {
-            // the pipelined round (§6.4) only for the first round of an
-            // execution that never lost its locks before: every retry uses the
-            // sequential sorted acquisition
-            const bool pipelined = p.lock_pipeline && tries == 0 && !lock_aborted;
-            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
-            if (r == C_OK) {
-                got = true;
-                tx.writeback(m);                                      // l.79-82
-            } else if (r == C_LOCK) {
-                cnt.inc(S_LOCK_RETRIES);                              // l.73-74: retry next iteration
-                if (p.k_lock && ++tries >= p.k_lock) {
-                    stage = 0;
-                    lock_aborted = true;
-                    cnt.inc(S_AB_LOCK);
-                }
-            } else {
-                stage = 0;
-                cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
-            }
-        }
-        PHASE_MARK(PH_LOCK);
-        unsigned gm;
-        const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
-        if (gm) have_snap = true;
-        PHASE_MARK(PH_STAMP);
-        if (got) {
-            tx.release_and_update(m, stamp);                          // l.84
-            if (p.tx_stamp) {
-                p.tx_stamp[tx_id] = stamp - clock_begin;
-                p.tx_result[tx_id] = result;
-            }
-            cnt.inc(S_COMMITS);
-            done = true;
-        }
-        PHASE_MARK(PH_RELEASE);
-        if (done || skip) {
-            stage = 0;
-            ++i;
-            backoff = 0;
-            lock_aborted = false;
-        } else if (p.backoff_ns && act && stage == 0) {
-            // exponential backoff after an abort (P:111 argues per-lane
-            // delays cannot work under SIMT; lanes here sleep independently
-            // under independent thread scheduling)
-            backoff = backoff ? min(backoff * 2u, 64u * p.backoff_ns) : p.backoff_ns;
-            __nanosleep(backoff);
-        }
-        // refill: lanes whose STM thread ran all K transactions take the next one
-        const bool need = t < p.T && i >= p.K;
-        const unsigned nm = __ballot_sync(FULL, need);
-        if (nm) {
-            const int leader = __ffs(nm) - 1;
-            unsigned long long base = 0;
-            if (static_cast<int>(prim::lane_id()) == leader) base = atomicAdd(work, static_cast<unsigned long long>(__popc(nm)));
-            base = __shfl_sync(FULL, base, leader);
-            if (need) {
-                t = P + base + __popc(nm & prim::lanemask_lt());
-                i = 0;
-            }
-        }
-        PHASE_MARK(PH_LOOP);
-    }
-    PHASE_FLUSH(p.meta + M_PHASE);
-    cnt.inc(S_POSTVAL, tx.n_postval);
-    cnt.inc(S_VBV, tx.n_vbv);
-    cnt.inc(S_SPINS, tx.n_spin);
-    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
-    flush_counters(cnt, p.meta + M_STATS);
-}
-
-// ---------------------------------------------------------------------------
-// CGL baseline: one global lock serialises every transaction, taken
-// with Algorithm 1 Scheme #3 (diverge on failure) plus a test before
-// the CAS.  The body runs in place; the stamp is taken under the lock.
-// ---------------------------------------------------------------------------
-template <class WL>
-__global__ void __launch_bounds__(256, WL::kMinBlocks) cgl_kernel(const KParams p)
-{
-    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (p.K == 0) t = p.T;
-    uint32_t* lock = reinterpret_cast<uint32_t*>(p.meta + M_CGL_LOCK);
-    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
-    const unsigned long long deadline = p.meta[M_DEADLINE];
-    GSTM_COUNTERS(cnt);
-    uint32_t i = 0, iter = 0, backoff = 0;
-    bool timed_out = false;
-    while (__any_sync(FULL, t < p.T)) {
-        if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = t < p.T;
-        if (act) {
-            cnt.inc(S_ATTEMPTS);
-            if (prim::ld_relaxed(lock) == 0 && prim::atom_cas_acquire(lock, 0u, 1u) == 0u) {
-                backoff = 0;
-                const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-                DirectCtx ctx{p.m, 0, false};
-                uint32_t result = 0;
-                WL::body(ctx, p.w, gen::tx_key(p.seed, t, i), t, i, result);   // critical section
-                uint32_t s;
-                if (ctx.nw) {
-                    s = static_cast<uint32_t>(prim::atom_add_relaxed64(p.m.clock, 1ull)) + 1u - clock_begin;
-                    cnt.inc(S_COMMITS);
-                } else {
-                    s = 0x80000000u | (static_cast<uint32_t>(prim::ld_relaxed64(p.m.clock)) - clock_begin);
-                    cnt.inc(S_COMMITS_RO);
-                }
-                if (ctx.bad) cnt.inc(S_ERRORS);
-                if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
-                prim::fence_release();
-                prim::st_relaxed(lock, 0u);                           // Scheme #3 l.15
-                if (++i >= p.K) { i = 0; t += P; }
-            } else {
-                cnt.inc(S_LOCK_RETRIES);
-                // optional per-thread exponential backoff (test-and-test-and-set
-                // with backoff; the paper's Scheme #3 has none: backoff_ns = 0)
-                if (p.backoff_ns) {
-                    backoff = backoff ? min(backoff * 2u, 256u * p.backoff_ns) : p.backoff_ns;
-                    __nanosleep(backoff);
-                }
-            }
-        }
-    }
-    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_INVALID);
-    flush_counters(cnt, p.meta + M_STATS);
-}
-
-// ---------------------------------------------------------------------------
-// FGL baseline: the hand-locking a programmer would write -- one lock per
-// stripe of the words the transaction will touch (per account, per bucket,
-// per k-means record), acquired in ascending id with try-lock and
-// release-all on failure, then the body in place.  No logs, no validation.
-// (The paper did not implement FGL; north_star asks for it.)
-// ---------------------------------------------------------------------------
-template <class WL>
-__global__ void __launch_bounds__(256, WL::kMinBlocks) fgl_kernel(const KParams p)
-{
-    using TX = Tx<1, 1, WL::FGL_LCAP>;      // only the sorted lock log is used
-    const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-    uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (p.K == 0) t = p.T;
-    const Meta m = p.m;
-    const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
-    const unsigned long long deadline = p.meta[M_DEADLINE];
-    GSTM_COUNTERS(cnt);
-    TX lk;
-    uint32_t i = 0, iter = 0;
-    bool timed_out = false;
-    while (__any_sync(FULL, t < p.T)) {
-        if (warp_late(iter++, deadline)) { timed_out = true; break; }
-        const bool act = t < p.T;
-        const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-        bool got = false;
-        int nw = 0;
-        uint32_t result = 0;
-        if (act) {
-            cnt.inc(S_ATTEMPTS);
-            const uint64_t x = gen::tx_key(p.seed, t, i);
-            lk.begin(0);
-            WL::fgl_words(p.w, x, t, i, [&](uint32_t w) { lk.insert_lock((m.lock_of(w) << 2) | 2u); });
-            if (lk.overflow) {
-                cnt.inc(S_ERRORS);
-            } else if (lk.get_locks_and_tbv(m)) {
-                got = true;
-                DirectCtx ctx{m, 0, false};
-                WL::body(ctx, p.w, x, t, i, result);
-                nw = ctx.nw;
-                if (ctx.bad) cnt.inc(S_ERRORS);
-                prim::fence_release();          // in-place writes before stamp and unlock
-            } else {
-                cnt.inc(S_LOCK_RETRIES);
-            }
-        }
-        unsigned gm;
-        uint32_t unused_snap;
-        const uint32_t stamp = warp_stamp(m.clock, got && nw > 0, gm, unused_snap);
-        if (got) {
-            uint32_t s;
-            if (nw > 0) {
-                s = stamp - clock_begin;
-                cnt.inc(S_COMMITS);
-            } else {
-                s = 0x80000000u | (static_cast<uint32_t>(prim::ld_acquire64(m.clock)) - clock_begin);
-                cnt.inc(S_COMMITS_RO);
-            }
-            if (p.tx_stamp) { p.tx_stamp[tx_id] = s; p.tx_result[tx_id] = result; }
-            if (GSTM_STRICT_FENCES) prim::fence_release();
-            lk.release_locks(m);
-        }
-        if (got || (act && lk.overflow)) {
-            if (++i >= p.K) { i = 0; t += P; }
-        } else if (act && p.backoff_ns) {
-            __nanosleep(p.backoff_ns);
-        }
-    }
-    if (__any_sync(FULL, timed_out) && prim::lane_id() == 0) set_err(p.meta, ERR_TIMEOUT);
-    if (__any_sync(FULL, cnt.error) && prim::lane_id() == 0) set_err(p.meta, ERR_LOGOVF);
-    flush_counters(cnt, p.meta + M_STATS);
-}
-
-// ---------------------------------------------------------------------------
-// descriptor dump (generator parity test): out[(i*T + t) * wpt + k]
-// ---------------------------------------------------------------------------
-template <class WL>
-__global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
-{
-    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (t >= p.T) return;
-    for (uint32_t i = 0; i < p.K; ++i) {
-        uint32_t d[WL::DESCR];
-        const int n = WL::descr(p.w, gen::tx_key(p.seed, t, i), d);
-        uint32_t* o = out + (static_cast<uint64_t>(i) * p.T + t) * wpt;
-        for (int k = 0; k < wpt; ++k) o[k] = k < n ? d[k] : 0u;
-    }
-}
+template <class WL> cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s);
+template <class WL> cudaError_t launch_descr_wl(const KParams& kp, uint32_t* out, int wpt, cudaStream_t s);
+template <class WL> bool check_wl(const WlParams& w, uint64_t* fp, int* dw);
 
 __global__ void prepare_kernel(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns)
 {
-    const unsigned long long now = globaltimer();
+    const unsigned long long now = globaltimer_ns();
     meta[M_CLOCK_BEGIN] = *clock;
     meta[M_DEADLINE] = now + timeout_ns;
     meta[M_T_START] = now;
     meta[M_WORK] = 0;
+    meta[M_SEQ] = 2ull * *clock;                    // STM-VBV sequence lock (tx_vbv.cuh)
     for (int k = 0; k < S_NSTATS; ++k) meta[M_STATS + k] = 0;
     *reinterpret_cast<uint32_t*>(meta + M_ERR) = 0;
     *reinterpret_cast<uint32_t*>(meta + M_CGL_LOCK) = 0;
@@ -449,7 +38,7 @@ __global__ void finish_kernel(unsigned long long* meta, const unsigned long long
     meta[M_CLOCK_END] = *clock;
     for (int k = 0; k < S_NSTATS; ++k) meta[M_TOTALS + k] += meta[M_STATS + k];
     meta[M_T_LAUNCHES] += 1;
-    meta[M_T_NS] += globaltimer() - meta[M_T_START];
+    meta[M_T_NS] += globaltimer_ns() - meta[M_T_START];
     meta[M_T_ERR] |= meta[M_ERR] & 0xffffffffull;
 }
 
@@ -528,52 +117,6 @@ cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, int v
     return cudaGetLastError();
 }
 
-// persistent grid for a kernel: the blocks that fit on the chip at once
-template <class K>
-static uint64_t resident_blocks(K kernel, int block)
-{
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    }
-    int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, 0) != cudaSuccess || per_sm < 1) per_sm = 1;
-    return static_cast<uint64_t>(per_sm) * (sms > 0 ? sms : 148);
-}
-
-template <class K>
-static cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s)
-{
-    uint64_t grid = (kp.T + block - 1) / block;
-    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block));
-    if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
-    if (grid == 0) return cudaSuccess;
-    kernel<<<static_cast<unsigned>(grid), block, 0, s>>>(kp);
-    return cudaGetLastError();
-}
-
-template <class WL>
-static cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
-{
-    uint64_t grid = (kp.T + block - 1) / block;
-    if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
-    if (grid == 0) return cudaSuccess;
-    const dim3 g(static_cast<unsigned>(grid)), b(block);
-    switch (kmode) {
-    case KMODE_HV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s);
-    case KMODE_TBV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s);
-    case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
-    case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
-    default: return cudaErrorInvalidValue;
-    }
-    return cudaGetLastError();
-}
 
 cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cudaStream_t s)
 {
@@ -587,14 +130,6 @@ cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cud
     return cudaErrorInvalidValue;
 }
 
-template <class WL>
-static cudaError_t launch_descr_wl(const KParams& kp, uint32_t* out, int wpt, cudaStream_t s)
-{
-    const uint64_t grid = (kp.T + 255) / 256;
-    if (grid) descr_kernel<WL><<<static_cast<unsigned>(grid), 256, 0, s>>>(kp, out, wpt);
-    return cudaGetLastError();
-}
-
 cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt, cudaStream_t s)
 {
     switch (workload) {
@@ -605,15 +140,6 @@ cudaError_t launch_descr(int workload, const KParams& kp, uint32_t* out, int wpt
     case WL_KM: return launch_descr_wl<KmWL>(kp, out, wpt, s);
     }
     return cudaErrorInvalidValue;
-}
-
-template <class WL>
-static bool check_wl(const WlParams& w, uint64_t* fp, int* dw)
-{
-    if (!WL::check(w)) return false;
-    *fp = WL::footprint(w);
-    *dw = WL::DESCR;
-    return true;
 }
 
 bool workload_check(int workload, const WlParams& w, uint64_t* fp, int* dw)

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include "gstm/tx.cuh"
 #include "gstm/tx_pair.cuh"
+#include "gstm/tx_vbv.cuh"
 #include "gstm/workloads.cuh"
 
 namespace gstm {
@@ -30,13 +31,17 @@ enum {
     M_T_ERR = 98 + S_NSTATS,           // OR of the error bits since reset
     M_PHASE = 112,                     // 8 phase-cycle accumulators (GSTM_PHASE_TIMING builds)
     M_WORK = 120,                      // next unstarted STM thread (persistent grid), own line
-    M_WORDS = 128
+    M_WORDS = 128,
+    // after the 64 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
+    M_SEQ = M_WORDS + 64 * 288 + 16,   // STM-VBV global sequence lock, own line
 };
 
 enum { ERR_LOGOVF = 1, ERR_TIMEOUT = 2, ERR_INVALID = 4 };
 
 enum { WL_RA = 0, WL_BANK = 1, WL_HT = 2, WL_EB = 3, WL_KM = 4 };
-enum { KMODE_HV = 1, KMODE_TBV = 2, KMODE_CGL = 3, KMODE_FGL = 4 };
+enum { KMODE_HV = 1, KMODE_TBV = 2, KMODE_CGL = 3, KMODE_FGL = 4, KMODE_HV_BACKOFF = 5, KMODE_VBV = 6, KMODE_HV_UNSORTED = 7 };
+// lock order / retry policy of the STM kernel (kernels.cu)
+enum { POL_SORTED = 0, POL_BACKOFF = 1, POL_UNSORTED = 2 };
 
 struct KParams {
     Meta m;

@@ -69,15 +69,17 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
 }
 
 // lock-log parity kernel: insert entries into a register-resident (variant 0)
-// or local-memory (variant 1) lock log and dump it.
-template <int LCAP>
+// or local-memory (variant 1) sorted lock log, or their encounter-order
+// counterparts (variants 2, 3: STM-HV-Backoff / unsorted ablation), and dump it.
+template <int LCAP, bool SORTED>
 __global__ void lock_log_kernel(const uint32_t* e, int n, uint32_t* out, int* out_n)
 {
     if (threadIdx.x || blockIdx.x) return;
-    Tx<1, 1, LCAP> tx;
+    using TX = Tx<1, 1, LCAP, false, SORTED>;
+    TX tx;
     tx.begin(0);
     for (int k = 0; k < n; ++k) tx.insert_lock(e[k]);
-    if constexpr (Tx<1, 1, LCAP>::kUnroll) {
+    if constexpr (TX::kUnroll) {
 #pragma unroll
         for (int k = 0; k < LCAP; ++k)
             if (k < tx.nl) out[k] = tx.l_ent[k];
@@ -98,8 +100,12 @@ cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* 
 
 cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s)
 {
-    if (variant == 0) lock_log_kernel<16><<<1, 32, 0, s>>>(entries, n, out, out_n);
-    else lock_log_kernel<256><<<1, 32, 0, s>>>(entries, n, out, out_n);
+    switch (variant) {
+    case 0: lock_log_kernel<16, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    case 1: lock_log_kernel<256, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    case 2: lock_log_kernel<16, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    default: lock_log_kernel<256, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    }
     return cudaGetLastError();
 }
 

@@ -1,0 +1,8 @@
+// wl_ra.cu -- RaWL, RaIncWL instantiations of the transaction kernels
+// (stm_kernels.cuh); one translation unit per workload keeps the build parallel.
+#include "stm_kernels.cuh"
+
+namespace gstm {
+GSTM_INSTANTIATE_WL(RaWL)
+GSTM_INSTANTIATE_WL(RaIncWL)
+}  // namespace gstm

@@ -21,7 +21,9 @@ LIB_PATH = os.path.join(_HERE, "lib", "libgstm.so")
 WL_RA, WL_BANK, WL_HT, WL_EB, WL_KM = 0, 1, 2, 3, 4
 WORKLOADS = {"ra": WL_RA, "bank": WL_BANK, "ht": WL_HT, "eb": WL_EB, "km": WL_KM}
 MODE_AUTO, MODE_HV, MODE_TBV, MODE_CGL, MODE_FGL = 0, 1, 2, 3, 4
-MODES = {"auto": MODE_AUTO, "hv": MODE_HV, "tbv": MODE_TBV, "cgl": MODE_CGL, "fgl": MODE_FGL}
+MODE_HV_BACKOFF, MODE_VBV, MODE_HV_UNSORTED = 5, 6, 7
+MODES = {"auto": MODE_AUTO, "hv": MODE_HV, "tbv": MODE_TBV, "cgl": MODE_CGL, "fgl": MODE_FGL,
+         "hv_backoff": MODE_HV_BACKOFF, "vbv": MODE_VBV, "hv_unsorted": MODE_HV_UNSORTED}
 MODE_NAMES = {v: k for k, v in MODES.items()}
 RO_FLAG = 0x80000000
 

@@ -39,8 +39,8 @@ def test_library_is_sm100a_and_self_contained(so):
     assert "libcudart" not in deps          # static cudart: nothing to resolve on the GPU box
     sass = subprocess.check_output(["cuobjdump", "-sass", so], text=True)
     funcs = dict(re.findall(r"Function : (\S+)\n(.*?)(?=\n\s*Function : |\Z)", sass, flags=re.S))
-    split = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb0EEEvNS_7KParamsE"]    # HV, paper layout
-    paired = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb1EEEvNS_7KParamsE"]   # HV, paired layout
+    split = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb0ELi0EEEvNS_7KParamsE"]    # HV, paper layout
+    paired = funcs["_ZN4gstm10stm_kernelINS_6BankWLELi1ELb1ELi0EEEvNS_7KParamsE"]   # HV, paired layout
     # the hot path is made of L2 atomics / strong gpu-scope accesses
     assert "ATOMG.E.OR.STRONG.GPU" in split and "LDG.E.STRONG.GPU" in split
     assert "ATOMG.E.OR.64.STRONG.GPU" in paired and "LDG.E.64.STRONG.GPU" in paired

@@ -72,15 +72,16 @@ def test_init_heap_parity(wl):
     assert (g.read_heap() == O.init_heap(op, 100_003)).all()
 
 
-@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256)])
+@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256), (2, 16), (3, 256)])
 def test_lock_log_parity(variant, cap):
-    """Encounter-time sorted lock log on the device vs the oracle."""
+    """Encounter-time sorted lock log (P:113-115) on the device vs the oracle;
+    variants 2/3: the encounter-order log of STM-HV-Backoff (Q32)."""
     rng = np.random.default_rng(variant)
     for trial in range(300):
         n = int(rng.integers(0, cap + 8))
         hi = int(rng.choice([4, 50, 1 << 20]))
         e = (rng.integers(0, hi, n).astype(np.uint32) << 2) | rng.integers(1, 4, n).astype(np.uint32)
-        want = O.lock_log(e)
+        want = O.lock_log(e, sorted_log=variant < 2)
         if want.size > cap:
             with pytest.raises(G.GstmError):
                 G.gstm_lock_log(e, variant)

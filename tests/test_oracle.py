@@ -335,6 +335,23 @@ def test_lock_log_sorted_dedup():
         [(1 << 2) | 1, (3 << 2) | 3, (9 << 2) | 3]
 
 
+def test_lock_log_encounter_order():
+    """Q32 (STM-HV-Backoff): first-occurrence order, bits merged; same
+    set of entries as the sorted log."""
+    assert O.lock_log([(9 << 2) | 1, (3 << 2) | 2, (9 << 2) | 2, (1 << 2) | 1, (3 << 2) | 1],
+                      sorted_log=False).tolist() == [(9 << 2) | 3, (3 << 2) | 3, (1 << 2) | 1]
+    rng = np.random.default_rng(1)
+    for _ in range(200):
+        n = int(rng.integers(1, 40))
+        ids = rng.integers(0, 50, n)
+        entries = (ids << 2) | rng.integers(1, 3, n)
+        enc = O.lock_log(entries, sorted_log=False)
+        # first occurrences, in order (numpy unique's return_index)
+        _, first = np.unique(ids, return_index=True)
+        assert (enc >> 2).tolist() == ids[np.sort(first)].tolist()
+        assert sorted(enc.tolist()) == O.lock_log(entries).tolist()
+
+
 def random_script(rng, n_tx, words, n_steps):
     """Random interleaving of n_tx transactions; each tx: BEGIN, a few
     READ/WRITE, COMMIT.  Returns the op list."""
