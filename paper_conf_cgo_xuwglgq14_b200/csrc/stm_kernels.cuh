@@ -179,6 +179,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     TX tx;
     tx.reset_stats();
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
+    uint32_t seq_fails = 0;   // POL_BACKOFF: consecutive failed sequential steps of this warp
     // stage 0: start (or re-execute) transaction (t, i); stage 1: its body
     // ran and it waits for its locks (a lost lock round is retried in the
     // warp's next iteration, after the winners committed)
@@ -275,6 +276,18 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // retries in the next iteration; more than k_lock failed
             // sequential attempts abort the transaction.
             unsigned seq = __ballot_sync(FULL, act && stage == 1 && tries > 0);
+            // "a backoff mechanism specific to GPU": sequential
+            // locking removes the livelock inside a warp; across warps two
+            // sequential lanes can still take encounter-ordered locks
+            // crosswise again and again, so a warp whose sequential step
+            // failed waits a randomised, exponentially growing delay before
+            // the next one -- warp-uniform, the only delay SIMT allows
+            if (seq && seq_fails) {
+                const uint32_t cap = 256u << min(seq_fails, 8u);
+                const uint32_t r = static_cast<uint32_t>(gen::mix64((blockIdx.x * 8u + (threadIdx.x >> 5)) * 0x9E3779B97F4A7C15ull + iter));
+                __nanosleep(__shfl_sync(FULL, r, 0) % cap);
+            }
+            bool seq_failed = false;
             while (seq) {
                 const int L = __ffs(seq) - 1;
                 seq &= seq - 1;
@@ -293,6 +306,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                         done = true;
                     } else if (r == C_LOCK) {
                         cnt.inc(S_LOCK_RETRIES);
+                        seq_failed = true;
                         if (p.k_lock && ++tries > p.k_lock) {
                             stage = 0;
                             lock_aborted = true;
@@ -306,6 +320,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 sl = __shfl_sync(FULL, sl, L);
                 if (sl) { next_snap = sl; have_snap = true; }   // the latest own stamp: a valid snapshot
             }
+            seq_failed = __any_sync(FULL, seq_failed);
+            seq_fails = seq_failed ? seq_fails + 1u : 0u;
         }
         PHASE_MARK(PH_RELEASE);
         if (done || skip) {
