@@ -58,6 +58,8 @@ class Params(C.Structure):
         ("ht_key_range", C.c_uint64),
         ("km_clusters", C.c_uint32),
         ("km_dims", C.c_uint32),
+        ("shard_bits", C.c_uint32),
+        ("shard", C.c_uint32),
     ]
 
 
@@ -91,6 +93,7 @@ def lib():
         L.or_draw.restype = u64; L.or_draw.argtypes = [u64, u64]
         L.or_bounded.restype = u64; L.or_bounded.argtypes = [u64, u64]
         L.or_txkey.restype = u64; L.or_txkey.argtypes = [u64, u64, u64]
+        L.or_key_owner.restype = u32; L.or_key_owner.argtypes = [u64, u32]
         L.or_descr.restype = i32
         L.or_descr.argtypes = [P(Params), u64, u64, u64, P(u32), i32]
         L.or_footprint.restype = u64; L.or_footprint.argtypes = [P(Params), u64, u64]
@@ -141,6 +144,11 @@ def draw(x: int, k: int) -> int:
 
 def bounded(r: int, n: int) -> int:
     return lib().or_bounded(r, n)
+
+
+def key_owner(key: int, bits: int) -> int:
+    """Shard owning an HT key under a 2^bits-way partition."""
+    return lib().or_key_owner(key, bits)
 
 
 def txkey(seed: int, t: int, i: int) -> int:

@@ -65,6 +65,11 @@ static uint32_t lo32(uint64_t v) { return (uint32_t)(v & 0xffffffffull); }
  *               c_j = lo32(draw(A+j))
  *   KM        : c, f_0..f_{D-1}   c = bounded(draw0, C); f_d = draw(1+d) >> 56
  */
+uint32_t or_key_owner(uint64_t key, uint32_t bits)
+{
+    return bits ? (uint32_t)(or_mix64(key) >> (64 - bits)) : 0u;
+}
+
 int or_descr(const or_params_t* p, uint64_t seed, uint64_t t, uint64_t i,
              uint32_t* out, int cap)
 {
@@ -97,7 +102,18 @@ int or_descr(const or_params_t* p, uint64_t seed, uint64_t t, uint64_t i,
     }
     case OR_WL_HT: {
         if (cap < 3 || p->ht_buckets == 0 || (p->ht_buckets & (p->ht_buckets - 1))) return -1;
-        uint64_t key = 1 + or_bounded(or_draw(x, 0), p->ht_key_range);
+        if (p->shard_bits > 8 || (p->shard >> p->shard_bits) != 0) return -1;
+        /* Key partition: the shard draws keys by rejection on
+         * the transaction's stream -- candidate 0 is draw 0 (the unpartitioned
+         * key), candidate j >= 1 is draw j+1 (draw 1 is the insert flag) --
+         * and takes the first one it owns.  4096 candidates bound the loop;
+         * running out (probability (1-2^-bits)^4096 < 1e-200) is an error. */
+        uint64_t key = 0;
+        for (uint64_t j = 0; j < 4096; ++j) {
+            uint64_t k = 1 + or_bounded(or_draw(x, j ? j + 1 : 0), p->ht_key_range);
+            if (or_key_owner(k, p->shard_bits) == p->shard) { key = k; break; }
+        }
+        if (key == 0) return -1;
         out[0] = (uint32_t)key;
         out[1] = or_bounded(or_draw(x, 1), 100) >= p->ht_lookup_pct ? 1u : 0u;
         out[2] = (uint32_t)(or_mix64(key) & (uint64_t)(p->ht_buckets - 1));

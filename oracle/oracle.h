@@ -51,6 +51,8 @@ typedef struct {
     uint64_t ht_key_range;  /* HT: keys uniform in [1, ht_key_range]            */
     uint32_t km_clusters;   /* KM: clusters                                     */
     uint32_t km_dims;       /* KM: features per point                           */
+    uint32_t shard_bits;    /* HT key partition: G = 2^shard_bits  */
+    uint32_t shard;         /* HT: this shard g in [0, G); 0 bits = no partition */
 } or_params_t;
 
 /* ---------------- gen.c: the seeded input generator ---------------------- */
@@ -64,6 +66,9 @@ uint64_t or_txkey(uint64_t seed, uint64_t t, uint64_t i);
  * small / params invalid. */
 int or_descr(const or_params_t* p, uint64_t seed, uint64_t t, uint64_t i,
              uint32_t* out, int cap);
+/* Owner shard of an HT key under a 2^bits-way key partition:
+ * the top `bits` bits of mix64(key) (the bucket uses the low bits). */
+uint32_t or_key_owner(uint64_t key, uint32_t bits);
 /* Heap words the workload needs for T threads x K transactions. */
 uint64_t or_footprint(const or_params_t* p, uint64_t T, uint64_t K);
 /* Workload-defined initial heap. */

@@ -75,30 +75,43 @@ __device__ __forceinline__ uint32_t warp_stamp(unsigned long long* clock, bool g
     return static_cast<uint32_t>(base) + __popc(gm & prim::lanemask_lt()) + 1u;
 }
 
-// Statistics counters: one block-shared array (shared-memory atomics on the
-// rare events), flushed to the launch's counters with one global atomic per
-// counter per block.  Kept out of registers (they cost occupancy).
+// Statistics counters: one private 32-bit slot per thread and counter in
+// block-shared memory (sh[k * kMaxBlock + threadIdx.x]: consecutive threads,
+// consecutive banks), bumped with a plain shared load/add/store -- no atomics,
+// so no same-address serialisation when every lane of a warp counts the same
+// event (a 64-bit shared atomicAdd is a CAS loop on sm_100a: up to 32 rounds
+// per warp and event).  Kept out of registers (they cost occupancy).  A slot
+// cannot wrap: every event costs at least one L2 round trip (> 300 ns) and
+// the watchdog ends a launch within timeout_ms (default 60 s), so one thread
+// counts < 2^28 events per launch.  At exit, a warp shuffle reduction and
+// one global atomic per counter per warp.
+constexpr int kMaxBlock = 256;
 struct Counters {
-    unsigned long long* sh;
+    uint32_t* sh;
     bool error = false;
     __device__ __forceinline__ void inc(int k, uint32_t v = 1u)
     {
-        if (v) atomicAdd(&sh[k], static_cast<unsigned long long>(v));
+        sh[k * kMaxBlock + threadIdx.x] += v;
         if (k == S_ERRORS) error = true;
     }
 };
 
 #define GSTM_COUNTERS(name)                                                 \
-    __shared__ unsigned long long name##_sh[S_NSTATS];                      \
-    if (threadIdx.x < S_NSTATS) name##_sh[threadIdx.x] = 0;                 \
-    __syncthreads();                                                        \
+    __shared__ uint32_t name##_sh[S_NSTATS * kMaxBlock];                    \
+    for (int k_ = 0; k_ < S_NSTATS; ++k_) name##_sh[k_ * kMaxBlock + threadIdx.x] = 0u; \
     Counters name{name##_sh}
 
-// block totals -> one global atomic per counter per block
+// per-warp totals -> one global atomic per counter per warp
 __device__ __forceinline__ void flush_counters(Counters& cnt, unsigned long long* stats)
 {
-    __syncthreads();
-    if (threadIdx.x < S_NSTATS && cnt.sh[threadIdx.x]) atomicAdd(stats + threadIdx.x, cnt.sh[threadIdx.x]);
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < S_NSTATS; ++k) {
+        unsigned long long v = cnt.sh[k * kMaxBlock + threadIdx.x];
+#pragma unroll
+        for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(prim::FULL, v, o);
+        if (prim::lane_id() == 0 && v) atomicAdd(stats + k, v);
+    }
 }
 
 __device__ __forceinline__ void set_err(unsigned long long* meta, uint32_t bits)

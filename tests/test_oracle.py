@@ -516,3 +516,74 @@ def test_brute_matches_python_permutations():
     assert n == 6 and nd == len(outs)
     for h, r in outs:
         assert O.brute(p, init, T, K, seed, np.array(h), np.array(r))[1]
+
+
+# --------------------------------------------------------------------------
+# key-partitioned HT: shard g of G = 2^bits owns the keys whose
+# mix64 top bits are g; its transactions draw keys by rejection
+# --------------------------------------------------------------------------
+def test_key_partition_is_a_uniform_partition_independent_of_buckets():
+    keys = np.arange(1, 1 << 15)
+    for bits in (1, 2, 3):
+        G = 1 << bits
+        own = np.array([O.key_owner(int(k), bits) for k in keys])
+        assert own.min() == 0 and own.max() == G - 1
+        e = len(keys) / G
+        counts = np.bincount(own, minlength=G)
+        assert float(((counts - e) ** 2 / e).sum()) < 40, counts       # chi2, G-1 <= 7 dof
+        if bits > 1:   # nested: the top bits-1 bits are the coarser partition
+            coarse = np.array([O.key_owner(int(k), bits - 1) for k in keys])
+            assert (own >> 1 == coarse).all()
+    # the owner (top bits) is independent of the bucket (low bits): inside one
+    # shard the keys still spread over all 16 buckets uniformly
+    own = np.array([O.key_owner(int(k), 2) for k in keys])
+    buckets = np.array([O.lib().or_mix64(int(k)) & 15 for k in keys[own == 1]])
+    counts = np.bincount(buckets, minlength=16)
+    e = counts.sum() / 16
+    assert float(((counts - e) ** 2 / e).sum()) < 52, counts
+    assert O.key_owner(12345, 0) == 0
+
+
+@pytest.mark.parametrize("bits", [0, 1, 3])
+def test_sharded_ht_key_is_first_owned_candidate(bits):
+    KR, B = 1 << 22, 1 << 10
+    for g in range(1 << bits):
+        p = O.params("ht", ht_buckets=B, ht_lookup_pct=90, ht_key_range=KR, shard_bits=bits, shard=g)
+        for t in range(40):
+            for i in range(3):
+                x = O.txkey(7, t, i)
+                j, key = 0, None
+                while key is None:
+                    k = 1 + O.bounded(O.draw(x, j + 1 if j else 0), KR)
+                    if O.key_owner(k, bits) == g:
+                        key = k
+                    j += 1
+                d = O.descr(p, 7, t, i)
+                assert int(d[0]) == key
+                assert int(d[1]) == (1 if O.bounded(O.draw(x, 1), 100) >= 90 else 0)
+                assert int(d[2]) == O.lib().or_mix64(key) & (B - 1)
+                if bits == 0:   # no partition: the key is draw 0, as before
+                    assert key == 1 + O.bounded(O.draw(x, 0), KR)
+
+
+def test_sharded_ht_shards_are_disjoint_and_owned():
+    T, K, B, KR, bits = 64, 4, 32, 512, 2
+    M = T * K
+    sets = []
+    for g in range(1 << bits):
+        p = O.params("ht", ht_buckets=B, ht_lookup_pct=50, ht_key_range=KR, shard_bits=bits, shard=g)
+        heap = np.zeros(B + 2 * M, dtype=np.uint32)
+        res, upd = O.serial(p, heap, T, K, 11)
+        ks = [k for b in range(B) for k in _ht_walk(heap, B, M, b)]
+        assert len(ks) == len(set(ks)) == int((res == 3).sum())
+        assert all(O.key_owner(k, bits) == g for k in ks)
+        sets.append(set(ks))
+    for a in range(len(sets)):
+        for b in range(a + 1, len(sets)):
+            assert not (sets[a] & sets[b])
+
+
+def test_sharded_ht_bad_shard_is_an_error():
+    p = O.params("ht", ht_buckets=16, ht_lookup_pct=50, ht_key_range=64, shard_bits=1, shard=2)
+    with pytest.raises(Exception):
+        O.descr(p, 1, 0, 0)
