@@ -17,6 +17,13 @@ N > 1 (torchrun, one rank per GPU): key-partitioned bank -- every rank owns
 its own 2^20 accounts and runs shard-local transfers (weak scaling); NCCL is
 used once, after timing, to reduce the stats and the balance invariant.
 
+--workload ht: the key-partitioned hash table of SURVEY §8e (BASELINE
+configs[2] shape per GPU: 2^20 buckets, 2^22 STM threads x 4 operations,
+90/10 lookup/insert, keys in [1, 2^22]); rank g of N = 2^b owns the keys whose
+mix64 top b bits are g, so every transaction is shard-local; the table is
+re-initialised (outside the timed brackets) before every step; after timing,
+one all-reduce checks that the tables hold exactly the inserted keys.
+
 Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
@@ -55,6 +62,8 @@ def parse(argv=None):
     ap.add_argument("--tx-per-thread", type=int, default=TX_PER_THREAD)
     ap.add_argument("--no-cgl", action="store_true", help="skip the CGL/FGL baselines and the variant table")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--workload", default="bank", choices=["bank", "ht"],
+                    help="bank (BASELINE configs[1], the headline) or the key-partitioned hash table")
     return ap.parse_args(argv)
 
 
@@ -244,14 +253,16 @@ def from_vector(v):
     return d
 
 
-def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None):
+def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None, wl="bank"):
     """W warm-up launches, then `steps` launches enqueued back to back (no
     host sync), each bracketed by CUDA events on the launching stream, the L2
     flush outside the brackets.  Returns (step ms list, summed stats, wall s,
     clocks)."""
     import torch
     for w in range(warmup):
-        g.launch("bank", T, K, seed0 + 100000 + w)
+        if wl == "ht":
+            g.init_heap("ht")
+        g.launch(wl, T, K, seed0 + 100000 + w)
     torch.cuda.synchronize()
     g.reset_stats_total()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
@@ -262,9 +273,11 @@ def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None):
     wall0 = time.perf_counter()
     for k in range(steps):
         flush.fill_(float(k))
+        if wl == "ht":
+            g.init_heap("ht")      # node ids are per launch: every step starts from an empty table
         e0, e1 = evs[k]
         e0.record(stream)
-        g.launch("bank", T, K, seed0 + k)
+        g.launch(wl, T, K, seed0 + k)
         e1.record(stream)
     torch.cuda.synchronize()
     wall = time.perf_counter() - wall0
@@ -483,10 +496,149 @@ def run_native(args):
     return 0
 
 
+# ---------------------------------------------------------------------------
+# native arm, key-partitioned hash table
+# ---------------------------------------------------------------------------
+HT_BUCKETS, HT_THREADS, HT_K, HT_KEYS, HT_BITS = 1 << 20, 1 << 22, 4, 1 << 22, 22
+
+
+def ht_walk_count(heap, B, M):
+    """Nodes reachable from the B bucket heads (vectorised chain walk) and
+    the number of distinct keys among them (verification, after timing)."""
+    import numpy as np
+    heads = heap[:B].astype(np.int64)
+    key, nxt = heap[B:B + M], heap[B + M:B + 2 * M]
+    cur, seen = heads[heads != 0], []
+    for _ in range(M + 1):
+        if not cur.size:
+            break
+        seen.append(key[cur - 1])
+        cur = nxt[cur - 1].astype(np.int64)
+        cur = cur[cur != 0]
+    keys = np.concatenate(seen) if seen else np.zeros(0, np.uint32)
+    return int(keys.size), int(np.unique(keys).size)
+
+
+def run_native_ht(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world & (world - 1) == 0, "the key partition needs a power-of-two number of ranks"
+    args.gpus = world
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_cgo_xuwglgq14_b200 import build as B
+    if rank == 0 or world == 1:
+        B.build()
+    if world > 1:
+        dist.barrier()
+    from paper_conf_cgo_xuwglgq14_b200 import gstm as G
+
+    T, K = HT_THREADS, HT_K
+    M = T * K
+    words = HT_BUCKETS + 2 * M
+    mode = args.mode if args.mode in ("hv", "tbv", "auto", "fgl", "hv_backoff") else "hv"
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
+
+    def handle():
+        g = G.Gstm(words, HT_BITS)
+        g.set_workload_defaults("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90,
+                                shard_bits=world.bit_length() - 1, shard=rank, k_lock=args.k_lock)
+        g.set_mode(mode)
+        g.set_stream(stream)
+        g.init_heap("ht")
+        return g
+
+    g = handle()
+    flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)
+    seed0 = shard_seed(rank)
+    if world > 1:
+        dist.barrier()
+    step_ms, st_tot, wall, clocks = timed_steps(g, stream, flush, T, K, seed0, args.steps, args.warmup, local,
+                                                wl="ht")
+    if world > 1:
+        dist.barrier()
+    t_ms = float(sum(step_ms))
+    mode_used = G.MODE_NAMES[st_tot.mode_used]
+    last = g.stats()                                     # the last timed step
+    nodes, distinct = ht_walk_count(g.read_heap(), HT_BUCKETS, M)
+    ok_local = float(nodes == distinct == last.commits)
+    vec, (t_ms, wall) = reduce_over_ranks(list(stats_vector(st_tot)) + [nodes, ok_local], 0.0, t_ms, wall,
+                                          world, dist, dev)
+    tot = from_vector(vec[:16])
+    keys_total, ok_ranks = int(vec[16]), int(vec[17])
+    extra = {}
+    if rank == 0:
+        h_in = np.zeros(words, dtype=np.uint32)
+        pin_in = torch.from_numpy(h_in.view(np.int32)).pin_memory()
+        pin_out = torch.empty(words, dtype=torch.int32).pin_memory()
+        hi, ho = pin_in.numpy().view(np.uint32), pin_out.numpy().view(np.uint32)
+        g2 = handle()
+        g2.run_host("ht", hi, ho, T, K, seed0)
+        e2e_ms, e2e_done = 0.0, 0
+        for k in range(max(3, min(args.steps, 5))):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            st2 = g2.run_host("ht", hi, ho, T, K, seed0 + 7 + k)
+            b.record(stream)
+            b.synchronize()
+            e2e_ms += a.elapsed_time(b)
+            e2e_done += st2.commits + st2.commits_ro
+        extra["e2e"] = {"value": e2e_done / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": words * 4,
+                        "d2h_bytes_per_step": words * 4 + 200}
+        g2.close()
+        extra["roofline"] = None
+        extra["roofline_note"] = "the roofline object is reported for the bank headline (bench.py default)"
+        if world == 1 and not args.no_cpu:
+            import oracle as O
+            p = O.params("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90)
+            Ts = 1 << 20
+            heap = np.zeros(HT_BUCKETS + 2 * Ts * K, dtype=np.uint32)
+            t0 = time.perf_counter()
+            O.serial(p, heap, Ts, K, SEED)
+            dt = time.perf_counter() - t0
+            extra["cpu_baseline"] = {"value": Ts * K / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                     "sample": f"serial oracle, {Ts} threads x {K} HT operations, {dt:.2f} s"}
+    done = tot["commits"] + tot["commits_ro"]
+    if rank == 0:
+        value = done / (t_ms * 1e-3)
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": "hash table insert/lookup (BASELINE configs[2]), key-partitioned over ranks",
+                       "buckets_per_gpu": HT_BUCKETS, "threads_per_gpu": T, "tx_per_thread": K,
+                       "lookup_pct": 90, "key_range": HT_KEYS, "lock_table_bits": HT_BITS,
+                       "variant": f"{mode}/split/k_lock={args.k_lock} (mode used: {mode_used})",
+                       "partition": f"{world} shard(s): rank g owns keys with mix64 top {world.bit_length() - 1} bits = g",
+                       "l2": "flushed (256 MiB write) between timed steps"},
+            "abort_ratio": tot["aborts"] / max(1.0, tot["aborts"] + done),
+            "stats": {k: int(v) for k, v in tot.items()},
+            "invariant_keys_ok": ok_ranks == world, "keys_in_tables_last_step": keys_total,
+            "clocks": clocks, "gpu_launches": 3 * args.steps, "wall_s_timed_region": wall,
+        }
+        line.update(extra)
+        print(json.dumps(line), flush=True)
+    g.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
+    if args.workload == "ht":
+        return run_native_ht(args)
     return run_native(args)
 
 

@@ -104,6 +104,13 @@ typedef struct {
                              /*    n_threads STM threads (grid-stride); 0 = no cap     */
     uint32_t lock_shift;     /* stripe size 2^lock_shift words per version lock      */
                              /*    (lock = (word >> shift) mod 2^bits); default 0     */
+    uint32_t shard_bits;     /* HT key partition: G = 2^shard_bits     */
+                             /*    shards (<= 8 bits); 0 = no partition               */
+    uint32_t shard;          /* HT: this handle's shard g < G; it runs only keys     */
+                             /*    whose mix64 top shard_bits bits equal g            */
+    uint32_t km_stride;      /* KM: words per cluster record (>= km_dims + 1; 0 =    */
+                             /*    km_dims + 1).  32 with lock_shift 5 = one version */
+                             /*    lock per record                        */
 } gstm_params_t;
 
 typedef struct {

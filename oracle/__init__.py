@@ -60,6 +60,7 @@ class Params(C.Structure):
         ("km_dims", C.c_uint32),
         ("shard_bits", C.c_uint32),
         ("shard", C.c_uint32),
+        ("km_stride", C.c_uint32),
     ]
 
 

@@ -143,7 +143,7 @@ uint64_t or_footprint(const or_params_t* p, uint64_t T, uint64_t K)
     switch (p->workload) {
     case OR_WL_RA: case OR_WL_BANK: case OR_WL_EB: return p->n_words;
     case OR_WL_HT: return (uint64_t)p->ht_buckets + 2ull * T * K;
-    case OR_WL_KM: return (uint64_t)p->km_clusters * (p->km_dims + 1ull);
+    case OR_WL_KM: return (uint64_t)p->km_clusters * (p->km_stride ? p->km_stride : p->km_dims + 1ull);
     }
     return 0;
 }

@@ -53,6 +53,7 @@ typedef struct {
     uint32_t km_dims;       /* KM: features per point                           */
     uint32_t shard_bits;    /* HT key partition: G = 2^shard_bits  */
     uint32_t shard;         /* HT: this shard g in [0, G); 0 bits = no partition */
+    uint32_t km_stride;     /* KM: words per record, >= km_dims+1 (0: km_dims+1) */
 } or_params_t;
 
 /* ---------------- gen.c: the seeded input generator ---------------------- */

@@ -102,6 +102,9 @@ static WlParams wl_params(const gstm_params_t& p, uint64_t T, uint64_t K)
     w.ht_key_range = p.ht_key_range;
     w.km_clusters = p.km_clusters;
     w.km_dims = p.km_dims;
+    w.km_stride = p.km_stride ? p.km_stride : p.km_dims + 1;
+    w.shard_bits = p.shard_bits;
+    w.shard = p.shard;
     w.T = T;
     w.K = K;
     return w;

@@ -23,7 +23,8 @@ struct WlParams {
     uint32_t n_reads, n_writes, ra_kind, n_accesses;
     uint32_t ht_buckets, ht_lookup_pct;
     uint64_t ht_key_range;
-    uint32_t km_clusters, km_dims;
+    uint32_t km_clusters, km_dims, km_stride;   // KM record = km_stride words
+    uint32_t shard_bits, shard;                 // HT key partition
     uint64_t T, K;           // launch shape (HT node layout needs M = T*K)
 };
 
@@ -220,12 +221,26 @@ struct HtWL {
     __host__ static bool check(const WlParams& p)
     {
         return p.ht_buckets && !(p.ht_buckets & (p.ht_buckets - 1)) && p.ht_key_range >= 1 &&
-               p.ht_key_range < (1ull << 32) && p.ht_buckets + 2 * p.T * p.K < (1ull << 32);
+               p.ht_key_range < (1ull << 32) && p.ht_buckets + 2 * p.T * p.K < (1ull << 32) &&
+               p.shard_bits <= 8 && (p.shard >> p.shard_bits) == 0;
     }
     __host__ static uint64_t footprint(const WlParams& p) { return p.ht_buckets + 2 * p.T * p.K; }
+    // Key partition over G = 2^shard_bits GPUs: shard g owns
+    // the keys whose mix64 top bits are g (the bucket uses the low bits) and
+    // draws its keys by rejection on the transaction's own stream: candidate
+    // 0 is draw 0 (the unpartitioned key), candidate j >= 1 is draw j+1
+    // (draw 1 is the insert flag).  After 4096 candidates (probability
+    // (1-1/G)^4096 < 1e-200) key = 0 reports an error.
     __device__ __forceinline__ static void key_of(const WlParams& p, uint64_t x, uint32_t& key, uint32_t& ins, uint32_t& bucket)
     {
         key = 1u + static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.ht_key_range));
+        if (p.shard_bits) {
+            const int sh = 64 - static_cast<int>(p.shard_bits);
+            for (uint32_t j = 2; (gen::mix64(key) >> sh) != p.shard; ++j) {
+                if (j > 4096) { key = 0; break; }
+                key = 1u + static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.ht_key_range));
+            }
+        }
         ins = gen::bounded(gen::draw(x, 1), 100) >= p.ht_lookup_pct ? 1u : 0u;
         bucket = static_cast<uint32_t>(gen::mix64(key) & (p.ht_buckets - 1));
     }
@@ -234,6 +249,7 @@ struct HtWL {
     {
         uint32_t key, ins, bucket;
         key_of(p, x, key, ins, bucket);
+        if (key == 0) { c.overflow(); return; }        // no owned key drawn (never in practice)
         const uint64_t B = p.ht_buckets, M = p.T * p.K;
         const uint32_t h0 = c.read(bucket);
         if (!c.ok()) return;
@@ -323,7 +339,8 @@ struct EbWL {
 };
 
 // ---- k-means cluster update (STAMP kmeans' transactional step) -------------
-// record of cluster c = [count, sum_0 .. sum_{D-1}] at word c*(D+1).
+// record of cluster c = [count, sum_0 .. sum_{D-1}] at word c*stride (stride >= D+1;
+// the default D+1 packs the records, 32 aligns each to its own 128 B line).
 struct KmWL {
     static constexpr int MAXD = 16;
     static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
@@ -333,13 +350,17 @@ struct KmWL {
     static constexpr bool kLocalLogs = GSTM_KM_LOCAL_LOGS;
     static constexpr int kMinBlocks = GSTM_KM_LOCAL_LOGS ? 2 : 1;
     static constexpr int DESCR = MAXD + 1;
-    __host__ static bool check(const WlParams& p) { return p.km_clusters > 0 && p.km_dims <= MAXD; }
-    __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * (p.km_dims + 1); }
+    __host__ static bool check(const WlParams& p)
+    {
+        return p.km_clusters > 0 && p.km_dims <= MAXD && p.km_stride >= p.km_dims + 1 &&
+               uint64_t(p.km_clusters) * p.km_stride < (1ull << 32);
+    }
+    __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * p.km_stride; }
     template <class Ctx>
     __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
     {
         const int D = static_cast<int>(p.km_dims);
-        const uint32_t base = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * (p.km_dims + 1);
+        const uint32_t base = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * p.km_stride;
         uint32_t a[MAXD + 1], v[MAXD + 1];
 #pragma unroll
         for (int k = 0; k <= MAXD; ++k) a[k] = base + k;
@@ -354,7 +375,7 @@ struct KmWL {
     template <class F>
     __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
     {
-        f(static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * (p.km_dims + 1));   // one lock per record
+        f(static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * p.km_stride);   // one lock per record
     }
     __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
     {

@@ -39,10 +39,13 @@ WL_CASES = [
     ("bank", dict(n_words=1 << 20)),
     ("bank", dict(n_words=3)),
     ("ht", dict(ht_buckets=1 << 20, ht_lookup_pct=90, ht_key_range=1 << 22)),
+    ("ht", dict(ht_buckets=1 << 20, ht_lookup_pct=90, ht_key_range=1 << 22, shard_bits=3, shard=5)),
+    ("ht", dict(ht_buckets=64, ht_lookup_pct=50, ht_key_range=100, shard_bits=1, shard=0)),
     ("eb", dict(n_accesses=64, n_words=1 << 26)),
     ("eb", dict(n_accesses=9, n_words=1000)),
     ("km", dict(km_clusters=1024, km_dims=16)),
     ("km", dict(km_clusters=5, km_dims=3)),
+    ("km", dict(km_clusters=1024, km_dims=16, km_stride=32)),
 ]
 
 

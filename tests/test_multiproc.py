@@ -80,3 +80,54 @@ def test_shard_seeds_are_distinct():
     import bench
     seeds = {bench.shard_seed(r) for r in range(8)}
     assert len(seeds) == 8
+
+
+def _ht_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    B, T, K, KR = 64, 128, 4, 2048
+    M = T * K
+    bits = world.bit_length() - 1
+    p = O.params("ht", ht_buckets=B, ht_key_range=KR, ht_lookup_pct=50, shard_bits=bits, shard=rank)
+    heap = np.zeros(B + 2 * M, dtype=np.uint32)
+    res, upd = O.serial(p, heap, T, K, bench.shard_seed(rank))
+    nodes, distinct = bench.ht_walk_count(heap, B, M)
+    ok = float(nodes == distinct == int(upd.sum()))
+    vec = np.zeros(16)
+    vec[0] = upd.sum()
+    out, _ = bench.reduce_over_ranks(list(vec) + [nodes, ok], 0.0, 1.0, 0.0, world, dist, torch.device("cpu"))
+    keys = sorted(int(heap[B + n - 1]) for n in range(1, M + 1) if heap[B + n - 1])
+    q.put((rank, out.tolist(), keys))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_two_rank_key_partitioned_ht_gloo():
+    """bench.py --workload ht host logic: each rank's shard (here the
+    oracle's serial run of it) holds only keys it owns; the one reduction
+    sums the key counts and the per-rank invariant flags."""
+    import sys
+    sys.path.insert(0, ROOT)
+    import oracle as O
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ht_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    total = sum(len(k) for _, _, k in got)
+    for rank, out, keys in got:
+        assert out[16] == total and out[17] == world             # key count SUM; every rank's invariant held
+        assert out[0] == total                                   # update commits = inserted keys
+        assert all(O.key_owner(k, 1) == rank for k in keys)
+    assert not set(got[0][2]) & set(got[1][2])                   # disjoint shards

@@ -147,17 +147,21 @@ def test_ra_increment_closed_form():
     assert int(heap.astype(np.uint64).sum()) == N * (N - 1) // 2 + R * T * K
 
 
-def test_km_closed_form():
+@pytest.mark.parametrize("stride", [0, 17, 32])
+def test_km_closed_form(stride):
     T, K, Cn, D = 16, 8, 4, 16
-    p = O.params("km", km_clusters=Cn, km_dims=D)
-    heap = np.zeros(Cn * (D + 1), dtype=np.uint32)
+    S = stride or D + 1
+    p = O.params("km", km_clusters=Cn, km_dims=D, km_stride=stride)
+    heap = np.zeros(Cn * S, dtype=np.uint32)
+    assert O.footprint(p, T, K) == Cn * S
     res, upd = O.serial(p, heap, T, K, 8)
     d = np.array([O.descr(p, 8, t, i) for i in range(K) for t in range(T)], dtype=np.int64)
     cnt = np.bincount(d[:, 0], minlength=Cn)
     sums = np.zeros((Cn, D), dtype=np.int64)
     np.add.at(sums, d[:, 0], d[:, 1:])
-    rec = heap.reshape(Cn, D + 1)
-    assert (rec[:, 0] == cnt).all() and (rec[:, 1:] == sums).all()
+    rec = heap.reshape(Cn, S)
+    assert (rec[:, 0] == cnt).all() and (rec[:, 1:D + 1] == sums).all()
+    assert (rec[:, D + 1:] == 0).all()          # record padding is never touched
     # result = count before: per cluster the results are 0..cnt-1 in order
     for c in range(Cn):
         assert sorted(res[d[:, 0] == c].tolist()) == list(range(cnt[c]))

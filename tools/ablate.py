@@ -90,7 +90,10 @@ def main():
         pad_mb = int(kv.pop("pad_mb", 0))       # shift where the handle's buffers land
         pad = torch.empty(pad_mb << 18, dtype=torch.float32, device="cuda") if pad_mb else None
         paired = bool(int(kv.pop("paired", 0)))
-        g = G.Gstm(shp["words"], bits, paired=paired)
+        words = int(kv.pop("words", 0)) or shp["words"]
+        if wl == "km" and "km_stride" in kv:
+            words = 1024 * int(kv["km_stride"])
+        g = G.Gstm(words, bits, paired=paired)
         if flush is None:
             flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
         g.set_workload_defaults(wl, **shp["params"], **{k: int(v) for k, v in kv.items()})
@@ -98,7 +101,7 @@ def main():
         g.set_stream(stream)
         theap = None
         if a.torch_heap:
-            theap = torch.empty(shp["words"], dtype=torch.int32, device="cuda")
+            theap = torch.empty(words, dtype=torch.int32, device="cuda")
             g.attach_heap(theap)
         g.init_heap(wl)
         for w in range(a.warmup):
