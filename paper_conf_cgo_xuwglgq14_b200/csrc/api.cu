@@ -86,6 +86,9 @@ static gstm_params_t default_params(int workload)
     p.lock_pipeline = 1;
     if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
     if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
+    // EB: the sequential first round is faster even when the lock log fits
+    // one pipelined chunk (A=8: 1.24 vs 0.94 G tx/s)
+    if (workload == GSTM_WL_EB) p.lock_pipeline = 0;
     return p;
 }
 

@@ -299,13 +299,44 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
         return true;
     }
 
+    // local-memory logs: kChunk atom.or.b64 at a time (tx.cuh)
+    static constexpr int kChunk = 8;
+    __device__ __forceinline__ bool get_locks_and_tbv_pipelined_local(const Meta& m)
+    {
+        bool ok = true;
+        for (int k0 = 0; k0 < nl; k0 += kChunk) {
+            unsigned long long old[kChunk];
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) old[j] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k0 + j] >> 2), 1ull << 32);
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) {
+                    l_old[k0 + j] = hi(old[j]);
+                    l_val[k0 + j] = lo(old[j]);
+                    ok &= !(hi(old[j]) & 1u);
+                }
+        }
+        prim::fence_acquire();
+        if (!ok) {
+            for (int k = 0; k < nl; ++k)
+                if (!(l_old[k] & 1u)) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), mk(l_val[k], l_old[k]));
+            n_acq = 0;
+            return false;
+        }
+        for (int k = 0; k < nl; ++k)
+            if ((l_ent[k] & 1u) && (l_old[k] >> 1) > snapshot) passTBV = false;
+        n_acq = nl;
+        return true;
+    }
+
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
         bool got;
         if constexpr (kUnroll) got = pipelined ? get_locks_and_tbv_pipelined(m) : get_locks_and_tbv(m);
-        else got = get_locks_and_tbv(m);
+        else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; }

@@ -96,7 +96,7 @@ def main():
         g = G.Gstm(words, bits, paired=paired)
         if flush is None:
             flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
-        g.set_workload_defaults(wl, **shp["params"], **{k: int(v) for k, v in kv.items()})
+        g.set_workload_defaults(wl, **dict(shp["params"], **{k: int(v) for k, v in kv.items()}))
         g.set_mode(mode)
         g.set_stream(stream)
         theap = None
