@@ -61,6 +61,10 @@ def full(path: str) -> dict:
     for m in FULL_METRICS:
         if m in col:
             out[m] = {"value": v[col[m]], "unit": u[col[m]]}
+    # every L2 request / sector breakdown the report holds (source unit, op)
+    out["l2_breakdown"] = {n: v[i] for n, i in col.items()
+                           if (n.startswith("lts__t_requests_srcunit") or n.startswith("lts__t_sectors_srcunit"))
+                           and n.endswith(".sum") and v[i] not in ("", "0", "n/a")}
     out["stalls_per_issue"] = {}
     for s in STALLS:
         n = f"smsp__average_warps_issue_stalled_{s}_per_issue_active.ratio"
