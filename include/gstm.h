@@ -100,7 +100,7 @@ typedef struct {
     uint32_t lock_pipeline;  /* 1: a transaction's first lock-acquisition round issues */
                              /*    all atom.or at once; later rounds  */
                              /*    are sequential in ascending id.  Local-memory logs  */
-                             /*    pipeline only logs of <= 8 locks.  Default 1 (EB: 0) */
+                             /*    pipeline only logs of <= 8 locks.  Default 1 (RA, EB: 0) */
     uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
                              /*    n_threads STM threads (grid-stride); 0 = no cap     */
     uint32_t lock_shift;     /* stripe size 2^lock_shift words per version lock      */

@@ -229,8 +229,8 @@ struct Tx {
         return false;
     }
 
-    // ---- A3.l27-33: wait while locked, then timestamp check --------------
-    __device__ __forceinline__ void check_lock(const Meta& m, uint32_t a, uint32_t vl, int mode)
+    // ---- A3.l27-29: wait while locked; returns the unlocked lock word -----
+    __device__ __forceinline__ uint32_t settle_lock(const Meta& m, uint32_t a, uint32_t vl)
     {
         uint32_t spins = 0;
         while (vl & 1u) {                                            // l.29
@@ -239,7 +239,12 @@ struct Tx {
             vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));      // l.28
         }
         n_spin += spins;
-        const uint32_t version = vl >> 1;                            // l.30
+        return vl;
+    }
+
+    // ---- A3.l30-33: timestamp check, PostValidation (HV) or abort (TBV) ---
+    __device__ __forceinline__ void check_version(const Meta& m, uint32_t version, int mode)
+    {
         if (opaque && version > snapshot) {                          // l.31
             if (mode == MODE_HV) {
                 if (!post_validation(m, version)) opaque = false;    // l.32-33
@@ -247,6 +252,13 @@ struct Tx {
                 opaque = false;                                      // TBV-only (Q18)
             }
         }
+    }
+
+    // ---- A3.l27-33: wait while locked, then timestamp check --------------
+    __device__ __forceinline__ void check_lock(const Meta& m, uint32_t a, uint32_t vl, int mode)
+    {
+        vl = settle_lock(m, a, vl);                                  // l.27-29
+        check_version(m, vl >> 1, mode);                             // l.30-33
     }
 
     // ---- A3.l21-35 TXRead(addr) -------------------------------------------
@@ -269,7 +281,14 @@ struct Tx {
     // Equivalent to N sequential TXReads with the value loads hoisted: each
     // value is still checked against its lock after it was loaded (DESIGN.md
     // §6.3), but the transaction pays 2 dependent memory round trips instead
-    // of 2N.
+    // of 2N.  For batches of more than 4 words the timestamp checks are
+    // merged: PostValidation
+    // (l.32) runs at most once, with the newest version seen, after every
+    // read of the batch is in the read-set -- the outcome sequential reads
+    // reach (a read-set consistent at a snapshot >= every version read), and
+    // one inlined copy of the rare path instead of N (code size: the
+    // instruction cache).  The lock inserts go through one
+    // rolled loop for the same reason.
     template <int N>
     __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode)
     {
@@ -287,12 +306,30 @@ struct Tx {
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
+        if constexpr (N <= 4) {
+            // small batches (bank: 2): per-read checks, fully unrolled
 #pragma unroll
-        for (int k = 0; k < N; ++k)
-            if (need[k]) {
-                check_lock(m, a[k], vl[k], mode);                    // l.27-33
-                insert_lock((m.lock_of(a[k]) << 2) | 1u);       // l.34
+            for (int k = 0; k < N; ++k)
+                if (need[k]) {
+                    check_lock(m, a[k], vl[k], mode);                // l.27-33
+                    insert_lock((m.lock_of(a[k]) << 2) | 1u);        // l.34
+                }
+        } else {
+            uint32_t newest = 0;
+#pragma unroll
+            for (int k = 0; k < N; ++k)
+                if (need[k]) newest = max(newest, settle_lock(m, a[k], vl[k]) >> 1);   // l.27-30
+            check_version(m, newest, mode);                          // l.31-33
+#pragma unroll 1
+            for (int k = 0; k < N; ++k) {
+                uint32_t ak = 0;
+                bool nk = false;
+#pragma unroll
+                for (int j = 0; j < N; ++j)
+                    if (j == k) { ak = a[j]; nk = need[j]; }
+                if (nk) insert_lock((m.lock_of(ak) << 2) | 1u);
             }
+        }
     }
 
     // Batched TXRead of n words (n only known at run time; arrays in local

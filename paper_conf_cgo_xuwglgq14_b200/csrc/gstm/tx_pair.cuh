@@ -141,19 +141,43 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
+        if constexpr (N <= 4) {
+            // small batches (bank: 2): per-read checks, fully unrolled
 #pragma unroll
-        for (int k = 0; k < N; ++k)
-            if (need[k]) {
-                pv[k] = settle(m, a[k], pv[k]);
-                v[k] = lo(pv[k]);
-                append_read(a[k], v[k]);
-            }
+            for (int k = 0; k < N; ++k)
+                if (need[k]) {
+                    pv[k] = settle(m, a[k], pv[k]);
+                    v[k] = lo(pv[k]);
+                    append_read(a[k], v[k]);
+                }
 #pragma unroll
-        for (int k = 0; k < N; ++k)
-            if (need[k]) {
-                check_version(m, hi(pv[k]), mode);
-                insert_lock((a[k] << 2) | 1u);
+            for (int k = 0; k < N; ++k)
+                if (need[k]) {
+                    check_version(m, hi(pv[k]), mode);
+                    insert_lock((a[k] << 2) | 1u);
+                }
+        } else {
+            uint32_t newest = 0;
+#pragma unroll
+            for (int k = 0; k < N; ++k)
+                if (need[k]) {
+                    pv[k] = settle(m, a[k], pv[k]);
+                    v[k] = lo(pv[k]);
+                    append_read(a[k], v[k]);
+                    newest = max(newest, hi(pv[k]) >> 1);
+                }
+            // one merged timestamp check per batch (tx.cuh read_batch)
+            check_version(m, newest << 1, mode);
+#pragma unroll 1
+            for (int k = 0; k < N; ++k) {
+                uint32_t ak = 0;
+                bool nk = false;
+#pragma unroll
+                for (int j = 0; j < N; ++j)
+                    if (j == k) { ak = a[j]; nk = need[j]; }
+                if (nk) insert_lock((ak << 2) | 1u);
             }
+        }
     }
 
     __device__ __forceinline__ void read_many(const Meta& m, const uint32_t* a, uint32_t* v, const bool* skip, int n,

@@ -85,7 +85,14 @@ __device__ __forceinline__ uint32_t lo32(uint64_t v) { return static_cast<uint32
 struct RaWL {
     static constexpr int MAXR = 8, MAXW = 8;
     static constexpr int RCAP = MAXR, WCAP = MAXW, LCAP = MAXR + MAXW, FGL_LCAP = MAXR + MAXW;
-    static constexpr int kMinBlocks = 2;
+#ifndef GSTM_RA_LOCAL_LOGS
+#define GSTM_RA_LOCAL_LOGS 1    // local-memory logs: 1.6x over the 128-register unrolled logs
+#endif
+    static constexpr bool kLocalLogs = GSTM_RA_LOCAL_LOGS;
+#ifndef GSTM_RA_MINB
+#define GSTM_RA_MINB 2
+#endif
+    static constexpr int kMinBlocks = GSTM_RA_MINB;
     static constexpr int DESCR = MAXR + 2 * MAXW;
     __host__ static bool check(const WlParams& p)
     {
@@ -106,12 +113,14 @@ struct RaWL {
 #pragma unroll
         for (int j = 0; j < MAXR; ++j)
             if (j < R) acc += v[j];
-#pragma unroll
-        for (int j = 0; j < MAXW; ++j)
-            if (j < W) {
-                const uint32_t w = static_cast<uint32_t>(gen::bounded(gen::draw(x, R + j), p.n_words));
-                c.write(w, acc + lo32(gen::draw(x, R + W + j)));
-            }
+        // rolled: one inlined copy of TXWrite (its sorted insert is unrolled
+        // over the lock log) instead of MAXW -- keeps the kernel's code in
+        // the instruction cache
+#pragma unroll 1
+        for (int j = 0; j < W; ++j) {
+            const uint32_t w = static_cast<uint32_t>(gen::bounded(gen::draw(x, R + j), p.n_words));
+            c.write(w, acc + lo32(gen::draw(x, R + W + j)));
+        }
         result = acc;
     }
     template <class F>
@@ -135,6 +144,7 @@ struct RaWL {
 struct RaIncWL {
     static constexpr int MAXR = 16;
     static constexpr int RCAP = MAXR, WCAP = MAXR, LCAP = MAXR, FGL_LCAP = MAXR;
+    static constexpr bool kLocalLogs = GSTM_RA_LOCAL_LOGS;
     static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = MAXR;
     __host__ static bool check(const WlParams& p) { return p.ra_kind == 1 && p.n_reads <= MAXR && p.n_words > 0; }
@@ -367,9 +377,8 @@ struct KmWL {
         c.template read_batch<MAXD + 1>(a, v, D + 1);
         if (!c.ok()) return;
         c.write(base, v[0] + 1u);
-#pragma unroll
-        for (int d = 0; d < MAXD; ++d)
-            if (d < D) c.write(base + 1 + d, v[1 + d] + static_cast<uint32_t>(gen::draw(x, 1 + d) >> 56));
+#pragma unroll 1
+        for (int d = 0; d < D; ++d) c.write(base + 1 + d, v[1 + d] + static_cast<uint32_t>(gen::draw(x, 1 + d) >> 56));
         result = v[0];
     }
     template <class F>
