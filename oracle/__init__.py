@@ -61,6 +61,7 @@ class Params(C.Structure):
         ("shard_bits", C.c_uint32),
         ("shard", C.c_uint32),
         ("km_stride", C.c_uint32),
+        ("km_assign", C.c_uint32),
     ]
 
 
@@ -95,6 +96,9 @@ def lib():
         L.or_bounded.restype = u64; L.or_bounded.argtypes = [u64, u64]
         L.or_txkey.restype = u64; L.or_txkey.argtypes = [u64, u64, u64]
         L.or_key_owner.restype = u32; L.or_key_owner.argtypes = [u64, u32]
+        L.or_km_centroids.restype = u64; L.or_km_centroids.argtypes = [P(Params)]
+        L.or_km_nearest.restype = u32; L.or_km_nearest.argtypes = [P(Params), P(u32), P(u32)]
+        L.or_km_recenter.restype = None; L.or_km_recenter.argtypes = [P(Params), P(u32)]
         L.or_descr.restype = i32
         L.or_descr.argtypes = [P(Params), u64, u64, u64, P(u32), i32]
         L.or_footprint.restype = u64; L.or_footprint.argtypes = [P(Params), u64, u64]
@@ -145,6 +149,22 @@ def draw(x: int, k: int) -> int:
 
 def bounded(r: int, n: int) -> int:
     return lib().or_bounded(r, n)
+
+
+def km_centroids(p: Params) -> int:
+    """Word offset of the k-means centroid table (after the records)."""
+    return lib().or_km_centroids(C.byref(p))
+
+
+def km_nearest(p: Params, heap: np.ndarray, f) -> int:
+    f = np.ascontiguousarray(f, dtype=np.uint32)
+    return lib().or_km_nearest(C.byref(p), _p(heap, C.c_uint32), _p(f, C.c_uint32))
+
+
+def km_recenter(p: Params, heap: np.ndarray) -> None:
+    """End of a Lloyd iteration (in place): centroids = floor means, records zeroed."""
+    assert heap.dtype == np.uint32 and heap.flags.c_contiguous
+    lib().or_km_recenter(C.byref(p), _p(heap, C.c_uint32))
 
 
 def key_owner(key: int, bits: int) -> int:

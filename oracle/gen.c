@@ -143,13 +143,19 @@ uint64_t or_footprint(const or_params_t* p, uint64_t T, uint64_t K)
     switch (p->workload) {
     case OR_WL_RA: case OR_WL_BANK: case OR_WL_EB: return p->n_words;
     case OR_WL_HT: return (uint64_t)p->ht_buckets + 2ull * T * K;
-    case OR_WL_KM: return (uint64_t)p->km_clusters * (p->km_stride ? p->km_stride : p->km_dims + 1ull);
+    case OR_WL_KM: return or_km_centroids(p) + (p->km_assign ? (uint64_t)p->km_clusters * p->km_dims : 0);
     }
     return 0;
 }
 
+uint64_t or_km_centroids(const or_params_t* p)
+{
+    return (uint64_t)p->km_clusters * (p->km_stride ? p->km_stride : p->km_dims + 1ull);
+}
+
 /* Initial heaps: RA and EB heap[k] = k; bank 1000 per
- * account; HT empty (all heads null, node words 0); KM all records zero. */
+ * account; HT empty (all heads null, node words 0); KM all records zero and,
+ * with km_assign, centroid word j of the table = splitmix64(j) >> 56. */
 void or_init_heap(const or_params_t* p, uint32_t* heap, uint64_t words)
 {
     for (uint64_t k = 0; k < words; ++k) {
@@ -158,5 +164,9 @@ void or_init_heap(const or_params_t* p, uint32_t* heap, uint64_t words)
         case OR_WL_BANK: heap[k] = 1000u; break;
         default: heap[k] = 0u; break;
         }
+    }
+    if (p->workload == OR_WL_KM && p->km_assign) {
+        uint64_t c0 = or_km_centroids(p), n = (uint64_t)p->km_clusters * p->km_dims;
+        for (uint64_t j = 0; j < n && c0 + j < words; ++j) heap[c0 + j] = (uint32_t)(or_splitmix64(j) >> 56);
     }
 }

@@ -54,6 +54,8 @@ typedef struct {
     uint32_t shard_bits;    /* HT key partition: G = 2^shard_bits  */
     uint32_t shard;         /* HT: this shard g in [0, G); 0 bits = no partition */
     uint32_t km_stride;     /* KM: words per record, >= km_dims+1 (0: km_dims+1) */
+    uint32_t km_assign;     /* KM: 1 = cluster = nearest centroid of the table   */
+                            /*     after the records (a full Lloyd iteration)    */
 } or_params_t;
 
 /* ---------------- gen.c: the seeded input generator ---------------------- */
@@ -74,6 +76,16 @@ uint32_t or_key_owner(uint64_t key, uint32_t bits);
 uint64_t or_footprint(const or_params_t* p, uint64_t T, uint64_t K);
 /* Workload-defined initial heap. */
 void or_init_heap(const or_params_t* p, uint32_t* heap, uint64_t words);
+
+/* k-means, full iteration (km_assign = 1): the centroid
+ * table (km_clusters x km_dims uint32) follows the records at word
+ * or_km_centroids(p).  or_km_nearest = argmin_c sum_d (f_d - cent[c][d])^2,
+ * exact integer arithmetic, ties to the lowest c.  or_km_recenter ends an
+ * iteration: cent[c][d] = floor(sum_d / count) for every record with count >
+ * 0 (others keep their centroid), then every record is zeroed. */
+uint64_t or_km_centroids(const or_params_t* p);
+uint32_t or_km_nearest(const or_params_t* p, const uint32_t* heap, const uint32_t* f);
+void or_km_recenter(const or_params_t* p, uint32_t* heap);
 
 /* ---------------- serial.c: serial executor and stamp-order replay ------- */
 /* Execute transaction (t,i) serially on heap.  *result = observable result,

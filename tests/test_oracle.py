@@ -591,3 +591,60 @@ def test_sharded_ht_bad_shard_is_an_error():
     p = O.params("ht", ht_buckets=16, ht_lookup_pct=50, ht_key_range=64, shard_bits=1, shard=2)
     with pytest.raises(Exception):
         O.descr(p, 1, 0, 0)
+
+
+# --------------------------------------------------------------------------
+# k-means full iteration (km_assign = 1): assignment + update transactions +
+# recenter = one Lloyd step of STAMP kmeans
+# --------------------------------------------------------------------------
+def _km_table(p, heap):
+    c0 = O.km_centroids(p)
+    return heap[c0:c0 + p.km_clusters * p.km_dims].reshape(p.km_clusters, p.km_dims).astype(np.int64)
+
+
+@pytest.mark.parametrize("Cn,D", [(37, 5), (64, 16), (1, 3)])
+def test_km_nearest_is_brute_force_argmin(Cn, D):
+    rng = np.random.default_rng(Cn * 100 + D)
+    p = O.params("km", km_clusters=Cn, km_dims=D, km_assign=1)
+    heap = np.zeros(O.footprint(p, 1, 1), dtype=np.uint32)
+    cent = rng.integers(0, 256, (Cn, D))
+    if Cn > 2:
+        cent[Cn - 1] = cent[1]                     # a duplicate row: the lower index must win
+    heap[O.km_centroids(p):] = cent.reshape(-1)
+    for _ in range(300):
+        f = rng.integers(0, 256, D)
+        d2 = ((f[None, :] - cent) ** 2).sum(1)
+        assert O.km_nearest(p, heap, f) == int(np.argmin(d2))      # argmin: first minimum
+    if Cn > 2:
+        assert O.km_nearest(p, heap, cent[1]) == 1
+
+
+def test_km_init_centroids_and_footprint():
+    p = O.params("km", km_clusters=8, km_dims=4, km_stride=8, km_assign=1)
+    assert O.km_centroids(p) == 64 and O.footprint(p, 3, 3) == 64 + 32
+    heap = O.init_heap(p, 96)
+    assert not heap[:64].any()
+    assert heap[64:].tolist() == [O.splitmix64(j) >> 56 for j in range(32)]
+
+
+@pytest.mark.parametrize("stride", [0, 32])
+def test_km_full_iteration_is_a_lloyd_step(stride):
+    T, K, Cn, D = 64, 8, 16, 4
+    p = O.params("km", km_clusters=Cn, km_dims=D, km_stride=stride, km_assign=1)
+    S = stride or D + 1
+    heap = O.init_heap(p, O.footprint(p, T, K))
+    for it in range(3):
+        cent = _km_table(p, heap).copy()
+        res, upd = O.serial(p, heap, T, K, 40 + it)
+        feats = np.array([O.descr(p, 40 + it, t, i)[1:] for i in range(K) for t in range(T)], dtype=np.int64)
+        assign = np.argmin(((feats[:, None, :] - cent[None, :, :]) ** 2).sum(2), axis=1)
+        rec = heap[:Cn * S].reshape(Cn, S).astype(np.int64)
+        cnt = np.bincount(assign, minlength=Cn)
+        sums = np.zeros((Cn, D), dtype=np.int64)
+        np.add.at(sums, assign, feats)
+        assert (rec[:, 0] == cnt).all() and (rec[:, 1:D + 1] == sums).all()
+        assert (_km_table(p, heap) == cent).all()            # transactions never touch the centroids
+        O.km_recenter(p, heap)
+        want = np.where(cnt[:, None] > 0, sums // np.maximum(cnt, 1)[:, None], cent)
+        assert (_km_table(p, heap) == want).all()
+        assert not heap[:Cn * S].any()                       # accumulators restart from zero
