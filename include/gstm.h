@@ -112,6 +112,12 @@ typedef struct {
     uint32_t km_stride;      /* KM: words per cluster record (>= km_dims + 1; 0 =    */
                              /*    km_dims + 1).  32 with lock_shift 5 = one version */
                              /*    lock per record                        */
+    uint32_t km_assign;      /* KM: 1 = a full k-means iteration:   */
+                             /*    each point joins its NEAREST centroid (exact int  */
+                             /*    squared distance, ties -> lowest index) from the  */
+                             /*    km_clusters x km_dims uint32 table stored after   */
+                             /*    the records; gstm_launch runs the assignment pass */
+                             /*    before the update transactions.  Table <= 64 KiB  */
 } gstm_params_t;
 
 typedef struct {
@@ -228,6 +234,15 @@ int gstm_read_tx_log(gstm_t* h, uint32_t* stamps, uint32_t* results, uint64_t n)
  * heap_in/heap_out may alias; pinned memory gives full copy bandwidth. */
 int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
                   uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed, gstm_stats_t* stats);
+
+/* End of a k-means iteration (params.km_assign = 1; STAMP kmeans):
+ * for every cluster record with count > 0, centroid[c][d] = floor(sum_d /
+ * count) (others keep their centroid), then every record is zeroed, ready
+ * for the next iteration's gstm_launch.  Asynchronous on the handle's
+ * stream.  GSTM_EINVAL without km_assign or if the heap cannot hold the
+ * records and the centroid table.  gstm_init_heap(GSTM_WL_KM) with
+ * km_assign fills the table with centroid word j = splitmix64(j) >> 56. */
+int gstm_km_recenter(gstm_t* h);
 
 /* ---- test and measurement entry points --------------------------------- */
 /* Transaction descriptors as generated on the device:

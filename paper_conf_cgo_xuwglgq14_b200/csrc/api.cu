@@ -50,6 +50,8 @@ struct gstm_handle {
     uint32_t* tx_stamp = nullptr;
     uint32_t* tx_result = nullptr;
     uint64_t log_cap = 0;
+    uint32_t* km_cluster = nullptr;  // KM full iteration: per-tx nearest centroid (km.cu)
+    uint64_t km_cap = 0;
     cudaStream_t own_stream = nullptr, stream = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     gstm_params_t params{};
@@ -107,6 +109,8 @@ static WlParams wl_params(const gstm_params_t& p, uint64_t T, uint64_t K)
     w.km_clusters = p.km_clusters;
     w.km_dims = p.km_dims;
     w.km_stride = p.km_stride ? p.km_stride : p.km_dims + 1;
+    w.km_assign = p.km_assign;
+    w.km_cluster = nullptr;
     w.shard_bits = p.shard_bits;
     w.shard = p.shard;
     w.T = T;
@@ -243,6 +247,7 @@ void gstm_destroy(gstm_t* h)
     cudaFree(h->scratch);
     cudaFree(h->tx_stamp);
     cudaFree(h->tx_result);
+    cudaFree(h->km_cluster);
     if (h->ev0) cudaEventDestroy(h->ev0);
     if (h->ev1) cudaEventDestroy(h->ev1);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -311,10 +316,47 @@ static int ensure_scratch(gstm_t* h, uint64_t words)
     return GSTM_OK;
 }
 
+// the device view of the handle's heap and lock table (tx.cuh Meta)
+static Meta meta_of(const gstm_t* h)
+{
+    Meta m;
+    memset(&m, 0, sizeof(m));
+    m.heap = h->heap;
+    m.locks = h->locks;
+    m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
+    m.clock = h->clock;
+    m.spin_cap = h->params.spin_cap ? h->params.spin_cap : (1u << 16);
+    m.lock_shift = h->params.lock_shift;
+    m.vshift = m.lshift = h->paired ? 1u : 0u;
+    return m;
+}
+
 int gstm_init_heap(gstm_t* h, int workload)
 {
     if (!h || workload < 0 || workload > 4) { set_error("gstm_init_heap: bad argument"); return GSTM_EINVAL; }
     CUDA_TRY(launch_init_heap(workload, h->heap, h->heap_words, h->paired ? 1 : 0, h->stream));
+    const gstm_params_t& P = h->params;
+    if (workload == GSTM_WL_KM && P.km_assign) {
+        // the centroid table after the records
+        const uint64_t stride = P.km_stride ? P.km_stride : P.km_dims + 1ull;
+        const uint64_t c0 = uint64_t(P.km_clusters) * stride, n = uint64_t(P.km_clusters) * P.km_dims;
+        if (c0 + n > h->heap_words) { set_error("gstm_init_heap: k-means centroid table beyond the heap"); return GSTM_EINVAL; }
+        CUDA_TRY(launch_km_init_centroids(meta_of(h), c0, n, h->stream));
+    }
+    return GSTM_OK;
+}
+
+int gstm_km_recenter(gstm_t* h)
+{
+    if (!h) { set_error("gstm_km_recenter: NULL handle"); return GSTM_EINVAL; }
+    const gstm_params_t& P = h->params;
+    const uint64_t stride = P.km_stride ? P.km_stride : P.km_dims + 1ull;
+    if (!P.km_assign || P.km_clusters == 0 || P.km_dims > 16 || stride < P.km_dims + 1ull ||
+        uint64_t(P.km_clusters) * (stride + P.km_dims) > h->heap_words) {
+        set_error("gstm_km_recenter: needs km_assign = 1 and a heap holding the records and the centroid table");
+        return GSTM_EINVAL;
+    }
+    CUDA_TRY(launch_km_recenter(meta_of(h), P.km_clusters, P.km_dims, static_cast<uint32_t>(stride), h->stream));
     return GSTM_OK;
 }
 
@@ -459,16 +501,26 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
         }
         h->log_cap = n_tx;
     }
+    const bool km_assign = workload == GSTM_WL_KM && P.km_assign;
+    if (km_assign && n_tx > h->km_cap) {
+        cudaFree(h->km_cluster);
+        h->km_cluster = nullptr;
+        h->km_cap = 0;
+        if (cudaMalloc(&h->km_cluster, n_tx * 4) != cudaSuccess) {
+            h->km_cluster = nullptr;
+            set_error("gstm_launch: cannot allocate the k-means assignment (%llu points)", (unsigned long long)n_tx);
+            return GSTM_ENOMEM;
+        }
+        h->km_cap = n_tx;
+    }
+    if (km_assign && uint64_t(P.km_clusters) * P.km_dims > 16384) {
+        set_error("gstm_launch: k-means centroid table > 64 KiB (km_clusters * km_dims > 16384)");
+        return GSTM_EINVAL;
+    }
     const int mode = resolve_mode(h, fp);
     KParams kp;
     memset(&kp, 0, sizeof(kp));
-    kp.m.heap = h->heap;
-    kp.m.locks = h->locks;
-    kp.m.lock_mask = static_cast<uint32_t>((1ull << h->bits) - 1);
-    kp.m.clock = h->clock;
-    kp.m.spin_cap = P.spin_cap ? P.spin_cap : (1u << 16);
-    kp.m.lock_shift = P.lock_shift;
-    kp.m.vshift = kp.m.lshift = h->paired ? 1u : 0u;
+    kp.m = meta_of(h);
     kp.paired = h->paired ? 1u : 0u;
     kp.w = w;
     kp.meta = h->meta;
@@ -486,6 +538,11 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));
+    if (km_assign && n_tx) {
+        // a full k-means iteration: every point's nearest centroid first
+        CUDA_TRY(launch_km_assign(kp, h->km_cluster, h->stream));
+        kp.w.km_cluster = h->km_cluster;
+    }
     CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
     CUDA_TRY(launch_finish(h->meta, h->clock, h->stream));
     CUDA_TRY(cudaEventRecord(h->ev1, h->stream));

@@ -24,6 +24,8 @@ struct WlParams {
     uint32_t ht_buckets, ht_lookup_pct;
     uint64_t ht_key_range;
     uint32_t km_clusters, km_dims, km_stride;   // KM record = km_stride words
+    uint32_t km_assign;                         // KM: cluster = nearest centroid (full iteration)
+    const uint32_t* km_cluster;                 // KM, km_assign: per-tx cluster from km_assign_kernel
     uint32_t shard_bits, shard;                 // HT key partition
     uint64_t T, K;           // launch shape (HT node layout needs M = T*K)
 };
@@ -365,12 +367,24 @@ struct KmWL {
         return p.km_clusters > 0 && p.km_dims <= MAXD && p.km_stride >= p.km_dims + 1 &&
                uint64_t(p.km_clusters) * p.km_stride < (1ull << 32);
     }
-    __host__ static uint64_t footprint(const WlParams& p) { return uint64_t(p.km_clusters) * p.km_stride; }
+    // records, then (km_assign) the C x D centroid table
+    __host__ static uint64_t footprint(const WlParams& p)
+    {
+        return uint64_t(p.km_clusters) * p.km_stride + (p.km_assign ? uint64_t(p.km_clusters) * p.km_dims : 0);
+    }
+    // the transaction's cluster: drawn by the generator, or (a full k-means
+    // iteration) its point's nearest centroid, computed before the launch's
+    // transactions by km_assign_kernel (km.cu)
+    __device__ __forceinline__ static uint32_t cluster(const WlParams& p, uint64_t x, uint64_t t, uint64_t i)
+    {
+        if (p.km_cluster) return p.km_cluster[i * p.T + t];
+        return static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters));
+    }
     template <class Ctx>
-    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t t, uint64_t i, uint32_t& result)
     {
         const int D = static_cast<int>(p.km_dims);
-        const uint32_t base = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * p.km_stride;
+        const uint32_t base = cluster(p, x, t, i) * p.km_stride;
         uint32_t a[MAXD + 1], v[MAXD + 1];
 #pragma unroll
         for (int k = 0; k <= MAXD; ++k) a[k] = base + k;
@@ -382,9 +396,9 @@ struct KmWL {
         result = v[0];
     }
     template <class F>
-    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t t, uint64_t i, F&& f)
     {
-        f(static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters)) * p.km_stride);   // one lock per record
+        f(cluster(p, x, t, i) * p.km_stride);   // one lock per record
     }
     __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
     {

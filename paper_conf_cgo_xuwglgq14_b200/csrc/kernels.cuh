@@ -68,6 +68,9 @@ cudaError_t launch_lock_halves(uint32_t* pairs, uint64_t words, uint32_t* out, c
 cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
                           cudaStream_t s);
 cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s);
+cudaError_t launch_km_assign(const KParams& kp, uint32_t* cluster, cudaStream_t s);
+cudaError_t launch_km_init_centroids(const Meta& m, uint64_t c0, uint64_t n, cudaStream_t s);
+cudaError_t launch_km_recenter(const Meta& m, uint32_t C, uint32_t D, uint32_t stride, cudaStream_t s);
 int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
 int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s);
 int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_words, uint32_t* locks, uint32_t lmask,

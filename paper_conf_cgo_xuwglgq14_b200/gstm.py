@@ -38,7 +38,7 @@ EXPORTS = [
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
     "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
-    "gstm_lock_log", "gstm_ubench",
+    "gstm_lock_log", "gstm_ubench", "gstm_km_recenter",
 ]
 
 
@@ -56,6 +56,7 @@ class gstm_params_t(C.Structure):
         ("spin_cap", C.c_uint32), ("timeout_ms", C.c_uint32), ("snapshot_reuse", C.c_uint32),
         ("lock_pipeline", C.c_uint32), ("max_threads", C.c_uint32), ("lock_shift", C.c_uint32),
         ("shard_bits", C.c_uint32), ("shard", C.c_uint32), ("km_stride", C.c_uint32),
+        ("km_assign", C.c_uint32),
     ]
 
 
@@ -104,6 +105,7 @@ def lib():
             "gstm_heap_words": (u64, [V]),
             "gstm_heap_ptr": (V, [V]),
             "gstm_init_heap": (i32, [V, i32]),
+            "gstm_km_recenter": (i32, [V]),
             "gstm_write_heap": (i32, [V, V, u64, u64]),
             "gstm_read_heap": (i32, [V, V, u64, u64]),
             "gstm_read_locks": (i32, [V, V, u64]),
@@ -275,6 +277,11 @@ class Gstm:
     # data
     def init_heap(self, workload) -> None:
         _check(lib().gstm_init_heap(self.h, _wl(workload)), "gstm_init_heap")
+
+    def km_recenter(self) -> None:
+        """End of a k-means iteration (params.km_assign = 1): centroids =
+        floor means of their records, records zeroed (asynchronous)."""
+        _check(lib().gstm_km_recenter(self.h), "gstm_km_recenter")
 
     def write_heap(self, a: np.ndarray, offset: int = 0) -> None:
         a = np.ascontiguousarray(a, dtype=np.uint32)
