@@ -33,6 +33,16 @@
 #ifndef GSTM_SPIN_NS
 #define GSTM_SPIN_NS 32
 #endif
+// measurement only (NOT a supported build): acquire operations become relaxed
+// and fence.acquire disappears, to price the CCTL.IVALL they compile to
+#ifndef GSTM_EXPERIMENT_NO_ACQ
+#define GSTM_EXPERIMENT_NO_ACQ 0
+#endif
+#if GSTM_EXPERIMENT_NO_ACQ
+#define GSTM_ACQ "relaxed"
+#else
+#define GSTM_ACQ "acquire"
+#endif
 
 namespace gstm {
 namespace prim {
@@ -49,14 +59,14 @@ __device__ __forceinline__ uint32_t ld_relaxed(const uint32_t* p)
 __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p)
 {
     uint32_t v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    asm volatile("ld." GSTM_ACQ ".gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
 
 __device__ __forceinline__ unsigned long long ld_acquire64(const unsigned long long* p)
 {
     unsigned long long v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    asm volatile("ld." GSTM_ACQ ".gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 
@@ -93,7 +103,11 @@ __device__ __forceinline__ void fence_acq_rel()
 // (value loads before lock-word loads).
 __device__ __forceinline__ void fence_acquire()
 {
+#if GSTM_EXPERIMENT_NO_ACQ
+    asm volatile("" ::: "memory");
+#else
     asm volatile("fence.acquire.gpu;" ::: "memory");
+#endif
 }
 
 // Release fence: orders every earlier access before the strong writes after
@@ -107,14 +121,14 @@ __device__ __forceinline__ void fence_release()
 __device__ __forceinline__ unsigned long long atom_add_acquire64(unsigned long long* p, unsigned long long v)
 {
     unsigned long long old;
-    asm volatile("atom.acquire.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    asm volatile("atom." GSTM_ACQ ".gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
     return old;
 }
 
 __device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t v)
 {
     uint32_t old;
-    asm volatile("atom.acquire.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    asm volatile("atom." GSTM_ACQ ".gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
     return old;
 }
 
@@ -135,7 +149,7 @@ __device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned l
 __device__ __forceinline__ unsigned long long atom_or_acquire_u64(unsigned long long* p, unsigned long long v)
 {
     unsigned long long old;
-    asm volatile("atom.acquire.gpu.global.or.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    asm volatile("atom." GSTM_ACQ ".gpu.global.or.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
     return old;
 }
 
@@ -156,7 +170,7 @@ __device__ __forceinline__ uint32_t atom_or_relaxed(uint32_t* p, uint32_t v)
 __device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, uint32_t v)
 {
     uint32_t old;
-    asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;"
+    asm volatile("atom." GSTM_ACQ ".gpu.global.cas.b32 %0, [%1], %2, %3;"
                  : "=r"(old) : "l"(p), "r"(cmp), "r"(v) : "memory");
     return old;
 }
@@ -165,7 +179,7 @@ __device__ __forceinline__ unsigned long long atom_cas_acquire64(unsigned long l
                                                                  unsigned long long v)
 {
     unsigned long long old;
-    asm volatile("atom.acquire.gpu.global.cas.b64 %0, [%1], %2, %3;"
+    asm volatile("atom." GSTM_ACQ ".gpu.global.cas.b64 %0, [%1], %2, %3;"
                  : "=l"(old) : "l"(p), "l"(cmp), "l"(v) : "memory");
     return old;
 }
