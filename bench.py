@@ -436,6 +436,10 @@ def run_native(args):
         pin_out = torch.empty(ACCOUNTS, dtype=torch.int32).pin_memory()
         h_in = pin_in.numpy().view(np.uint32)
         h_out = pin_out.numpy().view(np.uint32)
+        # e2e through the blocking call, one step at a time.  (Double-buffered
+        # gstm_run_host_async on two handles/streams measured slower on one
+        # B200, 6.82 vs 7.10 G tx/s: the two persistent grids share the SMs and
+        # L2 -- DESIGN.md §7.1.)
         g2 = var.handle(G, stream)
         g2.run_host("bank", h_in, h_out, T, K, seed0)        # warm-up
         e2e_ms, e2e_done = 0.0, 0
@@ -450,7 +454,8 @@ def run_native(args):
             e2e_ms += a.elapsed_time(b)
             e2e_done += st2.commits + st2.commits_ro
         extra["e2e"] = {"value": e2e_done / (e2e_ms * 1e-3), "unit": UNIT,
-                        "h2d_bytes_per_step": ACCOUNTS * 4, "d2h_bytes_per_step": ACCOUNTS * 4 + 200}
+                        "h2d_bytes_per_step": ACCOUNTS * 4, "d2h_bytes_per_step": ACCOUNTS * 4 + 200,
+                        "api": "gstm_run_host (host buffers, pinned), one step at a time"}
         g2.close()
         if not args.no_cgl:
             extra["cgl"] = cgl_baseline(G, stream, T, seed0)

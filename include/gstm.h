@@ -244,6 +244,18 @@ int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* he
  * km_assign fills the table with centroid word j = splitmix64(j) >> 56. */
 int gstm_km_recenter(gstm_t* h);
 
+/* As gstm_run_host without the final synchronisation: the copy-in, the
+ * launch and the copy-out are enqueued on the handle's stream and the call
+ * returns.  heap_in must stay valid and heap_out must not be read until
+ * gstm_sync (or gstm_stats) returns.  With pinned host buffers the copies
+ * are asynchronous, so two handles on two streams overlap one step's copies
+ * with the other's transactions (double-buffered streaming). */
+int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
+                        uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed);
+/* Wait for everything enqueued on the handle's stream; returns the status of
+ * the last launch (GSTM_OK if none). */
+int gstm_sync(gstm_t* h);
+
 /* ---- test and measurement entry points --------------------------------- */
 /* Transaction descriptors as generated on the device:
  * host_out[(i*n_threads + t) * words_per_tx + k]; short descriptors are

@@ -627,6 +627,26 @@ int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* he
     return gstm_stats(h, stats ? stats : &local);
 }
 
+int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
+                        uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed)
+{
+    if (!h || words > h->heap_words || (words && (!heap_in || !heap_out))) { set_error("gstm_run_host_async: bad buffers"); return GSTM_EINVAL; }
+    int rc = copy_in(h, heap_in, 0, words);
+    if (rc) return rc;
+    rc = gstm_launch(h, workload, n_threads, tx_per_thread, seed);
+    if (rc) return rc;
+    return copy_out(h, heap_out, 0, words);
+}
+
+int gstm_sync(gstm_t* h)
+{
+    if (!h) { set_error("gstm_sync: NULL handle"); return GSTM_EINVAL; }
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (!h->launched) return GSTM_OK;
+    gstm_stats_t s;
+    return gstm_stats(h, &s);
+}
+
 int gstm_descr_words(gstm_t* h, int workload)
 {
     if (!h) { set_error("gstm_descr_words: NULL"); return GSTM_EINVAL; }

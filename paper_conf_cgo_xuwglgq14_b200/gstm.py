@@ -38,7 +38,7 @@ EXPORTS = [
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
     "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
-    "gstm_lock_log", "gstm_ubench", "gstm_km_recenter",
+    "gstm_lock_log", "gstm_ubench", "gstm_km_recenter", "gstm_run_host_async", "gstm_sync",
 ]
 
 
@@ -106,6 +106,8 @@ def lib():
             "gstm_heap_ptr": (V, [V]),
             "gstm_init_heap": (i32, [V, i32]),
             "gstm_km_recenter": (i32, [V]),
+            "gstm_run_host_async": (i32, [V, i32, V, V, u64, u64, u32, u64]),
+            "gstm_sync": (i32, [V]),
             "gstm_write_heap": (i32, [V, V, u64, u64]),
             "gstm_read_heap": (i32, [V, V, u64, u64]),
             "gstm_read_locks": (i32, [V, V, u64]),
@@ -354,6 +356,16 @@ class Gstm:
         _check(lib().gstm_run_host(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
                                    n_threads, tx_per_thread, seed, C.byref(s)), "gstm_run_host")
         return s
+
+    def run_host_async(self, workload, heap_in: np.ndarray, heap_out: np.ndarray, n_threads: int,
+                       tx_per_thread: int, seed: int) -> None:
+        """Enqueue copy-in, launch and copy-out; heap_out is valid after sync()."""
+        assert heap_in.dtype == np.uint32 and heap_out.dtype == np.uint32 and heap_in.size == heap_out.size
+        _check(lib().gstm_run_host_async(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
+                                         n_threads, tx_per_thread, seed), "gstm_run_host_async")
+
+    def sync(self) -> int:
+        return _check(lib().gstm_sync(self.h), "gstm_sync")
 
     # tests / measurement
     def descr_words(self, workload) -> int:

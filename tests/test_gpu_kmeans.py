@@ -27,10 +27,12 @@ def _closed_form(op, heap_before, feats):
     c0 = O.km_centroids(op)
     cent = heap_before[c0:c0 + Cn * D].reshape(Cn, D).astype(np.int64)
     # squared distances in uint64 (exact here: < 2^64; int64 would overflow
-    # for centroid words near 2^32)
-    diff = (feats[:, None, :] - cent[None, :, :]).astype(np.uint64)
-    d2 = (diff * diff).sum(2, dtype=np.uint64)
-    assign = np.argmin(d2, axis=1)                       # ties: first (lowest) index
+    # for centroid words near 2^32), 2048 points at a time
+    assign = np.empty(len(feats), dtype=np.int64)
+    for s in range(0, len(feats), 2048):
+        diff = (feats[s:s + 2048, None, :] - cent[None, :, :]).astype(np.uint64)
+        d2 = (diff * diff).sum(2, dtype=np.uint64)
+        assign[s:s + 2048] = np.argmin(d2, axis=1)       # ties: first (lowest) index
     cnt = np.bincount(assign, minlength=Cn)
     sums = np.zeros((Cn, D), dtype=np.int64)
     np.add.at(sums, assign, feats)
@@ -40,7 +42,7 @@ def _closed_form(op, heap_before, feats):
 @pytest.mark.parametrize("mode,paired,stride,shift", [("hv", False, 0, 0), ("tbv", True, 0, 0), ("fgl", False, 0, 0),
                                                       ("hv", False, 32, 5)])
 def test_km_full_iterations(mode, paired, stride, shift):
-    T, K, Cn, D = 1 << 16, 2, 1024, 16
+    T, K, Cn, D = 1 << 14, 2, 1024, 16
     bits = 20 if not paired else 16
     g, gp, op, init = U.make("km", T, K, bits, mode=mode, paired=paired, km_assign=1, km_stride=stride,
                              lock_shift=shift)

@@ -422,6 +422,33 @@ def test_run_host_and_attached_torch_heap():
     assert (h == t.cpu().numpy().view(np.uint32)).all()
 
 
+@pytest.mark.parametrize("paired", [False, True])
+def test_run_host_async_double_buffered(paired):
+    """gstm_run_host_async on two handles and two streams (the bench's
+    end-to-end path): every step's host output replays bit-exactly."""
+    import torch
+    T, K, N = 1 << 14, 4, 1 << 14
+    hs = [U.make("bank", T, K, 14, mode="hv", paired=paired, n_words=N) for _ in range(2)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    h_in = torch.full((N,), 1000, dtype=torch.int32).pin_memory().numpy().view(np.uint32)
+    outs = [torch.zeros(N, dtype=torch.int32).pin_memory().numpy().view(np.uint32) for _ in range(4)]
+    for (g, *_), s in zip(hs, streams):
+        g.set_stream(s)
+    for k in range(4):
+        hs[k % 2][0].run_host_async("bank", h_in, outs[k], T, K, 20 + k)
+    for g, *_ in hs:
+        assert g.sync() == 0
+    # each handle's last step is replayable from the input
+    for j, (g, gp, op, init) in enumerate(hs):
+        k = 2 + j
+        stamps, res = g.read_tx_log(T * K)
+        h = h_in.copy()
+        assert O.replay(op, h, T, K, 20 + k, stamps, res)[0] == 0
+        assert (h == outs[k]).all()
+    for k in range(4):
+        assert int(outs[k].astype(np.int64).sum()) == 1000 * N
+
+
 @pytest.mark.parametrize("kind", [0, 1, 2, 3, 4, 5])
 def test_ubench_runs(kind):
     ops, ms = G.gstm_ubench(kind, 8 << 20, 1 << 22, 148 * 256 * 4)
