@@ -463,7 +463,11 @@ def run_native(args):
             table = [Variant("auto", "split"), Variant("tbv", "split"), Variant("hv", "split"),
                      Variant("tbv", "paired"), Variant("hv", "paired", prelock=1),
                      Variant("hv_backoff", "split"), Variant("hv_backoff", "paired", k_lock=1),
-                     Variant("fgl", "split"), Variant("fgl", "paired")]
+                     Variant("fgl", "split"), Variant("fgl", "paired"),
+                     # FGL launches one CUDA thread per STM thread; also give the
+                     # hand-locking ceiling the concurrency the STM grid runs at
+                     # (16 warps per SM), its measured best
+                     Variant("fgl", "split", max_threads=512 * torch.cuda.get_device_properties(dev).multi_processor_count)]
             extra["variants"] = variant_table(G, stream, flush, T, K, seed0,
                                               [v for v in table if v.name != var.name])
             fgl = [v for k, v in extra["variants"].items() if k.startswith("fgl")]

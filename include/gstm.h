@@ -97,10 +97,13 @@ typedef struct {
     uint32_t snapshot_reuse; /* 1: a warp that just committed starts its next txs at   */
                              /*    the clock value after its own commits instead of   */
                              /*    re-reading g_clock (A3.l4); default 1               */
-    uint32_t lock_pipeline;  /* 1: a transaction's first lock-acquisition round issues */
-                             /*    all atom.or at once; later rounds  */
-                             /*    are sequential in ascending id.  Local-memory logs  */
-                             /*    pipeline only logs of <= 8 locks.  Default 1 (RA, EB: 0) */
+    uint32_t lock_pipeline;  /* N > 0: the first lock-acquisition round of each of a   */
+                             /*    transaction's first N executions issues all atom.or */
+                             /*    at once; every other round is      */
+                             /*    sequential in ascending id (progress is kept for    */
+                             /*    any finite N).  0: always sequential.  Local-memory */
+                             /*    logs pipeline only logs of <= 8 locks.              */
+                             /*    Default 1 (RA, EB: 0)                               */
     uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
                              /*    n_threads STM threads (grid-stride); 0 = no cap     */
     uint32_t lock_shift;     /* stripe size 2^lock_shift words per version lock      */

@@ -83,6 +83,9 @@ struct Tx {
     uint32_t snapshot;
     bool opaque, passTBV, overflow;
     uint32_t n_postval, n_vbv, n_spin;    // per-thread statistics
+    // lanes of the warp that run this body together and call read_batch
+    // exactly once (a convergent workload, stm_kernels.cuh); 0 = unknown
+    unsigned sync_mask;
 
     __device__ __forceinline__ void reset_stats() { n_postval = n_vbv = n_spin = 0; }
 
@@ -95,6 +98,15 @@ struct Tx {
         opaque = passTBV = true;                  // l.3
         overflow = false;
         snapshot = snap;                          // l.4
+        sync_mask = 0u;
+    }
+
+    // Reconverge the lanes that run their bodies together after a rare,
+    // per-lane path (a lock spin, PostValidation): without it the warp stays
+    // split and executes the rest of the body once per group of lanes.
+    __device__ __forceinline__ void reconverge() const
+    {
+        if (sync_mask) __syncwarp(sync_mask);
     }
 
     __device__ __forceinline__ bool read_only() const { return nw == 0; }
@@ -307,19 +319,44 @@ struct Tx {
         for (int k = 0; k < N; ++k)
             if (need[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
         if constexpr (N <= 4) {
-            // small batches (bank: 2): per-read checks, fully unrolled
+            // small batches (bank: 2), fully unrolled: ONE spin loop re-reads
+            // every still-locked lock word of the batch together (l.27-29)
+            // and ONE timestamp check with the newest version (Q35): one copy
+            // of each rare path, so the lanes of a warp that take it take it
+            // together instead of one after the other
+            uint32_t spins = 0;
+            bool locked = false;
+#pragma unroll
+            for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
+            while (locked) {
+                if (++spins > m.spin_cap) { opaque = false; break; }
+                if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
+#pragma unroll
+                for (int k = 0; k < N; ++k)
+                    if (need[k] && (vl[k] & 1u)) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));   // l.28
+                locked = false;
+#pragma unroll
+                for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
+            }
+            n_spin += spins;
+            reconverge();
+            uint32_t newest = 0;
 #pragma unroll
             for (int k = 0; k < N; ++k)
-                if (need[k]) {
-                    check_lock(m, a[k], vl[k], mode);                // l.27-33
-                    insert_lock((m.lock_of(a[k]) << 2) | 1u);        // l.34
-                }
+                if (need[k]) newest = max(newest, vl[k] >> 1);
+            check_version(m, newest, mode);                          // l.30-33 (Q35)
+            reconverge();
+#pragma unroll
+            for (int k = 0; k < N; ++k)
+                if (need[k]) insert_lock((m.lock_of(a[k]) << 2) | 1u);   // l.34
         } else {
             uint32_t newest = 0;
 #pragma unroll
             for (int k = 0; k < N; ++k)
                 if (need[k]) newest = max(newest, settle_lock(m, a[k], vl[k]) >> 1);   // l.27-30
+            reconverge();
             check_version(m, newest, mode);                          // l.31-33
+            reconverge();
 #pragma unroll 1
             for (int k = 0; k < N; ++k) {
                 uint32_t ak = 0;
@@ -469,6 +506,54 @@ struct Tx {
         return true;
     }
 
+    // Register-resident logs: the pipelined first round and the sequential
+    // sorted acquisition in ONE code path, so the lanes of a warp that make a
+    // first attempt and those that retry after a lock abort share their memory
+    // round trips instead of running one branch after the other: round 0
+    // issues entry 0 for every lane and every entry for a pipelined lane;
+    // sequential lanes then take entries 1.. one at a time in ascending id,
+    // stopping at the first held lock (Q15), in lockstep with each other.
+    __device__ __forceinline__ bool get_locks_and_tbv_converged(const Meta& m, bool pipelined)
+    {
+        static_assert(kUnroll, "converged acquisition needs register-resident logs");
+        uint32_t vl[LCAP];
+        bool ok = true;
+        uint32_t set = 0;   // entries this attempt locked
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (k == 0 || pipelined)) vl[k] = prim::atom_or_relaxed(m.lock_ptr(l_ent[k] >> 2), 1u);   // l.45
+        prim::fence_acquire();
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (k == 0 || pipelined)) {
+                if (vl[k] & 1u) ok = false;                          // l.46
+                else set |= 1u << k;
+            }
+#pragma unroll
+        for (int k = 1; k < LCAP; ++k)
+            if (!pipelined && ok && k < nl) {                        // next entry only after the last succeeded
+                vl[k] = prim::atom_or_relaxed(m.lock_ptr(l_ent[k] >> 2), 1u);
+                prim::fence_acquire();
+                if (vl[k] & 1u) ok = false;
+                else set |= 1u << k;
+            }
+        if (!ok) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)                           // l.47: undo what this attempt set
+                if (set & (1u << k)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), vl[k]);
+            n_acq = 0;
+            return false;
+        }
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) {
+                l_old[k] = vl[k];
+                if ((l_ent[k] & 1u) && (vl[k] >> 1) > snapshot) passTBV = false;   // l.49-51
+            }
+        n_acq = nl;
+        return true;
+    }
+
     // The same first round for local-memory logs (EB, HT, KM): the atom.or go
     // out kChunk at a time (their results land in registers, then in the
     // local log), so a transaction with n locks pays ceil(n / kChunk) memory
@@ -515,7 +600,7 @@ struct Tx {
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
         bool got;
-        if constexpr (kUnroll) got = pipelined ? get_locks_and_tbv_pipelined(m) : get_locks_and_tbv(m);
+        if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
         else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75

@@ -43,6 +43,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
     using B::n_spin;
     using B::raw_lookup;
     using B::append_read;
+    using B::reconverge;
     using B::insert_lock;
 
     uint32_t l_val[LCAP];   // value each acquiring atom.or.b64 returned
@@ -142,20 +143,40 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
         for (int k = 0; k < N; ++k)
             if (need[k]) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
         if constexpr (N <= 4) {
-            // small batches (bank: 2): per-read checks, fully unrolled
+            // small batches (bank: 2), fully unrolled: ONE spin loop re-reads
+            // every still-locked pair of the batch together (l.27-29), and ONE
+            // timestamp check with the newest version (Q35) -- a single copy
+            // of each rare path, so lanes of a warp that take it take it
+            // together instead of one after the other
+            uint32_t spins = 0;
+            bool locked = false;
+#pragma unroll
+            for (int k = 0; k < N; ++k) locked |= need[k] && (hi(pv[k]) & 1u);
+            while (locked) {
+                if (++spins > m.spin_cap) { opaque = false; break; }
+                if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
+#pragma unroll
+                for (int k = 0; k < N; ++k)
+                    if (need[k] && (hi(pv[k]) & 1u)) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
+                locked = false;
+#pragma unroll
+                for (int k = 0; k < N; ++k) locked |= need[k] && (hi(pv[k]) & 1u);
+            }
+            n_spin += spins;
+            reconverge();
+            uint32_t newest = 0;
 #pragma unroll
             for (int k = 0; k < N; ++k)
                 if (need[k]) {
-                    pv[k] = settle(m, a[k], pv[k]);
                     v[k] = lo(pv[k]);
                     append_read(a[k], v[k]);
+                    newest = max(newest, hi(pv[k]) >> 1);
                 }
+            check_version(m, newest << 1, mode);                      // l.30-33 (Q35)
+            reconverge();
 #pragma unroll
             for (int k = 0; k < N; ++k)
-                if (need[k]) {
-                    check_version(m, hi(pv[k]), mode);
-                    insert_lock((a[k] << 2) | 1u);
-                }
+                if (need[k]) insert_lock((a[k] << 2) | 1u);          // l.34
         } else {
             uint32_t newest = 0;
 #pragma unroll
@@ -166,8 +187,10 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
                     append_read(a[k], v[k]);
                     newest = max(newest, hi(pv[k]) >> 1);
                 }
+            reconverge();
             // one merged timestamp check per batch (tx.cuh read_batch)
             check_version(m, newest << 1, mode);
+            reconverge();
 #pragma unroll 1
             for (int k = 0; k < N; ++k) {
                 uint32_t ak = 0;
@@ -323,6 +346,53 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
         return true;
     }
 
+    // Register-resident logs: the pipelined first round and the sequential
+    // sorted acquisition in ONE code path (tx.cuh get_locks_and_tbv_converged):
+    // round 0 issues entry 0 for every lane and every entry for a pipelined
+    // lane; sequential lanes then take entries 1.. one at a time, stopping at
+    // the first held lock (Q15), in lockstep with each other.
+    __device__ __forceinline__ bool get_locks_and_tbv_converged(const Meta& m, bool pipelined)
+    {
+        static_assert(kUnroll, "converged acquisition needs register-resident logs");
+        unsigned long long old[LCAP];
+        bool ok = true;
+        uint32_t set = 0;   // entries this attempt locked
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (k == 0 || pipelined)) old[k] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);  // l.45
+        prim::fence_acquire();
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl && (k == 0 || pipelined)) {
+                if (hi(old[k]) & 1u) ok = false;                     // l.46
+                else set |= 1u << k;
+            }
+#pragma unroll
+        for (int k = 1; k < LCAP; ++k)
+            if (!pipelined && ok && k < nl) {                        // sequential: next entry only after the last succeeded
+                old[k] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);
+                prim::fence_acquire();
+                if (hi(old[k]) & 1u) ok = false;
+                else set |= 1u << k;
+            }
+        if (!ok) {
+#pragma unroll
+            for (int k = 0; k < LCAP; ++k)                           // l.47: undo what this attempt set
+                if (set & (1u << k)) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), old[k]);
+            n_acq = 0;
+            return false;
+        }
+#pragma unroll
+        for (int k = 0; k < LCAP; ++k)
+            if (k < nl) {
+                l_old[k] = hi(old[k]);
+                l_val[k] = lo(old[k]);
+                if ((l_ent[k] & 1u) && (hi(old[k]) >> 1) > snapshot) passTBV = false;  // l.49-51
+            }
+        n_acq = nl;
+        return true;
+    }
+
     // local-memory logs: kChunk atom.or.b64 at a time (tx.cuh)
     static constexpr int kChunk = 8;
     __device__ __forceinline__ bool get_locks_and_tbv_pipelined_local(const Meta& m)
@@ -359,7 +429,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
         bool got;
-        if constexpr (kUnroll) got = pipelined ? get_locks_and_tbv_pipelined(m) : get_locks_and_tbv(m);
+        if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
         else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75

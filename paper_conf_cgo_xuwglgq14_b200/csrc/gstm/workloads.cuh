@@ -87,6 +87,7 @@ __device__ __forceinline__ uint32_t lo32(uint64_t v) { return static_cast<uint32
 struct RaWL {
     static constexpr int MAXR = 8, MAXW = 8;
     static constexpr int RCAP = MAXR, WCAP = MAXW, LCAP = MAXR + MAXW, FGL_LCAP = MAXR + MAXW;
+    static constexpr bool kConvergent = true;   // one read_batch per body
 #ifndef GSTM_RA_LOCAL_LOGS
 #define GSTM_RA_LOCAL_LOGS 1    // local-memory logs: 1.6x over the 128-register unrolled logs
 #endif
@@ -178,11 +179,15 @@ struct RaIncWL {
 
 // ---- bank transfer (BASELINE configs[1]) -----------------------------------
 struct BankWL {
-    static constexpr int RCAP = 2, WCAP = 2, LCAP = 4, FGL_LCAP = 2;
+    static constexpr int RCAP = 2, WCAP = 2, LCAP = 2, FGL_LCAP = 2;   // a != b: at most 2 lock ids
+    static constexpr bool kConvergent = true;   // one read_batch per body
 #ifndef GSTM_BANK_MINB
-#define GSTM_BANK_MINB 4
+#define GSTM_BANK_MINB 2
 #endif
     static constexpr int kMinBlocks = GSTM_BANK_MINB;   // 256-thread blocks per SM (register budget)
+    // 16 resident warps per SM (2 x 256 threads): the measured optimum
+    // between latency hiding and conflicts
+    static constexpr int kWarpsPerSM = 16;
     static constexpr int DESCR = 3;
     __host__ static bool check(const WlParams& p) { return p.n_words >= 2 && p.n_words <= (1ull << 32); }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
@@ -356,6 +361,7 @@ struct EbWL {
 struct KmWL {
     static constexpr int MAXD = 16;
     static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
+    static constexpr bool kConvergent = true;   // one read_batch per body
 #ifndef GSTM_KM_LOCAL_LOGS
 #define GSTM_KM_LOCAL_LOGS 1     // local-memory logs: 122 vs 254 registers, 2.5x faster
 #endif

@@ -31,6 +31,21 @@ struct LocalLogs { static constexpr bool value = false; };
 template <class WL>
 struct LocalLogs<WL, std::void_t<decltype(WL::kLocalLogs)>> { static constexpr bool value = WL::kLocalLogs; };
 
+// WL::kConvergent (optional): every body calls read_batch exactly once, so
+// the lanes that start bodies together may reconverge inside it (Tx::reconverge)
+template <class WL, class = void>
+struct Convergent { static constexpr bool value = false; };
+template <class WL>
+struct Convergent<WL, std::void_t<decltype(WL::kConvergent)>> { static constexpr bool value = WL::kConvergent; };
+
+// WL::kWarpsPerSM (optional): resident STM warps per SM the persistent grid
+// stops at (0 = as many as fit).  More concurrent transactions than that
+// only add conflicts.
+template <class WL, class = void>
+struct WarpsPerSM { static constexpr int value = 0; };
+template <class WL>
+struct WarpsPerSM<WL, std::void_t<decltype(WL::kWarpsPerSM)>> { static constexpr int value = WL::kWarpsPerSM; };
+
 __device__ __forceinline__ unsigned long long globaltimer()
 {
     unsigned long long t;
@@ -197,7 +212,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     // ran and it waits for its locks (a lost lock round is retried in the
     // warp's next iteration, after the winners committed)
     int stage = 0;
-    bool timed_out = false, have_snap = false, lock_aborted = false;
+    bool timed_out = false, have_snap = false;
+    uint32_t lock_aborts = 0;   // lock aborts of the current transaction
     PHASE_DECL();
 
     while (__any_sync(FULL, t < p.T)) {
@@ -210,11 +226,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         PHASE_MARK(PH_BEGIN);
         const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
         bool done = false, skip = false;
+        const unsigned body_mask = Convergent<WL>::value ? __ballot_sync(FULL, act && stage == 0) : 0u;
         if (act && stage == 0) {
             cnt.inc(S_ATTEMPTS);
             result = 0;
             const uint64_t x = gen::tx_key(p.seed, t, i);
             tx.begin(snap);                                           // TXBegin l.2-3
+            tx.sync_mask = body_mask;
             StmCtx<TX> ctx{tx, m, MODE};
             WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
             if (!tx.opaque) {
@@ -232,7 +250,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 // STM-HV-Backoff: an execution that follows a lock abort goes
                 // straight to the sequential step -- its parallel attempt
                 // already failed
-                tries = (POL == POL_BACKOFF && lock_aborted) ? 1u : 0u;
+                tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
             }
         }
         PHASE_MARK(PH_BODY);
@@ -245,10 +263,14 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         bool got = false;
         // (POL_BACKOFF: only the first, parallel attempt happens here)
         if (act && stage == 1 && (POL != POL_BACKOFF || tries == 0)) {
-            // the pipelined round (§6.4) only for the first round of an
-            // execution that never lost its locks before: every retry uses the
-            // sequential sorted acquisition
-            const bool pipelined = p.lock_pipeline && tries == 0 && !lock_aborted;
+            // the pipelined round (§6.4) only for the first round of the first
+            // p.lock_pipeline executions of a transaction: every later round
+            // and execution uses the sequential sorted acquisition.  A lane
+            // starts a new transaction only after committing its current one,
+            // so if nothing commits every lane turns sequential within
+            // p.lock_pipeline lock aborts, and the sorted argument
+            // gives progress: livelock freedom is kept for any finite count.
+            const bool pipelined = tries == 0 && lock_aborts < p.lock_pipeline;
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
             if (r == C_OK) {
                 got = true;
@@ -259,7 +281,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     tries = 1;                                        // -> the sequential step below
                 } else if (p.k_lock && ++tries >= p.k_lock) {
                     stage = 0;
-                    lock_aborted = true;
+                    ++lock_aborts;
                     cnt.inc(S_AB_LOCK);
                 }
             } else {
@@ -322,7 +344,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                         seq_failed = true;
                         if (p.k_lock && ++tries > p.k_lock) {
                             stage = 0;
-                            lock_aborted = true;
+                            ++lock_aborts;
                             cnt.inc(S_AB_LOCK);
                         }
                     } else {
@@ -341,7 +363,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             stage = 0;
             ++i;
             backoff = 0;
-            lock_aborted = false;
+            lock_aborts = 0;
         } else if (p.backoff_ns && act && stage == 0) {
             // exponential backoff after an abort (P:111 argues per-lane
             // delays cannot work under SIMT; lanes here sleep independently
@@ -602,7 +624,7 @@ __global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
 // host launch templates (instantiated per workload in wl_*.cu)
 // ---------------------------------------------------------------------------
 template <class K>
-inline uint64_t resident_blocks(K kernel, int block)
+inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0)
 {
     static int sms = 0;
     if (!sms) {
@@ -612,14 +634,15 @@ inline uint64_t resident_blocks(K kernel, int block)
     }
     int per_sm = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, 0) != cudaSuccess || per_sm < 1) per_sm = 1;
+    if (warps_per_sm > 0) per_sm = std::max(1, std::min(per_sm, warps_per_sm * 32 / block));
     return static_cast<uint64_t>(per_sm) * (sms > 0 ? sms : 148);
 }
 
 template <class K>
-inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s)
+inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s, int warps_per_sm = 0)
 {
     uint64_t grid = (kp.T + block - 1) / block;
-    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block));
+    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block, kp.max_threads ? 0 : warps_per_sm));
     if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
     if (grid == 0) return cudaSuccess;
     kernel<<<static_cast<unsigned>(grid), block, 0, s>>>(kp);
@@ -635,17 +658,17 @@ cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
     const dim3 g(static_cast<unsigned>(grid)), b(block);
     switch (kmode) {
     case KMODE_HV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s, WarpsPerSM<WL>::value)
+                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s, WarpsPerSM<WL>::value);
     case KMODE_TBV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s, WarpsPerSM<WL>::value)
+                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s, WarpsPerSM<WL>::value);
     case KMODE_HV_BACKOFF:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_BACKOFF>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_BACKOFF>, kp, block, s);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_BACKOFF>, kp, block, s, WarpsPerSM<WL>::value)
+                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_BACKOFF>, kp, block, s, WarpsPerSM<WL>::value);
     case KMODE_HV_UNSORTED:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_UNSORTED>, kp, block, s)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_UNSORTED>, kp, block, s);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_UNSORTED>, kp, block, s, WarpsPerSM<WL>::value)
+                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_UNSORTED>, kp, block, s, WarpsPerSM<WL>::value);
     case KMODE_VBV: vbv_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
