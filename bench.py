@@ -58,6 +58,8 @@ def parse(argv=None):
     ap.add_argument("--prelock", type=int, default=None,
                     help="pre-lock VBV (A3.l71); default 0 on the paired layout, 1 on the split one")
     ap.add_argument("--k-lock", type=int, default=1, help="lock rounds before a transaction re-executes")
+    ap.add_argument("--spin-cap", type=int, default=1,
+                    help="re-reads of a locked word before the transaction re-executes")
     ap.add_argument("--threads", type=int, default=THREADS)
     ap.add_argument("--tx-per-thread", type=int, default=TX_PER_THREAD)
     ap.add_argument("--no-cgl", action="store_true", help="skip the CGL/FGL baselines and the variant table")
@@ -132,7 +134,10 @@ def headline_variant(args) -> Variant:
     # k_lock = 1: a transaction that loses a lock round re-executes with fresh
     # reads instead of retrying the commit with stale ones (P:325 leaves the
     # number of attempts open; DESIGN.md §7.3 ablation)
-    return Variant(args.mode, args.layout, args.prelock, k_lock=args.k_lock)
+    # spin_cap = 1: a transaction that finds a word still locked after one
+    # re-read re-executes in its warp's next iteration instead of holding its
+    # warp up
+    return Variant(args.mode, args.layout, args.prelock, k_lock=args.k_lock, spin_cap=args.spin_cap)
 
 
 def config(args, label="hv/paired"):

@@ -86,7 +86,12 @@ static gstm_params_t default_params(int workload)
     p.timeout_ms = 60000;
     p.snapshot_reuse = 1;
     p.lock_pipeline = 1;
-    if (workload == GSTM_WL_BANK) p.n_words = 1ull << 20;
+    if (workload == GSTM_WL_BANK) {
+        p.n_words = 1ull << 20;
+        // a transaction pipelines the first lock round of its first 4
+        // executions (9.21 vs 8.83 G tx/s with 1)
+        p.lock_pipeline = 4;
+    }
     if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
     // RA and EB (random words, contended): the sequential first round is
     // faster even when the lock log fits one pipelined chunk (EB A=8: 1.24

@@ -367,6 +367,9 @@ struct KmWL {
 #endif
     static constexpr bool kLocalLogs = GSTM_KM_LOCAL_LOGS;
     static constexpr int kMinBlocks = GSTM_KM_LOCAL_LOGS ? 2 : 1;
+    // 1024 records: 8 resident warps per SM is the measured optimum
+    // (21.5 vs 17.9 M tx/s at 16)
+    static constexpr int kWarpsPerSM = 8;
     static constexpr int DESCR = MAXD + 1;
     __host__ static bool check(const WlParams& p)
     {
