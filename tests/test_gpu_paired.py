@@ -98,6 +98,33 @@ def test_paired_bank_config1_full_replay(mode):
     assert ((locks >> 1).astype(np.int64) == want).all()
 
 
+def test_paired_bank_headline_variant_full_replay():
+    """The exact configuration bench.py times (BASELINE configs[1] at full
+    size): STM-HV, paired layout, no pre-lock VBV, k_lock = 1, spin_cap = 1,
+    the bank defaults (first lock round pipelined for 4 executions, 16
+    resident warps per SM); two launches on one handle (the second starts a
+    new clock epoch on the first one's heap)."""
+    T, K = 1 << 20, 16
+    g, gp, op, init = U.make("bank", T, K, 20, mode="hv", paired=True, n_words=1 << 20, prelock_vbv=0, k_lock=1,
+                             spin_cap=1)
+    assert gp.lock_pipeline == 4 and gp.max_threads == 0
+    for seed in (1, 2):
+        st, heap, stamps, res = U.run_verified(g, "bank", op, init, T, K, seed)
+        assert int(heap.astype(np.int64).sum()) == 1000 * (1 << 20)
+        assert (heap.view(np.int32) >= 0).all()
+        locks = g.read_locks()
+        assert not (locks & 1).any()
+        upd = np.nonzero((stamps & O.RO_FLAG) == 0)[0]
+        d = g.dump_descr("bank", T, K, seed)[upd]
+        s_abs = stamps[upd].astype(np.int64) + st.clock_begin
+        want = np.zeros(1 << 20, dtype=np.int64)
+        np.maximum.at(want, d[:, 0].astype(np.int64), s_abs)
+        np.maximum.at(want, d[:, 1].astype(np.int64), s_abs)
+        touched = want > 0
+        assert ((locks >> 1).astype(np.int64)[touched] == want[touched]).all()
+        init = heap
+
+
 @pytest.mark.parametrize("mode", ["hv", "tbv", "fgl", "cgl"])
 @pytest.mark.parametrize("wl,kw,T,K,words,bits", [
     ("bank", dict(n_words=4), 2, 4, 4, 2),
@@ -136,11 +163,13 @@ def test_paired_ht_km_eb(mode):
 
 
 @pytest.mark.parametrize("mode", ["hv", "tbv", "fgl"])
-@pytest.mark.parametrize("pipeline", [0, 1])
-def test_paired_livelock_two_words(mode, pipeline):
+@pytest.mark.parametrize("pipeline,spin_cap", [(0, 0), (1, 0), (4, 1), (1000, 1)])
+def test_paired_livelock_two_words(mode, pipeline, spin_cap):
+    # lock_pipeline = N: a transaction pipelines the first lock round of its
+    # first N executions; progress must hold for any finite N (stm_kernels.cuh)
     T, K = 512, 8
     g, gp, op, init = U.make("ra", T, K, 1, mode=mode, paired=True, n_reads=2, n_writes=2, n_words=2,
-                             lock_pipeline=pipeline, k_lock=1)
+                             lock_pipeline=pipeline, k_lock=1, spin_cap=spin_cap)
     st, *_ = U.run_verified(g, "ra", op, init, T, K, 4)
     assert st.commits == T * K
 

@@ -294,14 +294,15 @@ def test_concurrency_cap_replay(mode, wl, kw, T, K, cap):
 
 
 @pytest.mark.parametrize("mode", ["hv", "tbv"])
-def test_k_lock_one_with_pipeline_progresses(mode):
-    """k_lock = 1 aborts on the first lost lock round; after such an abort a
-    transaction never uses the pipelined round again, so high contention
-    (RA configs[0]) still finishes (regression: pipelined-only retries
-    livelocked)."""
+@pytest.mark.parametrize("pipeline", [1, 4, 64])
+def test_k_lock_one_with_pipeline_progresses(mode, pipeline):
+    """k_lock = 1 aborts on the first lost lock round; after `pipeline` such
+    aborts a transaction never uses the pipelined round again, so high
+    contention (RA configs[0]) still finishes (regression: pipelined-only
+    retries livelocked)."""
     T, K = 256, 64
     g, gp, op, init = U.make("ra", T, K, 10, mode=mode, n_reads=4, n_writes=4, n_words=1024, k_lock=1,
-                             lock_pipeline=1, timeout_ms=20000)
+                             lock_pipeline=pipeline, timeout_ms=20000)
     st, *_ = U.run_verified(g, "ra", op, init, T, K, 3)
     assert st.aborts_lock > 0
 
