@@ -229,9 +229,17 @@ struct Tx {
                         again = true;                                // l.19 goto loop
                     }
             } else {
-                for (int k = 0; k < nr; ++k) {
-                    const uint32_t vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(r_addr[k])));
-                    if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                for (int k0 = 0; k0 < nr; k0 += 8) {                 // 8 lock loads in flight
+                    uint32_t vl[8];
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        if (k0 + j < nr) vl[j] = prim::ld_relaxed(m.lock_ptr(m.lock_of(r_addr[k0 + j])));
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        if (k0 + j < nr && ((vl[j] & 1u) || (vl[j] >> 1) > snapshot)) {
+                            newsnap = max(newsnap, vl[j] >> 1);
+                            again = true;
+                        }
                 }
             }
             snapshot = newsnap;

@@ -78,11 +78,18 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
                         if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
                     }
             } else {
-                for (int k = 0; k < nr; ++k) {
-                    const unsigned long long pv = prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]));
-                    ok &= (lo(pv) == r_val[k]);
-                    const uint32_t vl = hi(pv);
-                    if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                for (int k0 = 0; k0 < nr; k0 += 8) {                 // 8 pair loads in flight
+                    unsigned long long pv[8];
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        if (k0 + j < nr) pv[j] = prim::ld_relaxed_u64(m.pair_ptr(r_addr[k0 + j]));
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        if (k0 + j < nr) {
+                            ok &= (lo(pv[j]) == r_val[k0 + j]);
+                            const uint32_t vl = hi(pv[j]);
+                            if ((vl & 1u) || (vl >> 1) > snapshot) { newsnap = max(newsnap, vl >> 1); again = true; }
+                        }
                 }
             }
             if (!ok) return false;                                   // l.11
@@ -244,7 +251,15 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
             for (int k = 0; k < RCAP; ++k)
                 if (k < nr) ok &= (lo(pv[k]) == r_val[k]);
         } else {
-            for (int k = 0; k < nr; ++k) ok &= (lo(prim::ld_relaxed_u64(m.pair_ptr(r_addr[k]))) == r_val[k]);
+            for (int k0 = 0; k0 < nr; k0 += 8) {                     // 8 pair loads in flight
+                uint32_t cur[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    if (k0 + j < nr) cur[j] = lo(prim::ld_relaxed_u64(m.pair_ptr(r_addr[k0 + j])));
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    if (k0 + j < nr) ok &= (cur[j] == r_val[k0 + j]);
+            }
         }
         return ok;
     }
