@@ -105,7 +105,9 @@ typedef struct {
                              /*    logs pipeline only logs of <= 8 locks.              */
                              /*    Default 1 (RA, EB: 0)                               */
     uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
-                             /*    n_threads STM threads (grid-stride); 0 = no cap     */
+                             /*    n_threads STM threads; 0 = the workload's default:  */
+                             /*    what fits on the chip, at most 16 resident warps   */
+                             /*    per SM for bank and 8 for k-means */
     uint32_t lock_shift;     /* stripe size 2^lock_shift words per version lock      */
                              /*    (lock = (word >> shift) mod 2^bits); default 0     */
     uint32_t shard_bits;     /* HT key partition: G = 2^shard_bits     */

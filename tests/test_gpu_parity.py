@@ -293,6 +293,21 @@ def test_concurrency_cap_replay(mode, wl, kw, T, K, cap):
     assert st.commits + st.commits_ro == T * K
 
 
+@pytest.mark.parametrize("paired", [False, True])
+@pytest.mark.parametrize("T", [1023, 1024, 1025, 2047, 2053, 5 * 1024 + 37, 9 * 1024])
+def test_static_region_and_counter_boundaries(paired, T):
+    """The persistent grid runs STM threads g, g+P, ... of a static region
+    [0, Rs*P), Rs = max(1, T/P - 1), then threads from a shared counter
+    (stm_kernels.cuh): thread counts around multiples of P = 1024 lanes
+    must run every transaction of every STM thread exactly once, in order."""
+    K = 3
+    g, gp, op, init = U.make("bank", T, K, 12, mode="hv", paired=paired, n_words=1 << 12, max_threads=1024,
+                             block_threads=128, k_lock=1, spin_cap=1)
+    st, heap, *_ = U.run_verified(g, "bank", op, init, T, K, 17)
+    assert st.commits + st.commits_ro == T * K
+    assert int(heap.astype(np.int64).sum()) == 1000 << 12
+
+
 @pytest.mark.parametrize("mode", ["hv", "tbv"])
 @pytest.mark.parametrize("pipeline", [1, 4, 64])
 def test_k_lock_one_with_pipeline_progresses(mode, pipeline):
