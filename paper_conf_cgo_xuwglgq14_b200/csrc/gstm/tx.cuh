@@ -325,7 +325,13 @@ struct Tx {
         prim::fence_acquire();                                       // l.26
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (need[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
+            if (need[k]) {
+                // consecutive words of one stripe (a k-means record under one
+                // lock) share one lock-word load: it is issued after every
+                // value load of the batch, which is all l.26-28 asks
+                if (N > 4 && k > 0 && need[k - 1] && m.lock_of(a[k]) == m.lock_of(a[k - 1])) vl[k] = vl[k - 1];
+                else vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
+            }
         if constexpr (N <= 4) {
             // small batches (bank: 2), fully unrolled: ONE spin loop re-reads
             // every still-locked lock word of the batch together (l.27-29)

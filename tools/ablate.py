@@ -23,9 +23,11 @@ SHAPES = {
     "ra_paper": dict(words=1 << 23, bits=20, T=65536, K=16, params=dict(n_reads=4, n_writes=4, n_words=1 << 23)),
     "ht": dict(words=(1 << 20) + 2 * (1 << 24), bits=22, T=1 << 22, K=4, params=dict()),
     "km": dict(words=1024 * 17, bits=20, T=1 << 24, K=1, params=dict()),
+    # one version lock per 32-word-aligned k-means record
+    "km_rec": dict(words=1024 * 32, bits=20, T=1 << 24, K=1, params=dict(km_stride=32, lock_shift=5)),
     "eb": dict(words=1 << 26, bits=22, T=1 << 18, K=16, params=dict(n_words=1 << 26, n_accesses=16)),
 }
-WL_OF = {"bank": "bank", "ra": "ra", "ra_paper": "ra", "ht": "ht", "km": "km", "eb": "eb"}
+WL_OF = {"bank": "bank", "ra": "ra", "ra_paper": "ra", "ht": "ht", "km": "km", "km_rec": "km", "eb": "eb"}
 
 
 def parse_variant(s: str) -> dict:
