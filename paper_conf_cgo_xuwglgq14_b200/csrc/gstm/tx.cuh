@@ -644,6 +644,26 @@ struct Tx {
         prim::fence_release();                                       // l.82
     }
 
+    // The same write-back for a write-set made of runs of consecutive words
+    // (a k-means record, WL::kRunWriteback): a run of 4 words starting on a
+    // 16-byte boundary goes out as one vector store.  Split layout only.
+    __device__ __forceinline__ void writeback_runs(const Meta& m)
+    {
+        for (int k = 0; k < nw;) {
+            const uint32_t w = w_addr[k];
+            uint32_t* ptr = m.val_ptr(w);
+            if (m.vshift == 0 && k + 3 < nw && (reinterpret_cast<uintptr_t>(ptr) & 15u) == 0 &&
+                w_addr[k + 1] == w + 1 && w_addr[k + 2] == w + 2 && w_addr[k + 3] == w + 3) {
+                prim::st_relaxed_v4(ptr, w_val[k], w_val[k + 1], w_val[k + 2], w_val[k + 3]);
+                k += 4;
+            } else {
+                prim::st_relaxed(ptr, w_val[k]);
+                ++k;
+            }
+        }
+        prim::fence_release();                                       // l.82
+    }
+
     // ---- A3.l56-61 ReleaseAndUpdateLocks(version) -------------------------
     // Written locks get version<<1; read-only locks get back the exact word
     // the acquiring atomic returned (reading Q16: == lock - 1).

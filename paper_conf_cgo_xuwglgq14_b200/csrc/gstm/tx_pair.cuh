@@ -457,6 +457,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
     // l.79-82: nothing to do here -- each written value is published
     // together with its unlock in release_and_update
     __device__ __forceinline__ void writeback(const Meta&) {}
+    __device__ __forceinline__ void writeback_runs(const Meta&) {}
 
     // ---- A3.l80-84: written pairs get (new value, stamp<<1); read-only
     //      pairs get back exactly what the atomic returned --------------------

@@ -362,6 +362,7 @@ struct KmWL {
     static constexpr int MAXD = 16;
     static constexpr int RCAP = MAXD + 1, WCAP = MAXD + 1, LCAP = MAXD + 1, FGL_LCAP = 1;
     static constexpr bool kConvergent = true;   // one read_batch per body
+    static constexpr bool kRunWriteback = true;   // the record's words, in order
 #ifndef GSTM_KM_LOCAL_LOGS
 #define GSTM_KM_LOCAL_LOGS 1     // local-memory logs: 122 vs 254 registers, 2.5x faster
 #endif

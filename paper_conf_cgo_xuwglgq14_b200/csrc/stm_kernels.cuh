@@ -38,6 +38,13 @@ struct Convergent { static constexpr bool value = false; };
 template <class WL>
 struct Convergent<WL, std::void_t<decltype(WL::kConvergent)>> { static constexpr bool value = WL::kConvergent; };
 
+// WL::kRunWriteback (optional): the write-set is runs of consecutive words
+// (a record): write back with 16-byte vector stores (Tx::writeback_runs)
+template <class WL, class = void>
+struct RunWriteback { static constexpr bool value = false; };
+template <class WL>
+struct RunWriteback<WL, std::void_t<decltype(WL::kRunWriteback)>> { static constexpr bool value = WL::kRunWriteback; };
+
 // WL::kWarpsPerSM (optional): resident STM warps per SM the persistent grid
 // stops at (0 = as many as fit).  More concurrent transactions than that
 // only add conflicts.
@@ -280,7 +287,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
             if (r == C_OK) {
                 got = true;
-                tx.writeback(m);                                      // l.79-82
+                if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m); else tx.writeback(m);                                      // l.79-82
             } else if (r == C_LOCK) {
                 cnt.inc(S_LOCK_RETRIES);                              // l.73-74: retry next iteration
                 if (POL == POL_BACKOFF) {
@@ -336,7 +343,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 if (static_cast<int>(prim::lane_id()) == L) {
                     const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, false);
                     if (r == C_OK) {
-                        tx.writeback(m);                              // l.79-82
+                        if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m); else tx.writeback(m);                              // l.79-82
                         sl = static_cast<uint32_t>(clock_fetch_add(m.clock, 1u)) + 1u;   // l.83
                         tx.release_and_update(m, sl);                 // l.84
                         if (p.tx_stamp) {
