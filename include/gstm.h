@@ -123,6 +123,13 @@ typedef struct {
                              /*    km_clusters x km_dims uint32 table stored after   */
                              /*    the records; gstm_launch runs the assignment pass */
                              /*    before the update transactions.  Table <= 64 KiB  */
+    uint32_t l2_persist_locks; /* 1: the launch marks the version-lock table (split   */
+                             /*    layout) as persisting in L2 (an access-policy      */
+                             /*    window on the handle's stream, cleared after the   */
+                             /*    launch; the L2 set-aside stays reserved while the  */
+                             /*    knob is on), so random heap lines streaming from   */
+                             /*    HBM do not evict the locks (EB with a hot set      */
+                             /*    larger than L2).  Default 0 (EB: 1)                */
 } gstm_params_t;
 
 typedef struct {

@@ -1,4 +1,5 @@
 // api.cu -- the C ABI (include/gstm.h) over the kernels in kernels.cu.
+#include <algorithm>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -63,6 +64,38 @@ struct gstm_handle {
     uint64_t clock_bound = 0;    // upper bound of g_clock (host-tracked)
 };
 
+// L2 persistence for the version-lock table (params.l2_persist_locks): an
+// access-policy window on the handle's stream covering the lock table,
+// hit property persisting, set around the transaction kernel's launch.
+static cudaError_t set_l2_lock_window(gstm_t* h, bool on)
+{
+    static size_t max_persist = 0, max_window = 0;
+    if (!max_window) {
+        int dev = 0;
+        cudaDeviceProp pr;
+        cudaError_t e = cudaGetDevice(&dev);
+        if (e == cudaSuccess) e = cudaGetDeviceProperties(&pr, dev);
+        if (e != cudaSuccess) return e;
+        max_persist = pr.persistingL2CacheMaxSize;
+        max_window = pr.accessPolicyMaxWindowSize;
+        if (!max_window) return cudaErrorNotSupported;
+    }
+    cudaStreamAttrValue a;
+    memset(&a, 0, sizeof(a));
+    if (on) {
+        const size_t bytes = std::min(sizeof(uint32_t) << h->bits, max_window);
+        const size_t lim = std::min(bytes, max_persist);
+        cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+        if (e != cudaSuccess) return e;
+        a.accessPolicyWindow.base_ptr = h->locks;
+        a.accessPolicyWindow.num_bytes = bytes;
+        a.accessPolicyWindow.hitRatio = bytes ? std::min(1.0f, static_cast<float>(lim) / static_cast<float>(bytes)) : 0.f;
+        a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    }
+    return cudaStreamSetAttribute(h->stream, cudaStreamAttributeAccessPolicyWindow, &a);
+}
+
 static gstm_params_t default_params(int workload)
 {
     gstm_params_t p;
@@ -92,7 +125,12 @@ static gstm_params_t default_params(int workload)
         // executions (9.21 vs 8.83 G tx/s with 1)
         p.lock_pipeline = 4;
     }
-    if (workload == GSTM_WL_EB) p.n_words = 1ull << 20;
+    if (workload == GSTM_WL_EB) {
+        p.n_words = 1ull << 20;
+        // the hot set may exceed L2: keep the lock table there (DESIGN.md §6.10:
+        // hot set 2^26, A=16: 336 -> 369 M tx/s with 2^22 locks, 391 -> 453 with 2^24)
+        p.l2_persist_locks = 1;
+    }
     // RA and EB (random words, contended): the sequential first round is
     // faster even when the lock log fits one pipelined chunk (EB A=8: 1.24
     // vs 0.94 G tx/s; RA 8M words: 0.76 vs 0.53 G tx/s)
@@ -548,7 +586,10 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
         CUDA_TRY(launch_km_assign(kp, h->km_cluster, h->stream));
         kp.w.km_cluster = h->km_cluster;
     }
+    const bool persist = P.l2_persist_locks && !h->paired && h->locks;
+    if (persist) CUDA_TRY(set_l2_lock_window(h, true));
     CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
+    if (persist) CUDA_TRY(set_l2_lock_window(h, false));
     CUDA_TRY(launch_finish(h->meta, h->clock, h->stream));
     CUDA_TRY(cudaEventRecord(h->ev1, h->stream));
     h->clock_bound += n_tx;

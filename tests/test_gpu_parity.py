@@ -293,6 +293,21 @@ def test_concurrency_cap_replay(mode, wl, kw, T, K, cap):
     assert st.commits + st.commits_ro == T * K
 
 
+@pytest.mark.parametrize("mode", ["hv", "tbv", "fgl"])
+@pytest.mark.parametrize("persist", [0, 1])
+def test_l2_persisting_lock_table_replay(mode, persist):
+    """l2_persist_locks (an L2 access-policy window over the lock table around
+    the launch) changes placement only: EB with a hot set of 2^22 words stays
+    serializable, and the window does not leak to later launches."""
+    T, K, H = 1 << 15, 4, 1 << 22
+    g, gp, op, init = U.make("eb", T, K, 20, mode=mode, n_words=H, n_accesses=16, heap_words=H,
+                             l2_persist_locks=persist)
+    assert gp.l2_persist_locks == persist
+    st, heap, *_ = U.run_verified(g, "eb", op, init, T, K, 29)
+    g.set_params(gp)
+    U.run_verified(g, "eb", op, heap, T, K, 30)
+
+
 @pytest.mark.parametrize("paired", [False, True])
 @pytest.mark.parametrize("T", [1023, 1024, 1025, 2047, 2053, 5 * 1024 + 37, 9 * 1024])
 def test_static_region_and_counter_boundaries(paired, T):
