@@ -92,7 +92,9 @@ typedef struct {
     uint32_t backoff_ns;     /* warp-uniform backoff after an abort; 0 = none           */
     uint32_t verify;         /* record per-tx stamp and result (gstm_read_tx_log)       */
     uint32_t block_threads;  /* CUDA block size (multiple of 32, <= 256), default 256   */
-    uint32_t spin_cap;       /* bound on lock spins / PostValidation restarts          */
+    uint32_t spin_cap;       /* bound on lock spins / PostValidation restarts; past it */
+                             /*    the transaction re-executes (Q25, Q38).  0 = 65536; */
+                             /*    default 65536 (bank, RA: 1)                         */
     uint32_t timeout_ms;     /* device watchdog per launch, default 60000               */
     uint32_t snapshot_reuse; /* 1: a warp that just committed starts its next txs at   */
                              /*    the clock value after its own commits instead of   */
