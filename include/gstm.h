@@ -132,6 +132,10 @@ typedef struct {
                              /*    knob is on), so random heap lines streaming from   */
                              /*    HBM do not evict the locks (EB with a hot set      */
                              /*    larger than L2).  Default 0 (EB: 1)                */
+    uint32_t ra_partition;   /* RA: k > 0 = STM thread t addresses only its own words */
+                             /*    [t*k, t*k + k) (disjoint access sets: a unique,    */
+                             /*    conflict-free result); needs        */
+                             /*    n_threads * k <= n_words.  Default 0               */
 } gstm_params_t;
 
 typedef struct {

@@ -62,6 +62,7 @@ class Params(C.Structure):
         ("shard", C.c_uint32),
         ("km_stride", C.c_uint32),
         ("km_assign", C.c_uint32),
+        ("ra_partition", C.c_uint32),
     ]
 
 

@@ -77,16 +77,23 @@ int or_descr(const or_params_t* p, uint64_t seed, uint64_t t, uint64_t i,
     switch (p->workload) {
     case OR_WL_RA: {
         uint32_t R = p->n_reads, W = p->n_writes;
-        uint64_t N = p->n_words;
+        uint64_t N = p->n_words, base = 0;
         if (N == 0) return -1;
+        if (p->ra_partition) {
+            /* disjoint access sets: thread t draws its words
+             * from its own range [t*k, t*k + k) */
+            base = t * (uint64_t)p->ra_partition;
+            if (base + p->ra_partition > N) return -1;
+            N = p->ra_partition;
+        }
         if (p->ra_kind == 1) {
             if ((int)R > cap) return -1;
-            for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)or_bounded(or_draw(x, j), N);
+            for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)(base + or_bounded(or_draw(x, j), N));
             return (int)R;
         }
         if ((int)(R + 2 * W) > cap) return -1;
-        for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)or_bounded(or_draw(x, j), N);
-        for (uint32_t j = 0; j < W; ++j) out[R + j] = (uint32_t)or_bounded(or_draw(x, R + j), N);
+        for (uint32_t j = 0; j < R; ++j) out[j] = (uint32_t)(base + or_bounded(or_draw(x, j), N));
+        for (uint32_t j = 0; j < W; ++j) out[R + j] = (uint32_t)(base + or_bounded(or_draw(x, R + j), N));
         for (uint32_t j = 0; j < W; ++j) out[R + W + j] = lo32(or_draw(x, R + W + j));
         return (int)(R + 2 * W);
     }

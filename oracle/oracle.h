@@ -56,6 +56,9 @@ typedef struct {
     uint32_t km_stride;     /* KM: words per record, >= km_dims+1 (0: km_dims+1) */
     uint32_t km_assign;     /* KM: 1 = cluster = nearest centroid of the table   */
                             /*     after the records (a full Lloyd iteration)    */
+    uint32_t ra_partition;  /* RA: k > 0 = thread t addresses only its own words */
+                            /*     [t*k, t*k + k) (SURVEY §8c-O4 disjoint access */
+                            /*     sets: a unique, conflict-free result); 0 = off */
 } or_params_t;
 
 /* ---------------- gen.c: the seeded input generator ---------------------- */

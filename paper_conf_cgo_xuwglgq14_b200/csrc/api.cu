@@ -165,6 +165,7 @@ static WlParams wl_params(const gstm_params_t& p, uint64_t T, uint64_t K)
     w.km_cluster = nullptr;
     w.shard_bits = p.shard_bits;
     w.shard = p.shard;
+    w.ra_partition = p.ra_partition;
     w.T = T;
     w.K = K;
     return w;

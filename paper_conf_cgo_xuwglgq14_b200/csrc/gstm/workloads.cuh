@@ -27,6 +27,7 @@ struct WlParams {
     uint32_t km_assign;                         // KM: cluster = nearest centroid (full iteration)
     const uint32_t* km_cluster;                 // KM, km_assign: per-tx cluster from km_assign_kernel
     uint32_t shard_bits, shard;                 // HT key partition
+    uint32_t ra_partition;                      // RA: k > 0 = thread t uses only [t*k, t*k + k)
     uint64_t T, K;           // launch shape (HT node layout needs M = T*K)
 };
 
@@ -82,6 +83,19 @@ struct DirectCtx {
 
 __device__ __forceinline__ uint32_t lo32(uint64_t v) { return static_cast<uint32_t>(v); }
 
+// RA word of draw r for STM thread t: uniform over [0, n_words), or over the
+// thread's own range [t*k, t*k + k) with ra_partition = k (disjoint access
+// sets)
+__device__ __forceinline__ uint32_t ra_word(const WlParams& p, uint64_t r, uint64_t t)
+{
+    if (p.ra_partition) return static_cast<uint32_t>(t * p.ra_partition + gen::bounded(r, p.ra_partition));
+    return static_cast<uint32_t>(gen::bounded(r, p.n_words));
+}
+__host__ __forceinline__ bool ra_partition_fits(const WlParams& p)
+{
+    return !p.ra_partition || p.T * p.ra_partition <= p.n_words;
+}
+
 // ---- RA kind 0: R reads then W writes (Figure 1 random array) -------------
 // acc = sum of the words read; write w_j <- acc + c_j; result = acc.
 struct RaWL {
@@ -99,17 +113,17 @@ struct RaWL {
     static constexpr int DESCR = MAXR + 2 * MAXW;
     __host__ static bool check(const WlParams& p)
     {
-        return p.ra_kind == 0 && p.n_reads <= MAXR && p.n_writes <= MAXW && p.n_words > 0;
+        return p.ra_kind == 0 && p.n_reads <= MAXR && p.n_writes <= MAXW && p.n_words > 0 && ra_partition_fits(p);
     }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
     template <class Ctx>
-    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t t, uint64_t, uint32_t& result)
     {
         const int R = static_cast<int>(p.n_reads), W = static_cast<int>(p.n_writes);
         uint32_t a[MAXR], v[MAXR];
 #pragma unroll
         for (int j = 0; j < MAXR; ++j)
-            a[j] = j < R ? static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)) : 0u;
+            a[j] = j < R ? ra_word(p, gen::draw(x, j), t) : 0u;
         c.template read_batch<MAXR>(a, v, R);
         if (!c.ok()) return;
         uint32_t acc = 0;
@@ -121,21 +135,21 @@ struct RaWL {
         // the instruction cache
 #pragma unroll 1
         for (int j = 0; j < W; ++j) {
-            const uint32_t w = static_cast<uint32_t>(gen::bounded(gen::draw(x, R + j), p.n_words));
+            const uint32_t w = ra_word(p, gen::draw(x, R + j), t);
             c.write(w, acc + lo32(gen::draw(x, R + W + j)));
         }
         result = acc;
     }
     template <class F>
-    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t t, uint64_t, F&& f)
     {
         const uint32_t R = p.n_reads, W = p.n_writes;
-        for (uint32_t j = 0; j < R + W; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
+        for (uint32_t j = 0; j < R + W; ++j) f(ra_word(p, gen::draw(x, j), t));
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t t, uint32_t* out)
     {
         const uint32_t R = p.n_reads, W = p.n_writes;
-        for (uint32_t j = 0; j < R + W; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        for (uint32_t j = 0; j < R + W; ++j) out[j] = ra_word(p, gen::draw(x, j), t);
         for (uint32_t j = 0; j < W; ++j) out[R + W + j] = lo32(gen::draw(x, R + W + j));
         return static_cast<int>(R + 2 * W);
     }
@@ -150,14 +164,17 @@ struct RaIncWL {
     static constexpr bool kLocalLogs = GSTM_RA_LOCAL_LOGS;
     static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = MAXR;
-    __host__ static bool check(const WlParams& p) { return p.ra_kind == 1 && p.n_reads <= MAXR && p.n_words > 0; }
+    __host__ static bool check(const WlParams& p)
+    {
+        return p.ra_kind == 1 && p.n_reads <= MAXR && p.n_words > 0 && ra_partition_fits(p);
+    }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
     template <class Ctx>
-    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t t, uint64_t, uint32_t& result)
     {
         uint32_t acc = 0;
         for (uint32_t j = 0; j < p.n_reads; ++j) {
-            const uint32_t a = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+            const uint32_t a = ra_word(p, gen::draw(x, j), t);
             const uint32_t v = c.read(a);
             if (!c.ok()) return;       // Figure 1: break when not opaque
             c.write(a, v + 1u);
@@ -166,13 +183,13 @@ struct RaIncWL {
         result = acc;
     }
     template <class F>
-    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t, uint64_t, F&& f)
+    __device__ __forceinline__ static void fgl_words(const WlParams& p, uint64_t x, uint64_t t, uint64_t, F&& f)
     {
-        for (uint32_t j = 0; j < p.n_reads; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
+        for (uint32_t j = 0; j < p.n_reads; ++j) f(ra_word(p, gen::draw(x, j), t));
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t t, uint32_t* out)
     {
-        for (uint32_t j = 0; j < p.n_reads; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
+        for (uint32_t j = 0; j < p.n_reads; ++j) out[j] = ra_word(p, gen::draw(x, j), t);
         return static_cast<int>(p.n_reads);
     }
 };
@@ -221,7 +238,7 @@ struct BankWL {
         f(a);
         f(b);
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t, uint32_t* out)
     {
         accounts(p, x, out[0], out[1], out[2]);
         return 3;
@@ -295,7 +312,7 @@ struct HtWL {
         key_of(p, x, key, ins, bucket);
         f(bucket);      // one lock per bucket: node words are private until linked, then immutable
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t, uint32_t* out)
     {
         key_of(p, x, out[0], out[1], out[2]);
         return 3;
@@ -346,7 +363,7 @@ struct EbWL {
     {
         for (uint32_t j = 0; j < p.n_accesses; ++j) f(static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words)));
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t, uint32_t* out)
     {
         const uint32_t A = p.n_accesses;
         for (uint32_t j = 0; j < A; ++j) out[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
@@ -410,7 +427,7 @@ struct KmWL {
     {
         f(cluster(p, x, t, i) * p.km_stride);   // one lock per record
     }
-    __device__ static int descr(const WlParams& p, uint64_t x, uint32_t* out)
+    __device__ static int descr(const WlParams& p, uint64_t x, uint64_t, uint32_t* out)
     {
         out[0] = static_cast<uint32_t>(gen::bounded(gen::draw(x, 0), p.km_clusters));
         for (uint32_t d = 0; d < p.km_dims; ++d) out[1 + d] = static_cast<uint32_t>(gen::draw(x, 1 + d) >> 56);

@@ -484,7 +484,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) vbv_kernel(const KParams 
     const uint64_t P = static_cast<uint64_t>(gridDim.x) * blockDim.x;
     uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
     if (p.K == 0) t = p.T;
-    const Meta m = p.m;
+    // STM-VBV waits on the global sequence lock, not on a word's version
+    // lock: the short per-word spin bound of Q38 (spin_cap 1 for bank/RA)
+    // does not apply -- it would turn every concurrent writer into an abort
+    Meta m = p.m;
+    m.spin_cap = max(m.spin_cap, 1u << 16);
     unsigned long long* seq = p.meta + M_SEQ;
     const uint32_t clock_begin = static_cast<uint32_t>(p.meta[M_CLOCK_BEGIN]);
     const unsigned long long deadline = p.meta[M_DEADLINE];
@@ -633,7 +637,7 @@ __global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
     if (t >= p.T) return;
     for (uint32_t i = 0; i < p.K; ++i) {
         uint32_t d[WL::DESCR];
-        const int n = WL::descr(p.w, gen::tx_key(p.seed, t, i), d);
+        const int n = WL::descr(p.w, gen::tx_key(p.seed, t, i), t, d);
         uint32_t* o = out + (static_cast<uint64_t>(i) * p.T + t) * wpt;
         for (int k = 0; k < wpt; ++k) o[k] = k < n ? d[k] : 0u;
     }

@@ -9,7 +9,7 @@ from paper_conf_cgo_xuwglgq14_b200 import build as B
 from paper_conf_cgo_xuwglgq14_b200 import gstm as G
 
 WL_FIELDS = ["n_reads", "n_writes", "ra_kind", "n_words", "n_accesses", "ht_buckets", "ht_lookup_pct",
-             "ht_key_range", "km_clusters", "km_dims", "shard_bits", "shard", "km_stride", "km_assign"]
+             "ht_key_range", "km_clusters", "km_dims", "shard_bits", "shard", "km_stride", "km_assign", "ra_partition"]
 
 
 def ensure_built():

@@ -293,6 +293,31 @@ def test_concurrency_cap_replay(mode, wl, kw, T, K, cap):
     assert st.commits + st.commits_ro == T * K
 
 
+@pytest.mark.parametrize("mode", ["hv", "tbv", "hv_backoff", "vbv", "fgl", "cgl"])
+@pytest.mark.parametrize("kind", [0, 1])
+@pytest.mark.parametrize("paired", [False, True])
+def test_disjoint_access_sets_unique_result(mode, kind, paired):
+    """SURVEY §8c-O4 special case: thread t touches only [t*k, t*k + k)
+    (ra_partition = k) and every word has its own lock, so the result is
+    unique: the GPU heap and every result equal the canonical serial
+    execution bit for bit, and the STM never aborts."""
+    k, T, K = 16, 4096, 8
+    kw = dict(n_reads=4, n_writes=4) if kind == 0 else dict(n_reads=5)
+    g, gp, op, init = U.make("ra", T, K, 16, mode=mode, paired=paired, ra_kind=kind, n_words=T * k,
+                             ra_partition=k, **kw)
+    st, heap, stamps, res = U.run_verified(g, "ra", op, init, T, K, 31)
+    h = init.copy()
+    want_res, _ = O.serial(op, h, T, K, 31)
+    assert (heap == h).all()
+    assert (res[:T * K] == want_res).all()
+    if mode in ("hv", "tbv", "hv_backoff"):
+        assert st.aborts == 0 and st.lock_retries == 0 and st.postvalidations == 0, st.as_dict()
+    # a thread range beyond the heap is rejected, not silently wrapped
+    g.set_params(ra_partition=k + 1)
+    with pytest.raises(G.GstmError, match="EINVAL"):
+        g.launch("ra", T, K, 32)
+
+
 @pytest.mark.parametrize("mode", ["hv", "tbv", "fgl"])
 @pytest.mark.parametrize("persist", [0, 1])
 def test_l2_persisting_lock_table_replay(mode, persist):

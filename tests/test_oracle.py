@@ -648,3 +648,50 @@ def test_km_full_iteration_is_a_lloyd_step(stride):
         want = np.where(cnt[:, None] > 0, sums // np.maximum(cnt, 1)[:, None], cent)
         assert (_km_table(p, heap) == want).all()
         assert not heap[:Cn * S].any()                       # accumulators restart from zero
+
+
+# ---------------------------------------------------------------------------
+# disjoint access sets: thread t touches only [t*k, t*k + k)
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("kind", [0, 1])
+def test_ra_partition_descriptors_stay_in_the_thread_range(kind):
+    """Every word of thread t's transactions lies in [t*k, t*k + k), and a
+    thread range that does not fit the heap is rejected."""
+    k, T, K = 16, 37, 5
+    p = O.params("ra", n_reads=4, n_writes=3, ra_kind=kind, n_words=T * k, ra_partition=k)
+    nw = 4 if kind == 1 else 7
+    seen = set()
+    for t in range(T):
+        for i in range(K):
+            d = O.descr(p, 9, t, i)
+            words = d[:nw].astype(np.int64)
+            assert ((words >= t * k) & (words < t * k + k)).all()
+            seen.update(int(w) - t * k for w in words)
+    assert seen == set(range(k))          # the draws cover the range (uniform bounded draws)
+    small = O.params("ra", n_reads=4, n_writes=3, ra_kind=kind, n_words=T * k - 1, ra_partition=k)
+    with pytest.raises(Exception):
+        O.descr(small, 9, T - 1, 0)
+
+
+@pytest.mark.parametrize("kind", [0, 1])
+def test_ra_partition_result_is_order_independent(kind):
+    """With disjoint access sets the final heap and every result do not depend
+    on the serial order: canonical order (i-major) == thread-by-thread order ==
+    reversed thread order, computed with the single-transaction executor."""
+    k, T, K = 8, 24, 6
+    p = O.params("ra", n_reads=3, n_writes=2, ra_kind=kind, n_words=T * k, ra_partition=k)
+    init = O.init_heap(p, T * k)
+    h0 = init.copy()
+    res0, upd0 = O.serial(p, h0, T, K, 5)
+    for order in (range(T), reversed(range(T))):
+        h = init.copy()
+        res = np.zeros(T * K, dtype=np.uint32)
+        for t in order:
+            for i in range(K):
+                res[i * T + t], _ = O.exec_tx(p, h, T, K, 5, t, i)
+        assert (h == h0).all()
+        assert (res == res0).all()
+    # and brute force over every interleaving of a tiny instance: one outcome
+    q = O.params("ra", n_reads=2, n_writes=2, ra_kind=kind, n_words=6, ra_partition=2)
+    n, match, nd = O.brute(q, O.init_heap(q, 6), 3, 2, 11)
+    assert n > 1 and nd == 1
