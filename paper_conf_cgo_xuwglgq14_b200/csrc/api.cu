@@ -29,8 +29,12 @@ static void set_error(const char* fmt, ...)
         }                                                                                 \
     } while (0)
 
-static constexpr size_t kMetaBytes = 256 * 1024;  // metadata block (M_WORDS used) + g_clock candidates
-static constexpr int kClockCandidates = 64;        // candidate lines for g_clock after M_WORDS ...
+static constexpr size_t kMetaBytes = 1024 * 1024; // metadata block (M_WORDS used) + g_clock candidates
+// candidate lines for g_clock after M_WORDS ... (only ~1 line in 32 is fast: on
+// one B200, 2 of 64 probed lines ran the bank kernel at 9.6 G tx/s and the
+// other 62 at 7.0-7.5; 256 candidates miss them all with
+// probability ~0.03%)
+static constexpr int kClockCandidates = 256;
 static constexpr int kClockStride = 288;           // ... 2304 B apart (crosses 256 B and 2 KiB address bits)
 static_assert(gstm::M_SEQ >= gstm::M_WORDS + kClockCandidates * kClockStride + 16 && gstm::M_SEQ * 8 + 128 <= kMetaBytes,
               "STM-VBV sequence lock must sit on its own line after the clock candidates");

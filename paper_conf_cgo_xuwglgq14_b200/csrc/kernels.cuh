@@ -32,8 +32,8 @@ enum {
     M_PHASE = 112,                     // 8 phase-cycle accumulators (GSTM_PHASE_TIMING builds)
     M_WORK = 120,                      // next unstarted STM thread (persistent grid), own line
     M_WORDS = 128,
-    // after the 64 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
-    M_SEQ = M_WORDS + 64 * 288 + 16,   // STM-VBV global sequence lock, own line
+    // after the 256 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
+    M_SEQ = M_WORDS + 256 * 288 + 16,  // STM-VBV global sequence lock, own line
 };
 
 enum { ERR_LOGOVF = 1, ERR_TIMEOUT = 2, ERR_INVALID = 4 };
