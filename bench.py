@@ -495,6 +495,7 @@ def run_native(args):
             "abort_ratio": tot["aborts"] / max(1.0, tot["aborts"] + done),
             "stats": {k: int(v) for k, v in tot.items()},
             "invariant_total_balance_ok": bool(balance_ok),
+            "clock_slot": int(st_tot.clock_slot),      # probed g_clock line
             "clocks": clocks,
             "gpu_launches": 3 * args.steps,
             "wall_s_timed_region": wall,

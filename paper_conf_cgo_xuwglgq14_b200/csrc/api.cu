@@ -71,30 +71,61 @@ struct gstm_handle {
 // L2 persistence for the version-lock table (params.l2_persist_locks): an
 // access-policy window on the handle's stream covering the lock table,
 // hit property persisting, set around the transaction kernel's launch.
-static cudaError_t set_l2_lock_window(gstm_t* h, bool on)
+// The persisting set-aside (cudaLimitPersistingL2CacheSize) is device-wide and
+// outlives the handle that set it: it is released again (limit 0, persisting
+// lines demoted) before any launch that does not use it -- a leftover 64 MiB
+// set-aside cut EB with a 256 MiB lock table from 411 to 170 M tx/s.
+static bool g_l2_set_aside = false;
+
+static cudaError_t l2_limits(size_t* max_persist, size_t* max_window)
 {
-    static size_t max_persist = 0, max_window = 0;
-    if (!max_window) {
+    static size_t mp = 0, mw = 0;
+    if (!mw) {
         int dev = 0;
         cudaDeviceProp pr;
         cudaError_t e = cudaGetDevice(&dev);
         if (e == cudaSuccess) e = cudaGetDeviceProperties(&pr, dev);
         if (e != cudaSuccess) return e;
-        max_persist = pr.persistingL2CacheMaxSize;
-        max_window = pr.accessPolicyMaxWindowSize;
-        if (!max_window) return cudaErrorNotSupported;
+        mp = pr.persistingL2CacheMaxSize;
+        mw = pr.accessPolicyMaxWindowSize;
     }
-    // a table larger than the persisting set-aside would only shrink the L2
-    // left for everything else (measured: EB with 2^26 locks, 256 MiB, 384 ->
-    // 146 M tx/s): the knob then leaves the stream alone
-    if ((sizeof(uint32_t) << h->bits) > std::min(max_persist, max_window)) return cudaSuccess;
+    *max_persist = mp;
+    *max_window = mw;
+    return cudaSuccess;
+}
+
+// does the handle's lock table fit the persisting set-aside?  A larger table
+// would only shrink the L2 left for everything else (measured: EB with 2^26
+// locks, 256 MiB, 384 -> 146 M tx/s), so the knob then does nothing.
+static bool l2_persist_fits(const gstm_t* h)
+{
+    size_t mp = 0, mw = 0;
+    if (l2_limits(&mp, &mw) != cudaSuccess || !mp || !mw) return false;
+    return (sizeof(uint32_t) << h->bits) <= std::min(mp, mw);
+}
+
+static cudaError_t release_l2_set_aside()
+{
+    if (!g_l2_set_aside) return cudaSuccess;
+    g_l2_set_aside = false;
+    cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    if (e == cudaSuccess) e = cudaCtxResetPersistingL2Cache();
+    return e;
+}
+
+static cudaError_t set_l2_lock_window(gstm_t* h, bool on)
+{
     cudaStreamAttrValue a;
     memset(&a, 0, sizeof(a));
     if (on) {
-        const size_t bytes = std::min(sizeof(uint32_t) << h->bits, max_window);
-        const size_t lim = std::min(bytes, max_persist);
-        cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+        size_t mp = 0, mw = 0;
+        cudaError_t e = l2_limits(&mp, &mw);
         if (e != cudaSuccess) return e;
+        const size_t bytes = std::min(sizeof(uint32_t) << h->bits, mw);
+        const size_t lim = std::min(bytes, mp);
+        e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+        if (e != cudaSuccess) return e;
+        g_l2_set_aside = true;
         a.accessPolicyWindow.base_ptr = h->locks;
         a.accessPolicyWindow.num_bytes = bytes;
         a.accessPolicyWindow.hitRatio = bytes ? std::min(1.0f, static_cast<float>(lim) / static_cast<float>(bytes)) : 0.f;
@@ -298,6 +329,7 @@ uint32_t gstm_flags(const gstm_t* h) { return h && h->paired ? GSTM_CREATE_PAIRE
 
 void gstm_destroy(gstm_t* h)
 {
+    if (h && h->params.l2_persist_locks) release_l2_set_aside();
     if (!h) return;
     if (h->stream) cudaStreamSynchronize(h->stream);
     cudaFree(h->block);
@@ -600,8 +632,9 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
         CUDA_TRY(launch_km_assign(kp, h->km_cluster, h->stream));
         kp.w.km_cluster = h->km_cluster;
     }
-    const bool persist = P.l2_persist_locks && !h->paired && h->locks;
+    const bool persist = P.l2_persist_locks && !h->paired && h->locks && l2_persist_fits(h);
     if (persist) CUDA_TRY(set_l2_lock_window(h, true));
+    else CUDA_TRY(release_l2_set_aside());
     CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
     if (persist) CUDA_TRY(set_l2_lock_window(h, false));
     CUDA_TRY(launch_finish(h->meta, h->clock, h->stream));
