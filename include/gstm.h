@@ -166,7 +166,10 @@ typedef struct {
 /* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */
 /* Allocates a heap of heap_words uint32 (zeroed), a table of
  * 2^lock_table_bits version locks (0 <= bits <= 30, zeroed), the global clock
- * (0) and statistics.  Returns NULL on error (gstm_last_error). */
+ * (0) and statistics.  For tables of >= 2^14 locks it places g_clock on the
+ * fastest of 256 candidate L2 lines, measured with a short probe kernel
+ * (~120 ms; GSTM_CLOCK_SLOT=k forces line k).  Synchronous.
+ * Returns NULL on error (gstm_last_error). */
 gstm_t* gstm_create(uint64_t heap_words, uint32_t lock_table_bits);
 /* flags for gstm_create_ex */
 #define GSTM_CREATE_PAIRED 1u
