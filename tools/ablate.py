@@ -51,6 +51,8 @@ def main():
     ap.add_argument("--sync", action="store_true", help="host sync after every step")
     ap.add_argument("--seed-base", type=int, default=0)
     ap.add_argument("--flush-first", action="store_true", help="allocate the L2-flush buffer before the handle")
+    ap.add_argument("--pre-alloc-mb", type=int, default=0,
+                    help="cudaMalloc this many MiB before the handle (moves the handle's physical pages)")
     ap.add_argument("--variant-timeout", type=int, default=240, help="seconds per variant process")
     ap.add_argument("--inproc", action="store_true",
                     help="run all variants in this process (default: one fresh process per variant, so "
@@ -86,6 +88,7 @@ def main():
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
     flush = torch.empty(64 << 20, dtype=torch.float32, device="cuda") if a.flush_first else None
+    pre = torch.empty(a.pre_alloc_mb << 18, dtype=torch.float32, device="cuda") if a.pre_alloc_mb else None
     for var in a.variants:
         kv = parse_variant(var)
         mode = kv.pop("mode", "auto")
