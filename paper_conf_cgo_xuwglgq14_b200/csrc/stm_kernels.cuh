@@ -287,7 +287,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
             if (r == C_OK) {
                 got = true;
-                if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m); else tx.writeback(m);                                      // l.79-82
+                // l.79-82
+                if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m);
+                else tx.writeback(m);
             } else if (r == C_LOCK) {
                 cnt.inc(S_LOCK_RETRIES);                              // l.73-74: retry next iteration
                 if (POL == POL_BACKOFF) {
@@ -343,7 +345,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 if (static_cast<int>(prim::lane_id()) == L) {
                     const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, false);
                     if (r == C_OK) {
-                        if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m); else tx.writeback(m);                              // l.79-82
+                        // l.79-82
+                        if constexpr (RunWriteback<WL>::value) tx.writeback_runs(m);
+                        else tx.writeback(m);
                         sl = static_cast<uint32_t>(clock_fetch_add(m.clock, 1u)) + 1u;   // l.83
                         tx.release_and_update(m, sl);                 // l.84
                         if (p.tx_stamp) {
