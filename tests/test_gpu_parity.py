@@ -237,6 +237,45 @@ def test_ht_replay(mode):
     assert int(inserted.sum()) == len(keys_ins)
 
 
+@pytest.mark.parametrize("mode,extra", [("hv", dict(k_lock=1)), ("tbv", dict())])
+def test_ht_config2_full_size_replay(mode, extra):
+    """BASELINE configs[2] at full size, as `bench.py --workload ht` and
+    tools/ablate.py run it: 2^20 buckets, 2^22 threads x 4 (16.8M operations,
+    90/10 lookup/insert, keys in [1, 2^22]), 2^22 version locks: bit-exact
+    stamp-order replay of every result and of the final table."""
+    T, K = 1 << 22, 4
+    g, gp, op, init = U.make("ht", T, K, 22, mode=mode, **extra)
+    st, heap, stamps, res = U.run_verified(g, "ht", op, init, T, K, 7)
+    assert st.commits == int((res == 3).sum())
+
+
+@pytest.mark.parametrize("mode", ["hv", "fgl"])
+def test_km_config4_full_size_closed_form(mode):
+    """BASELINE configs[4] at full size: 16M points (K = 1), 1024 clusters x
+    16 dims, the default 8 resident warps per SM; the order-free result equals
+    bincount / add.at over the generated descriptors, and the replay holds."""
+    T, K, Cn, D = 1 << 24, 1, 1024, 16
+    g, gp, op, init = U.make("km", T, K, 20, mode=mode)
+    st, heap, stamps, res = U.run_verified(g, "km", op, init, T, K, 9)
+    d = g.dump_descr("km", T, K, 9).astype(np.int64)
+    rec = heap.reshape(Cn, D + 1).astype(np.int64)
+    assert (rec[:, 0] == np.bincount(d[:, 0], minlength=Cn)).all()
+    sums = np.zeros((Cn, D), dtype=np.int64)
+    np.add.at(sums, d[:, 0], d[:, 1:])
+    assert (rec[:, 1:] == sums).all()
+
+
+@pytest.mark.parametrize("mode", ["hv", "tbv"])
+def test_eb_config3_full_heap_replay(mode):
+    """BASELINE configs[3]'s largest point: a 2^26-word (256 MiB) heap with the
+    hot set the whole heap, A = 16 accesses, 2^22 version locks persisting in
+    L2 (the EB default), 2^18 threads x 4: bit-exact stamp-order replay."""
+    T, K, H = 1 << 18, 4, 1 << 26
+    g, gp, op, init = U.make("eb", T, K, 22, mode=mode, n_words=H, n_accesses=16, heap_words=H)
+    assert gp.l2_persist_locks == 1
+    U.run_verified(g, "eb", op, init, T, K, 13)
+
+
 def test_km_closed_form():
     """k-means cluster update: order-free result == numpy bincount / add.at."""
     T, K, Cn, D = 1 << 20, 1, 1024, 16
