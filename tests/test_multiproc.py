@@ -131,3 +131,29 @@ def test_two_rank_key_partitioned_ht_gloo():
         assert out[0] == total                                   # update commits = inserted keys
         assert all(O.key_owner(k, 1) == rank for k in keys)
     assert not set(got[0][2]) & set(got[1][2])                   # disjoint shards
+
+
+def test_bench_roofline_object_is_the_contract_and_the_cost_model():
+    """bench.py's `roofline` object (CPU-only arithmetic): contract keys, the
+    algorithmic sector model of DESIGN.md §7.2 (paired bank update = 2 pair
+    loads + 2 atom.or.b64 + 2 pair stores = 6 x 32 B; read-only = 2 loads;
+    split TBV update 10 sectors, + 2 pre-lock VBV loads for HV), and
+    achieved = bytes per launch / launch time."""
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    tot = {"commits": 1_000_000, "commits_ro": 250_000}
+    r = bench.roofline(bench.Variant("hv", "paired"), "hv", tot, t_ms=2.0, steps=2,
+                       peaks={"hbm_gbs": 6000.0}, peak_src="test", traffic=123)
+    assert {"bound", "achieved", "peak", "unit", "frac", "traffic"} <= set(r)
+    assert r["bound"] == "hbm" and r["unit"] == "GB/s" and r["traffic"] == 123
+    assert r["bytes_per_unit"] == {"update_tx": 192, "read_only_tx": 64}
+    per_launch = (1_000_000 * 192 + 250_000 * 64) / 2
+    assert r["algorithmic_bytes_per_launch"] == per_launch
+    assert abs(r["achieved"] - per_launch / 1e-3 / 1e9) < 1e-9
+    assert abs(r["frac"] - r["achieved"] / 6000.0) < 1e-12
+    split_tbv = bench.roofline(bench.Variant("tbv", "split"), "tbv", tot, 2.0, 2, {}, "fallback", traffic=0)
+    assert split_tbv["bytes_per_unit"] == {"update_tx": 320, "read_only_tx": 128}
+    assert split_tbv["peak"] == 6650.0                  # the profiling guide's fallback
+    split_hv = bench.roofline(bench.Variant("hv", "split"), "hv", tot, 2.0, 2, {}, "fallback", traffic=0)
+    assert split_hv["bytes_per_unit"]["update_tx"] == 384
