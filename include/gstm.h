@@ -265,16 +265,27 @@ int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* he
  * km_assign fills the table with centroid word j = splitmix64(j) >> 56. */
 int gstm_km_recenter(gstm_t* h);
 
-/* As gstm_run_host without the final synchronisation: the copy-in, the
- * launch and the copy-out are enqueued on the handle's stream and the call
- * returns.  heap_in must stay valid and heap_out must not be read until
- * gstm_sync (or gstm_stats) returns.  With pinned host buffers the copies
- * are asynchronous, so two handles on two streams overlap one step's copies
- * with the other's transactions (double-buffered streaming). */
+/* As gstm_run_host without the final synchronisation, pipelined: the
+ * host->device copy of heap_in goes on an internal copy-in stream into a
+ * device staging buffer, the staging -> heap move (pack kernel on the paired
+ * layout), the launch and the heap -> staging move go on the handle's stream,
+ * and the device->host copy into heap_out on an internal copy-out stream,
+ * ordered by events.  Consecutive calls on one handle therefore overlap step
+ * k+1's copy-in and step k's copy-out with step k's / k+1's transactions
+ * (DESIGN.md §7.1).  The first call after a gstm_join / gstm_sync starts
+ * after all work already enqueued on the handle's stream.  heap_in must stay
+ * valid and heap_out must not be read until gstm_sync (or gstm_join followed
+ * by a synchronisation of the handle's stream) returns; the stats of the
+ * last launch are in gstm_stats after gstm_sync, the running totals in
+ * gstm_stats_total.  words <= the heap size. */
 int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
                         uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed);
-/* Wait for everything enqueued on the handle's stream; returns the status of
- * the last launch (GSTM_OK if none). */
+/* Make the handle's stream wait (on the device, without blocking the host)
+ * for the last gstm_run_host_async copy-out, so an event recorded on that
+ * stream afterwards follows every copy.  GSTM_OK; no-op without calls. */
+int gstm_join(gstm_t* h);
+/* gstm_join, then wait for everything enqueued on the handle's stream;
+ * returns the status of the last launch (GSTM_OK if none). */
 int gstm_sync(gstm_t* h);
 
 /* ---- test and measurement entry points --------------------------------- */

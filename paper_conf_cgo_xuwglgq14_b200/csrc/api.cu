@@ -59,6 +59,15 @@ struct gstm_handle {
     uint64_t km_cap = 0;
     cudaStream_t own_stream = nullptr, stream = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    // pipelined host-buffer steps (gstm_run_host_async): copy streams,
+    // staging buffers and the events that order them
+    cudaStream_t s_in = nullptr, s_out = nullptr;
+    cudaEvent_t ev_call = nullptr, ev_in_ready = nullptr, ev_in_free = nullptr, ev_out_ready = nullptr,
+                ev_out_free = nullptr;
+    uint32_t* stage_in = nullptr;
+    uint32_t* stage_out = nullptr;
+    uint64_t stage_words = 0;
+    bool pipe_open = false;          // a pipelined call is in flight since the last join
     gstm_params_t params{};
     int mode = GSTM_MODE_AUTO;
     // last launch
@@ -337,8 +346,14 @@ void gstm_destroy(gstm_t* h)
     cudaFree(h->tx_stamp);
     cudaFree(h->tx_result);
     cudaFree(h->km_cluster);
-    if (h->ev0) cudaEventDestroy(h->ev0);
-    if (h->ev1) cudaEventDestroy(h->ev1);
+    if (h->s_in) cudaStreamSynchronize(h->s_in);
+    if (h->s_out) cudaStreamSynchronize(h->s_out);
+    cudaFree(h->stage_in);
+    cudaFree(h->stage_out);
+    for (cudaEvent_t e : {h->ev0, h->ev1, h->ev_call, h->ev_in_ready, h->ev_in_free, h->ev_out_ready, h->ev_out_free})
+        if (e) cudaEventDestroy(e);
+    if (h->s_in) cudaStreamDestroy(h->s_in);
+    if (h->s_out) cudaStreamDestroy(h->s_out);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
     delete h;
 }
@@ -720,20 +735,84 @@ int gstm_run_host(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* he
     return gstm_stats(h, stats ? stats : &local);
 }
 
+static int ensure_pipe(gstm_t* h, uint64_t words)
+{
+    if (!h->s_in) {
+        CUDA_TRY(cudaStreamCreateWithFlags(&h->s_in, cudaStreamNonBlocking));
+        CUDA_TRY(cudaStreamCreateWithFlags(&h->s_out, cudaStreamNonBlocking));
+        for (cudaEvent_t* e : {&h->ev_call, &h->ev_in_ready, &h->ev_in_free, &h->ev_out_ready, &h->ev_out_free})
+            CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+    }
+    if (h->stage_words < words) {
+        // the staging buffers may still be in use by calls in flight
+        CUDA_TRY(cudaStreamSynchronize(h->s_in));
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        CUDA_TRY(cudaStreamSynchronize(h->s_out));
+        cudaFree(h->stage_in);
+        cudaFree(h->stage_out);
+        h->stage_in = h->stage_out = nullptr;
+        h->stage_words = 0;
+        if (cudaMalloc(&h->stage_in, words * 4) != cudaSuccess || cudaMalloc(&h->stage_out, words * 4) != cudaSuccess) {
+            set_error("out of device memory (staging)");
+            return GSTM_ENOMEM;
+        }
+        h->stage_words = words;
+    }
+    return GSTM_OK;
+}
+
 int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32_t* heap_out, uint64_t words,
                         uint64_t n_threads, uint32_t tx_per_thread, uint64_t seed)
 {
     if (!h || words > h->heap_words || (words && (!heap_in || !heap_out))) { set_error("gstm_run_host_async: bad buffers"); return GSTM_EINVAL; }
-    int rc = copy_in(h, heap_in, 0, words);
+    if (!words) return gstm_launch(h, workload, n_threads, tx_per_thread, seed);
+    int rc = ensure_pipe(h, words);
     if (rc) return rc;
+    if (!h->pipe_open) {
+        // the first call of a pipeline follows everything already enqueued
+        // on the handle's stream (e.g. the caller's start event)
+        CUDA_TRY(cudaEventRecord(h->ev_call, h->stream));
+        CUDA_TRY(cudaStreamWaitEvent(h->s_in, h->ev_call, 0));
+        CUDA_TRY(cudaStreamWaitEvent(h->s_out, h->ev_call, 0));
+        h->pipe_open = true;
+    }
+    // copy-in: into the staging buffer once the previous step moved it out
+    CUDA_TRY(cudaStreamWaitEvent(h->s_in, h->ev_in_free, 0));
+    CUDA_TRY(cudaMemcpyAsync(h->stage_in, heap_in, words * 4, cudaMemcpyHostToDevice, h->s_in));
+    CUDA_TRY(cudaEventRecord(h->ev_in_ready, h->s_in));
+    // the step on the handle's stream: staging -> heap, transactions, heap -> staging
+    CUDA_TRY(cudaStreamWaitEvent(h->stream, h->ev_in_ready, 0));
+    if (h->paired) CUDA_TRY(launch_pack(h->stage_in, h->heap, words, 1, h->stream));
+    else CUDA_TRY(cudaMemcpyAsync(h->heap, h->stage_in, words * 4, cudaMemcpyDeviceToDevice, h->stream));
+    CUDA_TRY(cudaEventRecord(h->ev_in_free, h->stream));
     rc = gstm_launch(h, workload, n_threads, tx_per_thread, seed);
     if (rc) return rc;
-    return copy_out(h, heap_out, 0, words);
+    CUDA_TRY(cudaStreamWaitEvent(h->stream, h->ev_out_free, 0));
+    if (h->paired) CUDA_TRY(launch_pack(h->stage_out, h->heap, words, 0, h->stream));
+    else CUDA_TRY(cudaMemcpyAsync(h->stage_out, h->heap, words * 4, cudaMemcpyDeviceToDevice, h->stream));
+    CUDA_TRY(cudaEventRecord(h->ev_out_ready, h->stream));
+    // copy-out on its own stream, overlapping the next step's transactions
+    CUDA_TRY(cudaStreamWaitEvent(h->s_out, h->ev_out_ready, 0));
+    CUDA_TRY(cudaMemcpyAsync(heap_out, h->stage_out, words * 4, cudaMemcpyDeviceToHost, h->s_out));
+    CUDA_TRY(cudaEventRecord(h->ev_out_free, h->s_out));
+    return GSTM_OK;
+}
+
+int gstm_join(gstm_t* h)
+{
+    if (!h) { set_error("gstm_join: NULL handle"); return GSTM_EINVAL; }
+    if (h->pipe_open) {
+        CUDA_TRY(cudaStreamWaitEvent(h->stream, h->ev_out_free, 0));
+        h->pipe_open = false;
+    }
+    return GSTM_OK;
 }
 
 int gstm_sync(gstm_t* h)
 {
     if (!h) { set_error("gstm_sync: NULL handle"); return GSTM_EINVAL; }
+    int rc = gstm_join(h);
+    if (rc) return rc;
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     if (!h->launched) return GSTM_OK;
     gstm_stats_t s;

@@ -38,7 +38,7 @@ EXPORTS = [
     "gstm_read_locks", "gstm_read_clock", "gstm_reset_meta", "gstm_set_clock", "gstm_launch", "gstm_stats",
     "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
-    "gstm_lock_log", "gstm_ubench", "gstm_km_recenter", "gstm_run_host_async", "gstm_sync",
+    "gstm_lock_log", "gstm_ubench", "gstm_km_recenter", "gstm_run_host_async", "gstm_join", "gstm_sync",
 ]
 
 
@@ -108,6 +108,7 @@ def lib():
             "gstm_km_recenter": (i32, [V]),
             "gstm_run_host_async": (i32, [V, i32, V, V, u64, u64, u32, u64]),
             "gstm_sync": (i32, [V]),
+            "gstm_join": (i32, [V]),
             "gstm_write_heap": (i32, [V, V, u64, u64]),
             "gstm_read_heap": (i32, [V, V, u64, u64]),
             "gstm_read_locks": (i32, [V, V, u64]),
@@ -363,6 +364,10 @@ class Gstm:
         assert heap_in.dtype == np.uint32 and heap_out.dtype == np.uint32 and heap_in.size == heap_out.size
         _check(lib().gstm_run_host_async(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
                                          n_threads, tx_per_thread, seed), "gstm_run_host_async")
+
+    def join(self) -> int:
+        """Make the handle's stream wait (device-side) for the last run_host_async copy-out."""
+        return _check(lib().gstm_join(self.h), "gstm_join")
 
     def sync(self) -> int:
         return _check(lib().gstm_sync(self.h), "gstm_sync")

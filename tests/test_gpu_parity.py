@@ -544,6 +544,38 @@ def test_run_host_async_double_buffered(paired):
         assert int(outs[k].astype(np.int64).sum()) == 1000 * N
 
 
+@pytest.mark.parametrize("paired", [False, True])
+def test_run_host_async_pipelined_one_handle(paired):
+    """Consecutive gstm_run_host_async calls on ONE handle overlap step k+1's
+    copy-in and step k's copy-out with the transactions (internal copy
+    streams, staging buffers).  Disjoint access sets (ra_partition) make every
+    step's result unique, so each step's host output must equal the oracle's
+    serial execution of that step's own input, bit for bit; the handle's last
+    launch also replays, and a blocking call afterwards still works."""
+    import torch
+    k_part, T, K = 8, 2048, 4
+    N = T * k_part
+    g, gp, op, init = U.make("ra", T, K, 14, mode="hv", paired=paired, n_reads=4, n_writes=4, n_words=N,
+                             ra_partition=k_part)
+    rng = np.random.default_rng(5)
+    ins = [torch.from_numpy(rng.integers(0, 2**32, N, dtype=np.uint32).view(np.int32)).pin_memory().numpy().view(np.uint32)
+           for _ in range(5)]
+    outs = [torch.zeros(N, dtype=torch.int32).pin_memory().numpy().view(np.uint32) for _ in range(5)]
+    for k in range(5):
+        g.run_host_async("ra", ins[k], outs[k], T, K, 40 + k)
+    assert g.sync() == 0
+    for k in range(5):
+        h = ins[k].copy()
+        O.serial(op, h, T, K, 40 + k)
+        assert (outs[k] == h).all(), k
+    stamps, res = g.read_tx_log(T * K)
+    h = ins[4].copy()
+    assert O.replay(op, h, T, K, 44, stamps, res)[0] == 0 and (h == outs[4]).all()
+    out = np.zeros(N, dtype=np.uint32)
+    g.run_host("ra", ins[0], out, T, K, 40)
+    assert (out == outs[0]).all()
+
+
 @pytest.mark.parametrize("kind", [0, 1, 2, 3, 4, 5])
 def test_ubench_runs(kind):
     ops, ms = G.gstm_ubench(kind, 8 << 20, 1 << 22, 148 * 256 * 4)
