@@ -446,7 +446,10 @@ def run_native(args):
         # and its result out, on the library's copy streams, overlapping the
         # neighbouring steps' transactions; one CUDA-event
         # pair around all steps, joined onto the launching stream.
-        g2 = var.handle(G, stream)
+        # the same handle as the kernel-only measurement (its g_clock line
+        # was probed once; a second handle would draw its own placement,
+        # DESIGN.md §6.5)
+        g2 = g
         for w in range(2):                                    # warm-up
             g2.run_host_async("bank", h_in, h_out, T, K, seed0 + w)
         g2.sync()
@@ -470,7 +473,6 @@ def run_native(args):
                         "api": "gstm_run_host_async (host buffers, pinned; copies pipelined with the "
                                "neighbouring steps' transactions), gstm_join + CUDA events",
                         "steps": n_e2e}
-        g2.close()
         if not args.no_cgl:
             extra["cgl"] = cgl_baseline(G, stream, T, seed0)
             extra["stm_vbv"] = cgl_baseline(G, stream, T, seed0, mode="vbv")
