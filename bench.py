@@ -545,6 +545,12 @@ def ht_walk_count(heap, B, M):
     return int(keys.size), int(np.unique(keys).size)
 
 
+# A3.l71's pre-lock VBV is optional ("to reduce lock contention"); HT update
+# commits are 10% of the mix and rarely contend, so the R extra loads only cost
+# (measured: 5.44 -> 5.86 G tx/s without it)
+HT_PRELOCK = 0
+
+
 def run_native_ht(args):
     import numpy as np
     import torch
@@ -570,13 +576,15 @@ def run_native_ht(args):
     M = T * K
     words = HT_BUCKETS + 2 * M
     mode = args.mode if args.mode in ("hv", "tbv", "auto", "fgl", "hv_backoff") else "hv"
+    prelock = HT_PRELOCK if args.prelock is None else args.prelock
     stream = torch.cuda.Stream(device=dev)
     torch.cuda.set_stream(stream)
 
     def handle():
         g = G.Gstm(words, HT_BITS)
         g.set_workload_defaults("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90,
-                                shard_bits=world.bit_length() - 1, shard=rank, k_lock=args.k_lock)
+                                shard_bits=world.bit_length() - 1, shard=rank, k_lock=args.k_lock,
+                                prelock_vbv=prelock)
         g.set_mode(mode)
         g.set_stream(stream)
         g.init_heap("ht")
@@ -651,7 +659,9 @@ def run_native_ht(args):
             "config": {"workload": "hash table insert/lookup (BASELINE configs[2]), key-partitioned over ranks",
                        "buckets_per_gpu": HT_BUCKETS, "threads_per_gpu": T, "tx_per_thread": K,
                        "lookup_pct": 90, "key_range": HT_KEYS, "lock_table_bits": HT_BITS,
-                       "variant": f"{mode}/split/k_lock={args.k_lock} (mode used: {mode_used})",
+                       "variant": f"{mode}/split/k_lock={args.k_lock}"
+                                  + (f"/prelock={prelock}" if mode_used in ("hv", "hv_backoff") else "")
+                                  + f" (mode used: {mode_used})",
                        "partition": f"{world} shard(s): rank g owns keys with mix64 top {world.bit_length() - 1} bits = g",
                        "l2": "flushed (256 MiB write) between timed steps"},
             "abort_ratio": tot["aborts"] / max(1.0, tot["aborts"] + done),
