@@ -87,7 +87,7 @@ typedef struct {
     uint32_t km_clusters;    /* KM: cluster records                                     */
     uint32_t km_dims;        /* KM: features per point (<= 16)                          */
     /* runtime knobs */
-    uint32_t prelock_vbv;    /* HV: value-validate before locking (A3.l71), default 1   */
+    uint32_t prelock_vbv;    /* HV: value-validate before locking (A3.l71); 1, HT 0    */
     uint32_t k_lock;         /* lock-acquisition rounds before abort; 0 = inf   */
     uint32_t backoff_ns;     /* warp-uniform backoff after an abort; 0 = none           */
     uint32_t verify;         /* record per-tx stamp and result (gstm_read_tx_log)       */

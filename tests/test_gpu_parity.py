@@ -237,7 +237,7 @@ def test_ht_replay(mode):
     assert int(inserted.sum()) == len(keys_ins)
 
 
-@pytest.mark.parametrize("mode,extra", [("hv", dict(k_lock=1)), ("hv", dict(k_lock=1, prelock_vbv=0)), ("tbv", dict())])
+@pytest.mark.parametrize("mode,extra", [("hv", dict(k_lock=1)), ("hv", dict(k_lock=1, prelock_vbv=1)), ("tbv", dict())])
 def test_ht_config2_full_size_replay(mode, extra):
     """BASELINE configs[2] at full size, as `bench.py --workload ht` and
     tools/ablate.py run it: 2^20 buckets, 2^22 threads x 4 (16.8M operations,
