@@ -21,6 +21,11 @@
 #include <cstdint>
 #include "prim.cuh"
 
+// ablation builds: -DGSTM_PV_ATTR=__noinline__
+#ifndef GSTM_PV_ATTR
+#define GSTM_PV_ATTR __forceinline__
+#endif
+
 namespace gstm {
 
 enum { MODE_HV = 1, MODE_TBV = 2 };
@@ -208,7 +213,7 @@ struct Tx {
     // ---- A3.l6-20 PostValidation(version) --------------------------------
     // "snapshot <- version" (l.7) never lowers the snapshot (reading Q9);
     // restarts are bounded by spin_cap (the paper loops; bounded => abort).
-    __device__ __forceinline__ bool post_validation(const Meta& m, uint32_t version)
+    __device__ GSTM_PV_ATTR bool post_validation(const Meta& m, uint32_t version)
     {
         ++n_postval;
         if (version > snapshot) snapshot = version;                // l.7
