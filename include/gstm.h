@@ -102,8 +102,9 @@ typedef struct {
     uint32_t lock_pipeline;  /* N > 0: the first lock-acquisition round of each of a   */
                              /*    transaction's first N executions issues all atom.or */
                              /*    at once; every other round is      */
-                             /*    sequential in ascending id (progress is kept for    */
-                             /*    any finite N).  0: always sequential.  Local-memory */
+                             /*    sequential in ascending id (every round after a     */
+                             /*    failed one, for any k_lock; progress is kept for    */
+                             /*    any N).  0: always sequential.  Local-memory        */
                              /*    logs pipeline only logs of <= 8 locks.              */
                              /*    Default 1 (RA, EB: 0)                               */
     uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
@@ -128,8 +129,10 @@ typedef struct {
     uint32_t l2_persist_locks; /* 1: the launch marks the version-lock table (split   */
                              /*    layout) as persisting in L2 (an access-policy      */
                              /*    window on the handle's stream, cleared after the   */
-                             /*    launch; the L2 set-aside stays reserved while the  */
-                             /*    knob is on), so random heap lines streaming from   */
+                             /*    launch; the device-wide L2 set-aside is reference- */
+                             /*    counted per device and released when the last     */
+                             /*    handle using it launches without it or is          */
+                             /*    destroyed), so random heap lines streaming from    */
                              /*    HBM do not evict the locks (EB with a hot set      */
                              /*    larger than L2).  Default 0 (EB: 1)                */
     uint32_t ra_partition;   /* RA: k > 0 = STM thread t addresses only its own words */
@@ -161,6 +164,11 @@ typedef struct {
     int32_t status;              /* GSTM_OK, GSTM_ELOGOVF, GSTM_ETIMEOUT                */
     int32_t mode_used;           /* gstm_mode actually run (AUTO resolved)              */
     int32_t clock_slot;          /* metadata line chosen for g_clock (-1: fixed word)   */
+    uint64_t pipelined_rounds;   /* lock rounds that issued every atom.or at once       */
+                                 /*    (lock_pipeline): only the first  */
+                                 /*    round of an execution may be pipelined, so this  */
+                                 /*    is <= the executions that reached TXCommit's     */
+                                 /*    lock step (Q15, Q37)                             */
 } gstm_stats_t;
 
 /* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */
@@ -273,7 +281,9 @@ int gstm_km_recenter(gstm_t* h);
  * ordered by events.  Consecutive calls on one handle therefore overlap step
  * k+1's copy-in and step k's copy-out with step k's / k+1's transactions
  * (DESIGN.md §7.1).  The first call after a gstm_join / gstm_sync starts
- * after all work already enqueued on the handle's stream.  heap_in must stay
+ * after all work already enqueued on the handle's stream.  Steps may be
+ * chained in place (heap_in of a call overlapping heap_out of the previous
+ * call): that call's copy-in then waits for the previous copy-out.  heap_in must stay
  * valid and heap_out must not be read until gstm_sync (or gstm_join followed
  * by a synchronisation of the handle's stream) returns; the stats of the
  * last launch are in gstm_stats after gstm_sync, the running totals in

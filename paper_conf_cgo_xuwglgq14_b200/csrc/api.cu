@@ -4,6 +4,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <cuda_runtime.h>
 #include "../../include/gstm.h"
 #include "kernels.cuh"
@@ -68,6 +69,10 @@ struct gstm_handle {
     uint32_t* stage_out = nullptr;
     uint64_t stage_words = 0;
     bool pipe_open = false;          // a pipelined call is in flight since the last join
+    const uint32_t* last_out = nullptr;   // heap_out of the last pipelined call (alias check)
+    uint64_t last_out_words = 0;
+    int dev = 0;                     // the device the handle was created on
+    bool l2_user = false;            // counted in g_l2_users[dev] (l2_persist_locks)
     gstm_params_t params{};
     int mode = GSTM_MODE_AUTO;
     // last launch
@@ -81,25 +86,30 @@ struct gstm_handle {
 // access-policy window on the handle's stream covering the lock table,
 // hit property persisting, set around the transaction kernel's launch.
 // The persisting set-aside (cudaLimitPersistingL2CacheSize) is device-wide and
-// outlives the handle that set it: it is released again (limit 0, persisting
-// lines demoted) before any launch that does not use it -- a leftover 64 MiB
-// set-aside cut EB with a 256 MiB lock table from 411 to 170 M tx/s.
-static bool g_l2_set_aside = false;
+// outlives the handle that set it, so it is reference-counted per device: a
+// handle becomes a user at its first persisting launch and stops being one
+// when it launches without persistence or is destroyed; the set-aside is
+// released (limit 0, persisting lines demoted) when the last user stops --
+// a leftover 64 MiB set-aside cut EB with a 256 MiB lock table from 411 to
+// 170 M tx/s -- and never while another handle on the device still uses it.
+static constexpr int kMaxDevices = 64;
+static std::mutex g_l2_mu;
+static int g_l2_users[kMaxDevices];
+static size_t g_l2_limit[kMaxDevices];
 
-static cudaError_t l2_limits(size_t* max_persist, size_t* max_window)
+static cudaError_t l2_limits(int dev, size_t* max_persist, size_t* max_window)
 {
-    static size_t mp = 0, mw = 0;
-    if (!mw) {
-        int dev = 0;
+    static size_t mp[kMaxDevices], mw[kMaxDevices];
+    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    if (!mw[dev]) {
         cudaDeviceProp pr;
-        cudaError_t e = cudaGetDevice(&dev);
-        if (e == cudaSuccess) e = cudaGetDeviceProperties(&pr, dev);
+        cudaError_t e = cudaGetDeviceProperties(&pr, dev);
         if (e != cudaSuccess) return e;
-        mp = pr.persistingL2CacheMaxSize;
-        mw = pr.accessPolicyMaxWindowSize;
+        mp[dev] = pr.persistingL2CacheMaxSize;
+        mw[dev] = pr.accessPolicyMaxWindowSize;
     }
-    *max_persist = mp;
-    *max_window = mw;
+    *max_persist = mp[dev];
+    *max_window = mw[dev];
     return cudaSuccess;
 }
 
@@ -109,16 +119,39 @@ static cudaError_t l2_limits(size_t* max_persist, size_t* max_window)
 static bool l2_persist_fits(const gstm_t* h)
 {
     size_t mp = 0, mw = 0;
-    if (l2_limits(&mp, &mw) != cudaSuccess || !mp || !mw) return false;
+    if (l2_limits(h->dev, &mp, &mw) != cudaSuccess || !mp || !mw) return false;
     return (sizeof(uint32_t) << h->bits) <= std::min(mp, mw);
 }
 
-static cudaError_t release_l2_set_aside()
+// the handle stops using the set-aside; the last user on its device releases it
+static cudaError_t l2_unuse(gstm_t* h)
 {
-    if (!g_l2_set_aside) return cudaSuccess;
-    g_l2_set_aside = false;
+    std::lock_guard<std::mutex> g(g_l2_mu);
+    if (!h->l2_user) return cudaSuccess;
+    h->l2_user = false;
+    if (--g_l2_users[h->dev] > 0) return cudaSuccess;
+    g_l2_users[h->dev] = 0;
+    g_l2_limit[h->dev] = 0;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    if (cur != h->dev) cudaSetDevice(h->dev);
     cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
     if (e == cudaSuccess) e = cudaCtxResetPersistingL2Cache();
+    if (cur != h->dev) cudaSetDevice(cur);
+    return e;
+}
+
+// the handle uses the set-aside: grow the device's limit to what it needs
+static cudaError_t l2_use(gstm_t* h, size_t lim)
+{
+    std::lock_guard<std::mutex> g(g_l2_mu);
+    if (!h->l2_user) {
+        h->l2_user = true;
+        ++g_l2_users[h->dev];
+    }
+    if (lim <= g_l2_limit[h->dev]) return cudaSuccess;
+    cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+    if (e == cudaSuccess) g_l2_limit[h->dev] = lim;
     return e;
 }
 
@@ -128,13 +161,12 @@ static cudaError_t set_l2_lock_window(gstm_t* h, bool on)
     memset(&a, 0, sizeof(a));
     if (on) {
         size_t mp = 0, mw = 0;
-        cudaError_t e = l2_limits(&mp, &mw);
+        cudaError_t e = l2_limits(h->dev, &mp, &mw);
         if (e != cudaSuccess) return e;
         const size_t bytes = std::min(sizeof(uint32_t) << h->bits, mw);
         const size_t lim = std::min(bytes, mp);
-        e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+        e = l2_use(h, lim);
         if (e != cudaSuccess) return e;
-        g_l2_set_aside = true;
         a.accessPolicyWindow.base_ptr = h->locks;
         a.accessPolicyWindow.num_bytes = bytes;
         a.accessPolicyWindow.hitRatio = bytes ? std::min(1.0f, static_cast<float>(lim) / static_cast<float>(bytes)) : 0.f;
@@ -235,6 +267,7 @@ static void fill_stats(gstm_stats_t* out, const unsigned long long* s, double ms
     out->spins = s[S_SPINS];
     out->attempts = s[S_ATTEMPTS];
     out->errors = s[S_ERRORS];
+    out->pipelined_rounds = s[S_PIPELINED];
     out->elapsed_ms = ms;
     const double done = static_cast<double>(out->commits + out->commits_ro);
     out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
@@ -273,6 +306,8 @@ gstm_t* gstm_create_ex(uint64_t heap_words, uint32_t lock_table_bits, uint32_t f
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) { set_error("gstm_create: no CUDA device"); return nullptr; }
     gstm_t* h = new gstm_t();
+    cudaGetDevice(&h->dev);
+    if (h->dev < 0 || h->dev >= kMaxDevices) { set_error("gstm_create: device %d out of range", h->dev); delete h; return nullptr; }
     h->bits = lock_table_bits;
     h->paired = paired;
     h->params = default_params(GSTM_WL_RA);
@@ -341,9 +376,9 @@ uint32_t gstm_flags(const gstm_t* h) { return h && h->paired ? GSTM_CREATE_PAIRE
 
 void gstm_destroy(gstm_t* h)
 {
-    if (h && h->params.l2_persist_locks) release_l2_set_aside();
     if (!h) return;
     if (h->stream) cudaStreamSynchronize(h->stream);
+    l2_unuse(h);
     cudaFree(h->block);
     cudaFree(h->scratch);
     cudaFree(h->tx_stamp);
@@ -652,7 +687,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     }
     const bool persist = P.l2_persist_locks && !h->paired && h->locks && l2_persist_fits(h);
     if (persist) CUDA_TRY(set_l2_lock_window(h, true));
-    else CUDA_TRY(release_l2_set_aside());
+    else CUDA_TRY(l2_unuse(h));
     CUDA_TRY(launch_tx(workload, mode, kp, P.block_threads ? P.block_threads : 256, h->stream));
     if (persist) CUDA_TRY(set_l2_lock_window(h, false));
     CUDA_TRY(launch_finish(h->meta, h->clock, h->stream));
@@ -699,17 +734,17 @@ int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches)
 int gstm_reset_stats_total(gstm_t* h)
 {
     if (!h) { set_error("gstm_reset_stats_total: NULL"); return GSTM_EINVAL; }
-    CUDA_TRY(cudaMemsetAsync(h->meta + M_TOTALS, 0, (M_PHASE + 8 - M_TOTALS) * 8, h->stream));
+    CUDA_TRY(cudaMemsetAsync(h->meta + M_TOTALS, 0, (M_PHASE + kPhaseWords - M_TOTALS) * 8, h->stream));
     return GSTM_OK;
 }
 
 int gstm_phase_cycles(gstm_t* h, uint64_t* out, int n)
 {
     if (!h || !out || n < 0) { set_error("gstm_phase_cycles: bad argument"); return GSTM_EINVAL; }
-    unsigned long long ph[8];
+    unsigned long long ph[kPhaseWords];
     CUDA_TRY(cudaMemcpyAsync(ph, h->meta + M_PHASE, sizeof(ph), cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
-    for (int k = 0; k < n && k < 8; ++k) out[k] = ph[k];
+    for (int k = 0; k < n && k < kPhaseWords; ++k) out[k] = ph[k];
     return GSTM_OK;
 }
 
@@ -779,8 +814,12 @@ int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32
         CUDA_TRY(cudaStreamWaitEvent(h->s_out, h->ev_call, 0));
         h->pipe_open = true;
     }
-    // copy-in: into the staging buffer once the previous step moved it out
+    // copy-in: into the staging buffer once the previous step moved it out;
+    // if heap_in overlaps the previous call's heap_out (steps chained in
+    // place), also after that call's copy-out wrote it
     CUDA_TRY(cudaStreamWaitEvent(h->s_in, h->ev_in_free, 0));
+    if (h->last_out && heap_in < h->last_out + h->last_out_words && h->last_out < heap_in + words)
+        CUDA_TRY(cudaStreamWaitEvent(h->s_in, h->ev_out_free, 0));
     CUDA_TRY(cudaMemcpyAsync(h->stage_in, heap_in, words * 4, cudaMemcpyHostToDevice, h->s_in));
     CUDA_TRY(cudaEventRecord(h->ev_in_ready, h->s_in));
     // the step on the handle's stream: staging -> heap, transactions, heap -> staging
@@ -798,6 +837,8 @@ int gstm_run_host_async(gstm_t* h, int workload, const uint32_t* heap_in, uint32
     CUDA_TRY(cudaStreamWaitEvent(h->s_out, h->ev_out_ready, 0));
     CUDA_TRY(cudaMemcpyAsync(heap_out, h->stage_out, words * 4, cudaMemcpyDeviceToHost, h->s_out));
     CUDA_TRY(cudaEventRecord(h->ev_out_free, h->s_out));
+    h->last_out = heap_out;
+    h->last_out_words = words;
     return GSTM_OK;
 }
 
@@ -807,6 +848,8 @@ int gstm_join(gstm_t* h)
     if (h->pipe_open) {
         CUDA_TRY(cudaStreamWaitEvent(h->stream, h->ev_out_free, 0));
         h->pipe_open = false;
+        h->last_out = nullptr;     // the next call's copy-in follows this join
+        h->last_out_words = 0;
     }
     return GSTM_OK;
 }

@@ -12,10 +12,13 @@ namespace gstm {
 // statistics counters (uint64 each), in the handle's metadata block
 enum {
     S_COMMITS = 0, S_COMMITS_RO, S_AB_OPACITY, S_AB_PREVBV, S_AB_TBV, S_AB_COMMITVBV, S_AB_LOCK,
-    S_LOCK_RETRIES, S_POSTVAL, S_VBV, S_SPINS, S_ATTEMPTS, S_ERRORS, S_NSTATS
+    S_LOCK_RETRIES, S_POSTVAL, S_VBV, S_SPINS, S_ATTEMPTS, S_ERRORS,
+    S_PIPELINED,           // pipelined lock rounds: at most one per execution
+    S_NSTATS
 };
 
 // metadata block layout (uint64 words; hot words on their own 128 B lines)
+static_assert(S_NSTATS <= 29, "the running totals (M_TOTALS + S_NSTATS + 3) must end before M_PHASE");
 enum {
     M_CLOCK = 0,           // g_clock
     M_CLOCK_BEGIN = 16,    // g_clock when the launch started (read-only in kernels)
@@ -29,12 +32,14 @@ enum {
     M_T_LAUNCHES = 96 + S_NSTATS,      // launches since reset
     M_T_NS = 97 + S_NSTATS,            // device ns (globaltimer) since reset
     M_T_ERR = 98 + S_NSTATS,           // OR of the error bits since reset
-    M_PHASE = 112,                     // 8 phase-cycle accumulators (GSTM_PHASE_TIMING builds)
-    M_WORK = 120,                      // next unstarted STM thread (persistent grid), own line
-    M_WORDS = 128,
+    M_PHASE = 128,                     // 16 phase-cycle accumulators (GSTM_PHASE_TIMING builds)
+    M_WORK = 144,                      // next unstarted STM thread (persistent grid), own line
+    M_WORDS = 160,
     // after the 256 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
     M_SEQ = M_WORDS + 256 * 288 + 16,  // STM-VBV global sequence lock, own line
 };
+
+constexpr int kPhaseWords = 16;    // M_PHASE .. M_PHASE + 15
 
 enum { ERR_LOGOVF = 1, ERR_TIMEOUT = 2, ERR_INVALID = 4 };
 

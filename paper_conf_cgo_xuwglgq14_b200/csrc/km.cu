@@ -28,7 +28,7 @@ __global__ void __launch_bounds__(256) km_assign_kernel(const KParams p, uint32_
         wide |= cent[j] >= 4096u;
     }
     // features are < 256: with every centroid word < 4096 a squared distance
-    // fits 32 bits (16 * 4096^2 = 2^28); otherwise the exact 64-bit loop
+    // fits 32 bits (16 * 4096^2 = 2^28); otherwise the exact 128-bit loop
     wide = __syncthreads_or(wide);
     const uint64_t n = p.T * p.K;
     for (uint64_t id = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; id < n; id += uint64_t(gridDim.x) * blockDim.x) {
@@ -52,13 +52,16 @@ __global__ void __launch_bounds__(256) km_assign_kernel(const KParams p, uint32_
                 if (dist < best_d) { best_d = dist; best = c; }    // strict: ties keep the lowest c
             }
         } else {
-            unsigned long long best_d = ~0ull;
+            // any uint32 centroid word: |f - c| < 2^32, its square fits 64
+            // bits unsigned, and 16 squares fit 128 bits -- exact, no wrap
+            unsigned __int128 best_d = ~static_cast<unsigned __int128>(0);
             for (uint32_t c = 0; c < C; ++c) {
                 const uint32_t* cc = cent + c * D;
-                unsigned long long dist = 0;
+                unsigned __int128 dist = 0;
                 for (uint32_t d = 0; d < D; ++d) {
-                    const long long e = static_cast<long long>(f[d]) - static_cast<long long>(cc[d]);
-                    dist += static_cast<unsigned long long>(e * e);
+                    const uint32_t a = static_cast<uint32_t>(f[d]), b = cc[d];
+                    const unsigned long long e = a > b ? static_cast<unsigned long long>(a - b) : static_cast<unsigned long long>(b - a);
+                    dist += static_cast<unsigned __int128>(e * e);
                 }
                 if (dist < best_d) { best_d = dist; best = c; }
             }
@@ -91,14 +94,14 @@ __global__ void km_recenter_kernel(Meta m, uint32_t C, uint32_t D, uint32_t stri
 cudaError_t launch_km_assign(const KParams& kp, uint32_t* cluster, cudaStream_t s)
 {
     const size_t smem = size_t(kp.w.km_clusters) * kp.w.km_dims * 4;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(km_assign_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
     int sms = 148, dev = 0;
     cudaGetDevice(&dev);
+    static bool attr[64];          // the attribute is set once per device
+    if (dev < 0 || dev >= 64 || !attr[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(km_assign_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+        if (e != cudaSuccess) return e;
+        if (dev >= 0 && dev < 64) attr[dev] = true;
+    }
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const uint64_t n = kp.T * kp.K;
     uint64_t grid = std::min<uint64_t>((n + 255) / 256, uint64_t(sms) * 3);   // 3 blocks of 64 KiB per SM

@@ -276,14 +276,16 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         bool got = false;
         // (POL_BACKOFF: only the first, parallel attempt happens here)
         if (act && stage == 1 && (POL != POL_BACKOFF || tries == 0)) {
-            // the pipelined round (§6.4) only for the first round of the first
-            // p.lock_pipeline executions of a transaction: every later round
-            // and execution uses the sequential sorted acquisition.  A lane
-            // starts a new transaction only after committing its current one,
-            // so if nothing commits every lane turns sequential within
-            // p.lock_pipeline lock aborts, and the sorted argument
-            // gives progress: livelock freedom is kept for any finite count.
+            // the pipelined round (§6.4) only for the FIRST round of each of
+            // the first p.lock_pipeline executions of a transaction: every
+            // later round of an execution (tries > 0, counted for any k_lock,
+            // 0 included) is the sequential sorted acquisition.  So at most
+            // one round per execution is pipelined (S_PIPELINED checks it);
+            // a round that follows a failed round is sequential, and among
+            // sequential lanes the holder of the highest contended lock
+            // always progresses (Q15, Q37).
             const bool pipelined = tries == 0 && lock_aborts < p.lock_pipeline;
+            if (pipelined) cnt.inc(S_PIPELINED);
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
             if (r == C_OK) {
                 got = true;
@@ -292,9 +294,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 else tx.writeback(m);
             } else if (r == C_LOCK) {
                 cnt.inc(S_LOCK_RETRIES);                              // l.73-74: retry next iteration
+                // every failed round counts, whatever k_lock is: tries > 0
+                // makes every later round of this execution sequential (Q15,
+                // Q37; k_lock = 0 retries forever, but never pipelined again)
+                tries += (tries != ~0u) ? 1u : 0u;
                 if (POL == POL_BACKOFF) {
                     tries = 1;                                        // -> the sequential step below
-                } else if (p.k_lock && ++tries >= p.k_lock) {
+                } else if (p.k_lock && tries >= p.k_lock) {
                     stage = 0;
                     ++lock_aborts;
                     cnt.inc(S_AB_LOCK);
@@ -653,10 +659,15 @@ __global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
 template <class K>
 inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0)
 {
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
+    // SM count of the CURRENT device (cached per device: one process may
+    // drive handles on several GPUs)
+    static int sms_of[64];
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64) {
+        if (!sms_of[dev]) cudaDeviceGetAttribute(&sms_of[dev], cudaDevAttrMultiProcessorCount, dev);
+        sms = sms_of[dev];
+    } else {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     }
     int per_sm = 0;

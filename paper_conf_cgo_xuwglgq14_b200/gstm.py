@@ -69,7 +69,7 @@ class gstm_stats_t(C.Structure):
         ("attempts", C.c_uint64), ("errors", C.c_uint64), ("clock_begin", C.c_uint64),
         ("clock_end", C.c_uint64), ("elapsed_ms", C.c_double), ("tx_per_s", C.c_double),
         ("abort_ratio", C.c_double), ("status", C.c_int32), ("mode_used", C.c_int32),
-        ("clock_slot", C.c_int32),
+        ("clock_slot", C.c_int32), ("pipelined_rounds", C.c_uint64),
     ]
 
     def as_dict(self) -> dict:

@@ -87,6 +87,37 @@ def test_km_assign_ties_and_wide_centroids():
         assert cnt[7] == 0                                   # never chosen over its twin, row 3
 
 
+def test_km_assign_exact_when_64bit_sum_would_wrap():
+    """The device assignment is the exact argmin for any uint32 centroid word
+    (DESIGN.md §3.4): per point, a row whose squared distance (~2^64) wraps
+    modulo 2^64 to a small number must lose to a row at distance 9e6."""
+    import math
+    T, K, Cn, D = 64, 1, 128, 16
+    g, gp, op, init = U.make("km", T, K, 16, mode="hv", km_clusters=Cn, km_dims=D, km_assign=1)
+    feats = g.dump_descr("km", T, K, 21)[:, 1:D + 1].astype(np.int64)
+    cent = np.full((Cn, D), 0xFFFFFFFF, dtype=np.uint64)
+    want = np.zeros(Cn, dtype=np.int64)
+    for t in range(T):
+        f = [int(x) for x in feats[t]]
+        wrap = list(f)
+        wrap[0] = 0xFFFFFFFF
+        wrap[1] = f[1] + math.isqrt((1 << 33) * (1 + f[0]) - (1 + f[0]) ** 2) + 1
+        near = list(f)
+        near[0] += 3000
+        cent[2 * t], cent[2 * t + 1] = wrap, near
+        d_wrap = sum((a - b) ** 2 for a, b in zip(f, wrap))
+        assert d_wrap % (1 << 64) < 3000 ** 2 < d_wrap
+        exact = [sum((a - int(b)) ** 2 for a, b in zip(f, row)) for row in cent.tolist()]
+        want[int(np.argmin(exact))] += 1
+    assert want[1::2].sum() == T                    # every point's nearest is a "near" row
+    heap = init.copy()
+    c0 = O.km_centroids(op)
+    heap[c0:c0 + Cn * D] = cent.astype(np.uint32).reshape(-1)
+    g.write_heap(heap)
+    st, after, *_ = U.run_verified(g, "km", op, heap, T, K, 21)
+    assert (after[:Cn * (D + 1)].reshape(Cn, D + 1)[:, 0] == want).all()
+
+
 def test_km_recenter_needs_assign():
     g, gp, op, init = U.make("km", 64, 1, 10)
     with pytest.raises(G.GstmError):

@@ -318,6 +318,28 @@ def test_livelock_freedom_two_words(mode, k_lock, pipeline):
     assert st.commits == T * K
 
 
+@pytest.mark.parametrize("paired", [False, True])
+@pytest.mark.parametrize("mode", ["hv", "tbv"])
+@pytest.mark.parametrize("pipeline", [1, 1000])
+def test_pipelined_at_most_one_round_per_execution(paired, mode, pipeline):
+    """k_lock = 0 (Algorithm 3 verbatim: retry the lock step forever) with the
+    pipelined first round (Q37): only the FIRST round of an
+    execution may issue all its atom.or at once -- a round after a failed
+    round must be the sequential sorted acquisition, else two transactions
+    that each win one of {w0, w1} can fail each other forever.
+    16 warps, every transaction takes both words in random order."""
+    T, K = 512, 8
+    g, gp, op, init = U.make("ra", T, K, 1 if paired else 10, mode=mode, paired=paired, n_reads=2, n_writes=2,
+                             n_words=2, k_lock=0, lock_pipeline=pipeline)
+    st, *_ = U.run_verified(g, "ra", op, init, T, K, 4)
+    assert st.commits == T * K
+    assert st.aborts_lock == 0                      # k_lock = 0 never gives up a lock step
+    assert st.lock_retries > 0, "no lock contention: the test exercises nothing"
+    reached_lock_step = st.commits + st.aborts_prevbv + st.aborts_tbv + st.aborts_commit_vbv + st.aborts_lock
+    assert 0 < st.pipelined_rounds <= reached_lock_step, st.as_dict()
+    g.close()
+
+
 @pytest.mark.parametrize("mode", ["hv", "tbv", "cgl", "fgl"])
 @pytest.mark.parametrize("wl,kw,T,K,cap", [
     ("bank", dict(n_words=1 << 12), 1 << 16, 3, 2048),
@@ -370,6 +392,35 @@ def test_l2_persisting_lock_table_replay(mode, persist):
     st, heap, *_ = U.run_verified(g, "eb", op, init, T, K, 29)
     g.set_params(gp)
     U.run_verified(g, "eb", op, heap, T, K, 30)
+
+
+def test_l2_set_aside_is_reference_counted_per_device():
+    """The persisting-L2 set-aside is device-wide: a handle launching WITHOUT
+    persistence must not release the set-aside another live handle uses; the
+    last user's destroy releases it (api.cu l2_use / l2_unuse)."""
+    rt = pytest.importorskip("cuda.bindings.runtime")
+    import gc
+    import torch
+    torch.cuda.init()
+    gc.collect()                                # handles of earlier tests release their set-aside
+
+    def limit():
+        err, v = rt.cudaDeviceGetLimit(rt.cudaLimit.cudaLimitPersistingL2CacheSize)
+        assert err == rt.cudaError_t.cudaSuccess
+        return v
+
+    T, K, H = 1 << 12, 2, 1 << 20
+    a, _, opa, inita = U.make("eb", T, K, 20, mode="hv", n_words=H, n_accesses=8, heap_words=H, l2_persist_locks=1)
+    b, _, opb, initb = U.make("eb", T, K, 20, mode="hv", n_words=H, n_accesses=8, heap_words=H, l2_persist_locks=0)
+    U.run_verified(a, "eb", opa, inita, T, K, 1)
+    held = limit()
+    assert held >= 4 << 20                      # the 2^20-lock table (4 MiB) is set aside
+    U.run_verified(b, "eb", opb, initb, T, K, 2)
+    assert limit() == held                      # b does not release a's set-aside
+    b.close()
+    assert limit() == held
+    a.close()
+    assert limit() == 0                         # the last user released it
 
 
 @pytest.mark.parametrize("paired", [False, True])
@@ -574,6 +625,27 @@ def test_run_host_async_pipelined_one_handle(paired):
     out = np.zeros(N, dtype=np.uint32)
     g.run_host("ra", ins[0], out, T, K, 40)
     assert (out == outs[0]).all()
+
+
+@pytest.mark.parametrize("paired", [False, True])
+def test_run_host_async_chained_in_place(paired):
+    """Steps chained in place: every call passes the SAME pinned buffer as
+    heap_in and heap_out, so step k+1 must read step k's output (its copy-in
+    waits for step k's copy-out).  Disjoint access sets make each step's result
+    unique: after n steps the buffer equals n serial oracle steps, bit for bit."""
+    import torch
+    k_part, T, K, n = 8, 2048, 4, 6
+    N = T * k_part
+    g, gp, op, init = U.make("ra", T, K, 14, mode="hv", paired=paired, n_reads=4, n_writes=4, n_words=N,
+                             ra_partition=k_part)
+    rng = np.random.default_rng(17)
+    buf = torch.from_numpy(rng.integers(0, 2**32, N, dtype=np.uint32).view(np.int32)).pin_memory().numpy().view(np.uint32)
+    want = buf.copy()
+    for k in range(n):
+        g.run_host_async("ra", buf, buf, T, K, 60 + k)
+        O.serial(op, want, T, K, 60 + k)
+    assert g.sync() == 0
+    assert (buf == want).all()
 
 
 @pytest.mark.parametrize("kind", [0, 1, 2, 3, 4, 5])

@@ -619,6 +619,37 @@ def test_km_nearest_is_brute_force_argmin(Cn, D):
         assert O.km_nearest(p, heap, cent[1]) == 1
 
 
+def _wrapping_row(f, D):
+    """A centroid row whose exact squared distance to f is ~2^64 but whose
+    sum taken mod 2^64 is small: (2^32-1-f0)^2 = 2^64 - 2^33(1+f0) + (1+f0)^2,
+    and dim 1 adds back just over 2^33(1+f0)."""
+    import math
+    row = [int(x) for x in f]
+    row[0] = 0xFFFFFFFF
+    need = (1 << 33) * (1 + int(f[0])) - (1 + int(f[0])) ** 2
+    row[1] = int(f[1]) + math.isqrt(need) + 1
+    return row
+
+
+def test_km_nearest_exact_for_wide_uint32_centroids():
+    """The assignment is the exact argmin of the integer squared distance
+     for ANY uint32 centroid word: a row whose distance wraps
+    modulo 2^64 to a small number must not win (Python big integers are the
+    brute force)."""
+    D, Cn = 16, 4
+    p = O.params("km", km_clusters=Cn, km_dims=D, km_assign=1)
+    rng = np.random.default_rng(9)
+    for _ in range(50):
+        f = rng.integers(0, 256, D)
+        rows = [_wrapping_row(f, D), [int(x) + (3000 if d == 0 else 0) for d, x in enumerate(f)],
+                [0xFFFFFFFF] * D, [int(x) for x in rng.integers(0, 1 << 32, D, dtype=np.uint64)]]
+        exact = [sum((int(a) - int(b)) ** 2 for a, b in zip(f, r)) for r in rows]
+        assert exact[0] % (1 << 64) < exact[1] < exact[0]   # a 64-bit sum would pick row 0
+        heap = np.zeros(O.footprint(p, 1, 1), dtype=np.uint32)
+        heap[O.km_centroids(p):] = np.array(rows, dtype=np.uint64).astype(np.uint32).reshape(-1)
+        assert O.km_nearest(p, heap, f.astype(np.uint32)) == int(np.argmin(exact)) == 1
+
+
 def test_km_init_centroids_and_footprint():
     p = O.params("km", km_clusters=8, km_dims=4, km_stride=8, km_assign=1)
     assert O.km_centroids(p) == 64 and O.footprint(p, 3, 3) == 64 + 32
