@@ -6,23 +6,27 @@ One "step" = one gstm_launch of the whole hot path (TXBegin / TXRead /
 TXWrite / TXCommit of every transaction) over one batch of synthetic input:
 BASELINE configs[1], bank transfer, 2^20 accounts, 2^20 STM threads x 16
 transactions (16M transactions), 2^20 version locks.  Headline variant:
-STM-HV on the paired layout; the paper's
-STM-Optimized (AUTO) on the paper's split layout, the other STM variants, FGL
-and CGL are reported in the same line.  The heap is resident in HBM before
-the timed region; L2 is flushed (256 MiB write) between timed steps.
+STM-HV on the paired layout.  The heap is resident in
+HBM before the timed region; L2 is flushed (256 MiB write) between timed
+steps.
+
+The same JSON line carries, per BASELINE config (RA configs[0], HT
+configs[2], two EB configs[3] points, KM configs[4]): the STM rate and abort
+ratio, the CGL and FGL rates at that config, speedup_vs_cgl, and the fraction
+of the config's measured op-mix roof.  The long tables (the
+bank variant table, CGL probes, roof sweeps) go to stderr as one JSON object.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
 
-N > 1 (torchrun, one rank per GPU): key-partitioned bank -- every rank owns
-its own 2^20 accounts and runs shard-local transfers (weak scaling); NCCL is
-used once, after timing, to reduce the stats and the balance invariant.
+N > 1: one rank per GPU (the driver launches torchrun; without WORLD_SIZE in
+the environment bench.py re-launches itself under torch.distributed.run):
+key-partitioned bank -- every rank owns its own 2^20 accounts and runs
+shard-local transfers (weak scaling); NCCL is used once, after timing, to
+reduce the stats and the balance invariant.
 
 --workload ht: the key-partitioned hash table of SURVEY §8e (BASELINE
-configs[2] shape per GPU: 2^20 buckets, 2^22 STM threads x 4 operations,
-90/10 lookup/insert, keys in [1, 2^22]); rank g of N = 2^b owns the keys whose
-mix64 top b bits are g, so every transaction is shard-local; the table is
-re-initialised (outside the timed brackets) before every step; after timing,
-one all-reduce checks that the tables hold exactly the inserted keys.
+configs[2] shape per GPU); rank g of N = 2^b owns the keys whose mix64 top b
+bits are g.
 
 Prints ONE JSON line on rank 0.
 """
@@ -31,6 +35,8 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import socket
+import statistics
 import subprocess
 import sys
 import time
@@ -45,6 +51,7 @@ THREADS = 1 << 20
 TX_PER_THREAD = 16
 BITS = 20
 SEED = 20140215
+SMS = 148
 
 
 def parse(argv=None):
@@ -62,10 +69,16 @@ def parse(argv=None):
                     help="re-reads of a locked word before the transaction re-executes")
     ap.add_argument("--threads", type=int, default=THREADS)
     ap.add_argument("--tx-per-thread", type=int, default=TX_PER_THREAD)
-    ap.add_argument("--no-cgl", action="store_true", help="skip the CGL/FGL baselines and the variant table")
+    ap.add_argument("--no-cgl", action="store_true", help="skip the bank CGL/FGL baselines and the variant table")
+    ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs")
+    ap.add_argument("--only-configs", default="", help="comma list of config names to run (default: all)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--workload", default="bank", choices=["bank", "ht"],
                     help="bank (BASELINE configs[1], the headline) or the key-partitioned hash table")
+    ap.add_argument("--host-selftest", action="store_true",
+                    help="CPU-only check of the multi-rank host logic (gloo, no GPU, fake device steps); "
+                         "its line says selftest and is never a measurement")
+    ap.add_argument("--cpu-oracle-leg", default=None, help=argparse.SUPPRESS)
     return ap.parse_args(argv)
 
 
@@ -86,6 +99,23 @@ def reduce_over_ranks(stats_vec, balance, t_ms, wall, world, dist, device):
         dist.all_reduce(vec, op=dist.ReduceOp.SUM)
         dist.all_reduce(tm, op=dist.ReduceOp.MAX)
     return vec.cpu().numpy(), tm.cpu().tolist()
+
+
+def free_port() -> int:
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def self_launch(args) -> int:
+    """--gpus N > 1 without a torchrun environment: re-launch this script as
+    N ranks under torch.distributed.run (one process per GPU) and pass its
+    output through, so `python bench.py --gpus N` really runs N ranks."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 class Variant:
@@ -113,22 +143,6 @@ class Variant:
         g.init_heap("bank")
         return g
 
-    # Algorithmic L2 requests of one committed bank transaction (Algorithm 3
-    # on the bank body, verify off); every request touches
-    # one 32 B sector of a random word (or word pair).
-    def ops(self, mode_used: str):
-        if self.layout == "paired":
-            upd = {"ld": 2, "atom": 2, "st": 2}      # 2 pair loads; 2 atom.or.b64 (lock + value); 2 pair stores
-            ro = {"ld": 2, "atom": 0, "st": 0}
-            if mode_used in ("hv", "hv_backoff") and self.prelock:
-                upd = dict(upd, ld=4)
-        else:
-            upd = {"ld": 4, "atom": 2, "st": 4}      # 2 values + 2 lock words; 2 atom.or; 2 write-back + 2 release
-            ro = {"ld": 4, "atom": 0, "st": 0}
-            if mode_used in ("hv", "hv_backoff") and self.prelock:
-                upd = dict(upd, ld=6)                 # + pre-lock VBV of the 2 values (A3.l71)
-        return upd, ro
-
 
 def headline_variant(args) -> Variant:
     # k_lock = 1: a transaction that loses a lock round re-executes with fresh
@@ -140,7 +154,8 @@ def headline_variant(args) -> Variant:
     return Variant(args.mode, args.layout, args.prelock, k_lock=args.k_lock, spin_cap=args.spin_cap)
 
 
-def config(args, label="hv/paired"):
+def config(args):
+    """The workload of the line (identical in both arms: no implementation keys)."""
     return {
         "workload": "bank transfer (BASELINE configs[1]): 2-account transfer tx, total-balance invariant",
         "accounts_per_gpu": ACCOUNTS,
@@ -148,43 +163,90 @@ def config(args, label="hv/paired"):
         "tx_per_thread": args.tx_per_thread,
         "tx_per_step_per_gpu": args.threads * args.tx_per_thread,
         "lock_table_bits": BITS,
-        "variant": label,
         "partition": "key-partitioned shards, shard-local transfers" if args.gpus > 1 else "single shard",
         "l2": "flushed (256 MiB write) between timed steps",
     }
 
 
 # ---------------------------------------------------------------------------
-# reference arm: the CPU oracle as it stands (serial executor), rank 0 only
+# CPU oracle legs (the only places bench.py executes oracle/)
 # ---------------------------------------------------------------------------
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def cpu_oracle_leg(spec: str) -> int:
+    """Child process (pinned by its parent with taskset -c 0): time the
+    serial oracle over `reps` full bank steps; print the seconds per rep."""
+    T, K, seed, reps = (int(x) for x in spec.split(","))
+    import oracle as O
+    p = O.params("bank", n_words=ACCOUNTS)
+    times = []
+    for r in range(reps):
+        heap = O.init_heap(p, ACCOUNTS)
+        t0 = time.perf_counter()
+        O.serial(p, heap, T, K, seed + r)
+        times.append(time.perf_counter() - t0)
+    print(json.dumps({"times_s": times, "affinity": sorted(os.sched_getaffinity(0))}), flush=True)
+    return 0
+
+
+def cpu_baseline(T, K, seed, reps=5):
+    """The serial oracle (oracle/serial.c or_serial, gcc -O2, one thread) over
+    the full step (T x K bank transfers), pinned to core 0 with taskset,
+    median of `reps` runs; the box's core count and CPU model recorded."""
+    leg = [sys.executable, os.path.abspath(__file__), "--cpu-oracle-leg", f"{T},{K},{seed},{reps}"]
+    pinned = subprocess.run(["taskset", "-c", "0"] + leg, capture_output=True, text=True)
+    how = "taskset -c 0"
+    if pinned.returncode != 0:
+        pinned = subprocess.run(leg, capture_output=True, text=True)
+        how = "unpinned (taskset unavailable)"
+    out = json.loads(pinned.stdout.strip().splitlines()[-1])
+    med = statistics.median(out["times_s"])
+    return {"value": T * K / med, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread, {how}) over one full step: "
+                      f"{T} threads x {K} tx = {T * K} bank transfers; median of {reps} runs "
+                      f"({min(out['times_s']):.3f}-{max(out['times_s']):.3f} s)",
+            "host_cores": os.cpu_count(), "cpu_model": cpu_model(), "affinity": out["affinity"]}
+
+
 def run_reference(args):
+    """Reference arm of this tier: the CPU oracle as it stands, on the SAME
+    workload as the native line (2^20 threads x 16 = 16.8M transfers per
+    step), rank 0 only."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
     import oracle as O
 
     p = O.params("bank", n_words=ACCOUNTS)
-    sample_threads = min(args.threads, 1 << 18)          # bounded sample: 4M tx per step
-    K = args.tx_per_thread
-    heap = O.init_heap(p, ACCOUNTS)
-    if args.warmup > 0:
-        O.serial(p, heap.copy(), sample_threads // 16, K, SEED)
+    T, K = args.threads, args.tx_per_thread
+    for w in range(args.warmup):
+        O.serial(p, O.init_heap(p, ACCOUNTS), max(1, T // 64), K, SEED + 100000 + w)
     times = []
-    n = sample_threads * K
     for s in range(args.steps):
+        heap = O.init_heap(p, ACCOUNTS)
         t0 = time.perf_counter()
-        O.serial(p, heap, sample_threads, K, SEED + s)
+        O.serial(p, heap, T, K, SEED + s)
         times.append(time.perf_counter() - t0)
     tot = sum(times)
-    val = n * args.steps / tot
+    val = T * K * args.steps / tot
     line = {
         "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
-        "data": "synthetic", "config": config(args, "serial CPU oracle"),
+        "data": "synthetic", "config": config(args), "variant": "serial CPU oracle",
         "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread) over "
-                                   f"{sample_threads} threads x {K} tx = {n} bank transfers per step"},
+                         "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread) over the full "
+                                   f"step: {T} threads x {K} tx = {T * K} bank transfers per step",
+                         "host_cores": os.cpu_count(), "cpu_model": cpu_model()},
         "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -240,33 +302,35 @@ def measured_peaks():
 
 
 KEYS = ["commits", "commits_ro", "aborts", "aborts_opacity", "aborts_prevbv", "aborts_tbv", "aborts_commit_vbv",
-        "aborts_lock", "lock_retries", "postvalidations", "vbv_runs", "spins", "attempts", "errors"]
+        "aborts_lock", "lock_retries", "postvalidations", "vbv_runs", "spins", "attempts", "errors",
+        "reads_update", "reads_ro", "writes_update", "locks_update", "pipelined_rounds"]
+NVEC = len(KEYS) + 1
 
 
 def stats_vector(st):
     import numpy as np
-    v = np.zeros(16, dtype=np.float64)
+    v = np.zeros(NVEC, dtype=np.float64)
     for i, k in enumerate(KEYS):
-        v[i] = getattr(st, k)
-    v[14] = st.elapsed_ms
+        v[i] = st[k] if isinstance(st, dict) else getattr(st, k)
+    v[len(KEYS)] = st["elapsed_ms"] if isinstance(st, dict) else st.elapsed_ms
     return v
 
 
 def from_vector(v):
     d = {k: float(v[i]) for i, k in enumerate(KEYS)}
-    d["lib_elapsed_ms"] = float(v[14])
+    d["lib_elapsed_ms"] = float(v[len(KEYS)])
     return d
 
 
-def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None, wl="bank"):
+def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None, wl="bank", reinit=False):
     """W warm-up launches, then `steps` launches enqueued back to back (no
     host sync), each bracketed by CUDA events on the launching stream, the L2
-    flush outside the brackets.  Returns (step ms list, summed stats, wall s,
-    clocks)."""
+    flush (and, for HT, the table re-initialisation) outside the brackets.
+    Returns (step ms list, summed stats, wall s, clocks)."""
     import torch
     for w in range(warmup):
-        if wl == "ht":
-            g.init_heap("ht")
+        if reinit:
+            g.init_heap(wl)
         g.launch(wl, T, K, seed0 + 100000 + w)
     torch.cuda.synchronize()
     g.reset_stats_total()
@@ -278,8 +342,8 @@ def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None, 
     wall0 = time.perf_counter()
     for k in range(steps):
         flush.fill_(float(k))
-        if wl == "ht":
-            g.init_heap("ht")      # node ids are per launch: every step starts from an empty table
+        if reinit:
+            g.init_heap(wl)
         e0, e1 = evs[k]
         e0.record(stream)
         g.launch(wl, T, K, seed0 + k)
@@ -292,73 +356,97 @@ def timed_steps(g, stream, flush, T, K, seed0, steps, warmup, sampler_dev=None, 
     return [a.elapsed_time(b) for a, b in evs], st, wall, clocks
 
 
-def roofline(var: Variant, mode_used, tot, t_ms, steps, peaks, peak_src, traffic=None):
-    upd, ro = var.ops(mode_used)
-    b_upd, b_ro = 32 * sum(upd.values()), 32 * sum(ro.values())
-    bytes_per_launch = (tot["commits"] * b_upd + tot["commits_ro"] * b_ro) / steps
-    dur_s = t_ms * 1e-3 / steps
-    achieved = bytes_per_launch / dur_s / 1e9
-    peak = float(peaks.get("hbm_gbs", 6650.0))
-    prof = os.path.join(ROOT, "profiles", "bank_ncu_full.json")
-    if traffic is None and os.path.exists(prof):
-        try:
-            traffic = json.load(open(prof)).get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
-    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": traffic, "kernel": f"stm_kernel<BankWL, MODE_{mode_used.upper()}, "
-                                         f"{'paired' if var.layout == 'paired' else 'split'}>",
-            "algorithmic_bytes_per_launch": bytes_per_launch,
-            "bytes_per_unit": {"update_tx": b_upd, "read_only_tx": b_ro}, "peak_source": peak_src,
-            "note": "each random word (or word+lock pair) access counted as one 32 B sector; launch duration = "
-                    "CUDA events on the launching stream, averaged over the timed steps"}
+# ---------------------------------------------------------------------------
+# rooflines
+# ---------------------------------------------------------------------------
+def pow2_ceil(x: int) -> int:
+    return 1 << max(7, (int(x) - 1).bit_length())
 
 
-def roofline_l2(G, var: Variant, mode_used, tot, t_ms, steps):
-    """L2-atomic roofline: the same PTX operations, measured on this box by
-    gstm_ubench over a table of the heap's size (L2-resident)."""
-    threads = 148 * 2048
-    tbl = 8 << 20 if var.layout == "paired" else 4 << 20
-    A = G.gstm_ubench(0, tbl, 1 << 26, threads)[0]       # random atom.or
-    L = G.gstm_ubench(2, tbl, 1 << 26, threads)[0]       # random ld.relaxed.gpu
-    S = G.gstm_ubench(3, tbl, 1 << 26, threads)[0]       # random st.relaxed.gpu
-    Cl = G.gstm_ubench(5, 256, 1 << 24, threads)[0]      # warp-aggregated clock increments
-    upd, ro = var.ops(mode_used)
-    per = lambda m: m["ld"] / L + m["atom"] / A + m["st"] / S
-    roof_s = (tot["commits"] * (per(upd) + 1.0 / Cl) + tot["commits_ro"] * per(ro)) / steps
-    dur_s = t_ms * 1e-3 / steps
-    done = (tot["commits"] + tot["commits_ro"]) / steps
-    return {"bound": "l2_atomic", "frac": roof_s / dur_s, "roof_tx_per_s": done / roof_s,
-            "achieved_tx_per_s": done / dur_s,
-            "peaks_ops_per_s": {"atom_or_random": A, "ld_relaxed_random": L, "st_relaxed_random": S,
-                                "clock_increments_warp_aggregated": Cl, "table_bytes": tbl},
-            "ops_per_update_tx": dict(upd, clock=1), "ops_per_read_only_tx": ro,
-            "model": "time = sum over op classes of count / measured rate (one shared L2 request pipeline)"}
+def class_peaks(G, table_bytes: int, paired: bool, threads: int = SMS * 2048):
+    """Per-op-class L2 rates (gstm_ubench, same PTX ops, random addresses over
+    a table of the footprint's size): the denominators of SURVEY §8(d)'s
+    max formula."""
+    tb = min(pow2_ceil(table_bytes), 1 << 30)
+    k_ld, k_atom, k_st = (7, 6, 8) if paired else (2, 0, 3)
+    return {"ld": G.gstm_ubench(k_ld, tb, 1 << 26, threads)[0],
+            "atom": G.gstm_ubench(k_atom, tb, 1 << 26, threads)[0],
+            "st": G.gstm_ubench(k_st, tb, 1 << 26, threads)[0],
+            "clock": G.gstm_ubench(5, 256, 1 << 24, threads)[0],
+            "table_bytes": tb}
 
 
-def cgl_baseline(G, stream, T, seed, mode="cgl"):
+def op_mix_roof(G, R, stream, wl, st, mode, prelock, pipelined, words, bits, paired, T,
+                records=None, n_tx=1 << 22, warps=(4, 8, 16, 32, 64)):
+    """The measured op-mix roof of the committed transactions of `st`: max over
+    occupancies of gstm_ubench_mix on a scratch handle of the same layout and
+    size (its g_clock line probed like the measured handle's)."""
+    prog = R.programs_from_stats(wl, st, paired, mode, prelock, pipelined, records)
+    h = G.Gstm(words, bits, paired=paired)
+    h.set_stream(stream)
+    sweep = {}
+    if records:                 # one thread per record: each record's transactions form one serial chain
+        block = 256 if records[0] % 256 == 0 else 32
+        occ = [max(block, records[0] // block * block)]
+    else:
+        block = 256
+        occ = sorted({max(256, min(SMS * 32 * w, T) // 256 * 256) for w in warps})
+    for th in occ:
+        tps, _ = G.gstm_ubench_mix(h.h, words, prog, max(n_tx, th), th, block)
+        sweep[th] = tps
+    h.close()
+    best = max(sweep, key=sweep.get)
+    return {"roof_tx_per_s": sweep[best], "threads": best, "sweep": {str(k): v for k, v in sweep.items()},
+            "ops_per_tx": R.op_counts(prog), "round_trips_per_tx": R.round_trips(prog), "program": prog}
+
+
+def max_formula(ops: dict, peaks: dict) -> float:
+    """roof_tx/s = 1 / max_i(cost_i / peak_i)."""
+    return 1.0 / max(ops[c] / peaks[c] for c in ("ld", "atom", "st", "clock") if ops[c] > 0)
+
+
+def roofline_object(achieved_tx_s, roof, maxf, sectors_per_tx, note):
+    """The contract's roofline object.  bound "l2": the path is a chain of
+    random L2 round trips over an L2-resident footprint (DESIGN.md §7.2);
+    achieved and peak are algorithmic L2 sector bytes per second (32 B per
+    random access of the committed transactions' own op mix), so frac =
+    achieved tx/s / measured op-mix roof tx/s."""
+    b = 32.0 * sectors_per_tx
+    return {"bound": "l2", "achieved": achieved_tx_s * b / 1e9, "peak": roof["roof_tx_per_s"] * b / 1e9,
+            "unit": "GB/s", "frac": achieved_tx_s / roof["roof_tx_per_s"], "traffic": None,
+            "roof_tx_per_s": roof["roof_tx_per_s"], "roof_threads": roof["threads"],
+            "roof_source": "measured: gstm_ubench_mix (the committed transactions' exact op mix, no conflicts, "
+                           "max over occupancy)",
+            "max_formula_tx_per_s": maxf, "frac_max_formula": achieved_tx_s / maxf,
+            "bytes_per_tx": b, "round_trips_per_tx": roof["round_trips_per_tx"], "note": note}
+
+
+# ---------------------------------------------------------------------------
+# baselines
+# ---------------------------------------------------------------------------
+def cgl_rate(G, make_handle, wl, T, K, seed, budget_s=0.4, reinit=False, mode="cgl"):
     """CGL serialises every transaction, so its rate depends on how many
     threads fight for the one lock, not on the batch size.  Probe the paper's
     Scheme #3 (backoff 0) and test-and-test-and-set with exponential backoff
-    at several thread counts and divide by the FASTEST (the most favourable
-    baseline), then time it on a bounded sample of ~0.5 s.  mode="vbv": the
-    same for STM-VBV, whose writers are serialised by one sequence lock
-    (backoff does not apply)."""
-    g = Variant(mode).handle(G, stream)
+    at 1 warp per SM and at T threads, take the FASTEST (the most favourable
+    baseline), then time it on a bounded sample of ~budget_s."""
+    g = make_handle(mode)
     probes = {}
-    for Tc in (148 * 32, 1 << 14, 1 << 16, 1 << 18):
+    for Tc in sorted({min(T, SMS * 32), min(T, 1 << 14)} | ({T} if T <= 1 << 16 else set())):
         for bo in ((0, 256) if mode == "cgl" else (0,)):
             g.set_params(backoff_ns=bo)
-            probes[(Tc, bo)] = g.run("bank", Tc, max(1, (1 << 14) // Tc), seed + 11 + bo).tx_per_s
+            if reinit:
+                g.init_heap(wl)
+            probes[(Tc, bo)] = g.run(wl, Tc, max(1, min(K, (1 << 12) // Tc)), seed + 11 + bo).tx_per_s
     (Tc, bo) = max(probes, key=probes.get)
     g.set_params(backoff_ns=bo)
-    Kc = max(1, int(probes[(Tc, bo)] * 0.5) // Tc)
-    st = g.run("bank", Tc, Kc, seed + 12)
+    Kc = max(1, min(K, int(probes[(Tc, bo)] * budget_s) // Tc))
+    if reinit:
+        g.init_heap(wl)
+    st = g.run(wl, Tc, Kc, seed + 12)
     g.close()
-    return {"value": st.tx_per_s, "unit": UNIT, "threads": Tc, "tx_per_thread": Kc, "backoff_ns": bo,
-            "probe_tx_per_s": {f"T={k[0]},backoff={k[1]}": v for k, v in probes.items()},
-            "sample": f"{Tc} threads x {Kc} tx at the fastest probed CGL configuration",
-            "elapsed_ms": st.elapsed_ms, "abort_ratio": st.abort_ratio, "kernel": f"{mode}_kernel<BankWL>"}
+    return {"value": st.tx_per_s, "threads": Tc, "tx_per_thread": Kc, "backoff_ns": bo,
+            "abort_ratio": st.abort_ratio, "probe_tx_per_s": {f"T={k[0]},backoff={k[1]}": v for k, v in probes.items()}}
 
 
 def variant_table(G, stream, flush, T, K, seed, variants, steps=8, warmup=3):
@@ -368,29 +456,123 @@ def variant_table(G, stream, flush, T, K, seed, variants, steps=8, warmup=3):
         g = var.handle(G, stream)
         ms, st, _, _ = timed_steps(g, stream, flush, T, K, seed, steps, warmup)
         done = st.commits + st.commits_ro
-        out[var.name] = {"value": done / (sum(ms) * 1e-3), "unit": UNIT, "ms_per_step": sum(ms) / steps,
-                         "abort_ratio": st.aborts / max(1, st.aborts + done),
-                         "mode_used": G.MODE_NAMES[st.mode_used]}
+        out[var.name] = {"value": done / (sum(ms) * 1e-3), "ms_per_step": sum(ms) / steps,
+                         "abort_ratio": st.aborts / max(1, st.aborts + done), "mode_used": G.MODE_NAMES[st.mode_used]}
         g.close()
         torch.cuda.synchronize()
     return out
 
 
-def cpu_baseline(T, K, seed):
-    import oracle as O
-    p = O.params("bank", n_words=ACCOUNTS)
-    heap = O.init_heap(p, ACCOUNTS)
-    t0 = time.perf_counter()
-    O.serial(p, heap, T, K, seed)
-    dt = time.perf_counter() - t0
-    return {"value": T * K / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread) over one full step: "
-                      f"{T} threads x {K} tx = {T * K} bank transfers, {dt:.2f} s"}
+# ---------------------------------------------------------------------------
+# the other BASELINE configs (RA, HT, EB, KM): STM vs CGL vs FGL + op-mix roof
+# ---------------------------------------------------------------------------
+HT_BUCKETS, HT_THREADS, HT_K, HT_KEYS, HT_BITS = 1 << 20, 1 << 22, 4, 1 << 22, 22
+
+CONFIGS = {
+    # name: (workload, heap words, lock bits, params, T, K, steps, note)
+    "ra_c0": ("ra", 1024, 10, dict(n_reads=4, n_writes=4, n_words=1024), 256, 1024, 3,
+              "BASELINE configs[0]: random array, 1K words, 256 threads, 4R+4W, 2^10 locks"),
+    "ht_c2": ("ht", HT_BUCKETS + 2 * HT_THREADS * HT_K, HT_BITS,
+              dict(ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90), HT_THREADS, HT_K, 5,
+              "BASELINE configs[2]: chained hash table, 2^20 buckets, 2^22 threads x 4, 90/10 lookup/insert, "
+              "keys in [1, 2^22], 2^22 locks; table re-initialised before every step"),
+    "eb_c3_h26_a16": ("eb", 1 << 26, 24, dict(n_words=1 << 26, n_accesses=16), 1 << 18, 16, 5,
+                      "BASELINE configs[3]: EigenBench-style, 2^26-word heap = hot set, 16 accesses (8R/8W), "
+                      "2^24 locks (persisting in L2), 2^18 threads x 16"),
+    "eb_c3_h10_a64": ("eb", 1 << 10, 10, dict(n_words=1 << 10, n_accesses=64), 4096, 4, 1,
+                      "BASELINE configs[3] high-contention corner: hot set 2^10 words, 64 accesses (32R/32W), "
+                      "2^10 locks, 4096 STM threads x 4; STM concurrency probed (max_threads) like CGL's"),
+    "km_c4": ("km", 1024 * 17, 20, dict(km_clusters=1024, km_dims=16), 1 << 24, 1, 1,
+              "BASELINE configs[4]: k-means cluster update, 16M points, 1024 centroids x 16 dims, record = 17 "
+              "words, 2^20 locks"),
+}
+
+
+def first_round_pipelined(wl, gp, st) -> bool:
+    """Does the kernel issue a transaction's first lock round all at once
+    ?  Register logs (bank) always may; local-memory logs only
+    when the lock log fits one 8-atomic chunk (Q36)."""
+    if gp.lock_pipeline == 0:
+        return False
+    if wl == "bank":
+        return True
+    return st.commits > 0 and st.locks_update / st.commits <= 8
+
+
+def run_config(G, R, stream, flush, name, seed):
+    import torch
+    wl, words, bits, kw, T, K, steps, note = CONFIGS[name]
+    reinit = wl == "ht"
+    out = {"workload": note}
+
+    def make(mode, **extra):
+        g = G.Gstm(words, bits)
+        g.set_workload_defaults(wl, **kw, **extra)
+        g.set_mode(mode)
+        g.set_stream(stream)
+        g.init_heap(wl)
+        return g
+
+    extra = {}
+    if name == "eb_c3_h10_a64":
+        # the contention corner: every pair of transactions conflicts, so
+        # concurrency is a conflict knob; probe it like CGL's thread count
+        probes = {}
+        for cap in (32, 128, 512, 2048, 4096):
+            g = make("hv", max_threads=cap)
+            probes[cap] = g.run(wl, T, 1, seed + 5).tx_per_s
+            g.close()
+        extra["max_threads"] = max(probes, key=probes.get)
+        out["stm_concurrency_probe"] = probes
+    res = {}
+    for mode in ("hv", "tbv", "fgl"):
+        g = make(mode, **(extra if mode != "fgl" else {}))
+        ms, st, _, _ = timed_steps(g, stream, flush, T, K, seed, steps, 1, wl=wl, reinit=reinit)
+        done = st.commits + st.commits_ro
+        res[mode] = (done / (sum(ms) * 1e-3), st.aborts / max(1, st.aborts + done), st, g.params())
+        g.close()
+        torch.cuda.synchronize()
+    cgl = cgl_rate(G, lambda m: make(m), wl, T, K, seed, reinit=reinit)
+    v, ab, st, gp = res["hv"]
+    out.update({"stm": {"mode": "hv", "value": v, "abort_ratio": ab},
+                "stm_tbv": {"value": res["tbv"][0], "abort_ratio": res["tbv"][1]},
+                "fgl": res["fgl"][0], "cgl": cgl["value"], "speedup_vs_cgl": v / cgl["value"],
+                "threads": T, "tx_per_thread": K, "steps": steps})
+    records = (1024, 17) if wl == "km" else None
+    roof = op_mix_roof(G, R, stream, wl, st, "hv", bool(gp.prelock_vbv), first_round_pipelined(wl, gp, st),
+                       words, bits, False, T, records=records)
+    per_tx = roof["ops_per_tx"]
+    sectors = per_tx["ld"] + per_tx["atom"] + per_tx["st"]
+    peaks = class_peaks(G, words * 4 + (4 << bits), False)
+    out["roof"] = {"roof_tx_per_s": roof["roof_tx_per_s"], "frac": v / roof["roof_tx_per_s"],
+                   "threads": roof["threads"], "round_trips_per_tx": roof["round_trips_per_tx"],
+                   "max_formula_tx_per_s": max_formula(per_tx, peaks),
+                   "kind": "contention: 1024 records, one serial chain each" if records else "op mix, no conflicts"}
+    detail = {"cgl": cgl, "roof": {k: v for k, v in roof.items() if k != "program"}, "class_peaks": peaks,
+              "hv_stats": {k: getattr(st, k) for k in KEYS}}
+    return out, detail
 
 
 # ---------------------------------------------------------------------------
-# native arm
+# native arm (bank headline)
 # ---------------------------------------------------------------------------
+class FakeBankDevice:
+    """--host-selftest: stands in for the GPU step on a CPU-only box so the
+    multi-rank host logic (launch, shard seeds, barrier, the one reduction,
+    the JSON line) can be tested with gloo.  Deterministic fake counts; no
+    oracle, no kernels; the line it produces says "selftest"."""
+
+    def __init__(self, rank):
+        self.rank = rank
+
+    def run(self, args, seed0):
+        n = args.threads * args.tx_per_thread
+        st = {k: 0.0 for k in KEYS}
+        st.update(commits=n - n // 16, commits_ro=n // 16, aborts=n // 10, attempts=n + n // 10,
+                  elapsed_ms=1.0 + self.rank)
+        return [1.0 + 0.5 * self.rank] * args.steps, st, 0.01, None, float(ACCOUNTS * 1000)
+
+
 def run_native(args):
     import numpy as np
     import torch
@@ -400,134 +582,188 @@ def run_native(args):
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     args.gpus = world
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    if args.host_selftest:
+        dev, backend = torch.device("cpu"), "gloo"
+    else:
+        torch.cuda.set_device(local)
+        dev, backend = torch.device("cuda", local), "nccl"
+    comm = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+        comm = {"backend": backend, "nranks": dist.get_world_size()}
 
-    from paper_conf_cgo_xuwglgq14_b200 import build as B
-    if rank == 0 or world == 1:
-        B.build()
-    if world > 1:
-        dist.barrier()
-    from paper_conf_cgo_xuwglgq14_b200 import gstm as G
-
-    T, K = args.threads, args.tx_per_thread
-    # one non-default stream for everything (the library, the L2 flush, the
-    # CUDA events): torch's legacy default stream has handle 0
-    stream = torch.cuda.Stream(device=dev)
-    torch.cuda.set_stream(stream)
-    var = headline_variant(args)
-    g = var.handle(G, stream)
-    flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)    # 256 MiB > 126 MB L2
     seed0 = shard_seed(rank)
-    if world > 1:
-        dist.barrier()
-    step_ms, st_tot, wall, clocks = timed_steps(g, stream, flush, T, K, seed0, args.steps, args.warmup, local)
-    if world > 1:
-        dist.barrier()
+    extra, detail = {}, {}
+    if args.host_selftest:
+        fake = FakeBankDevice(rank)
+        if world > 1:
+            dist.barrier()
+        step_ms, st_tot, wall, clocks, bal = fake.run(args, seed0)
+        if world > 1:
+            dist.barrier()
+        mode_used, var_name, g = "hv", "selftest", None
+    else:
+        from paper_conf_cgo_xuwglgq14_b200 import build as B
+        if rank == 0 or world == 1:
+            B.build()
+        if world > 1:
+            dist.barrier()
+        from paper_conf_cgo_xuwglgq14_b200 import gstm as G
+        from paper_conf_cgo_xuwglgq14_b200 import roofline as R
+
+        T, K = args.threads, args.tx_per_thread
+        # one non-default stream for everything (the library, the L2 flush, the
+        # CUDA events): torch's legacy default stream has handle 0
+        stream = torch.cuda.Stream(device=dev)
+        torch.cuda.set_stream(stream)
+        var = headline_variant(args)
+        var_name = var.name
+        g = var.handle(G, stream)
+        flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)    # 256 MiB > 126 MB L2
+        if world > 1:
+            dist.barrier()
+        step_ms, st, wall, clocks = timed_steps(g, stream, flush, T, K, seed0, args.steps, args.warmup, local)
+        if world > 1:
+            dist.barrier()
+        st_tot = {k: getattr(st, k) for k in KEYS}
+        st_tot["elapsed_ms"] = st.elapsed_ms
+        mode_used = G.MODE_NAMES[st.mode_used]
+        bal = float(g.read_heap().astype(np.int64).sum())
     t_ms = float(sum(step_ms))
-    mode_used = G.MODE_NAMES[st_tot.mode_used]
-    heap = g.read_heap()
-    bal = float(heap.astype(np.int64).sum())
     vec, (t_ms, wall) = reduce_over_ranks(stats_vector(st_tot), bal, t_ms, wall, world, dist, dev)
-    tot = from_vector(vec[:16])
-    balance_ok = int(vec[16]) == world * ACCOUNTS * 1000
-
-    extra = {}
-    if rank == 0:
-        # e2e through the C ABI with HOST buffers (H2D + launch + D2H timed)
-        pin_in = torch.full((ACCOUNTS,), 1000, dtype=torch.int32).pin_memory()
-        pin_out = torch.empty(ACCOUNTS, dtype=torch.int32).pin_memory()
-        h_in = pin_in.numpy().view(np.uint32)
-        h_out = pin_out.numpy().view(np.uint32)
-        # e2e through the pipelined host-buffer call (gstm_run_host_async):
-        # every step copies its 4 MiB of balances in from pinned host memory
-        # and its result out, on the library's copy streams, overlapping the
-        # neighbouring steps' transactions; one CUDA-event
-        # pair around all steps, joined onto the launching stream.
-        # the same handle as the kernel-only measurement (its g_clock line
-        # was probed once; a second handle would draw its own placement,
-        # DESIGN.md §6.5)
-        g2 = g
-        for w in range(2):                                    # warm-up
-            g2.run_host_async("bank", h_in, h_out, T, K, seed0 + w)
-        g2.sync()
-        g2.reset_stats_total()
-        n_e2e = max(3, min(args.steps, 10))
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        for k in range(n_e2e):
-            flush.fill_(float(k))
-            g2.run_host_async("bank", h_in, h_out, T, K, seed0 + 7 + k)
-        g2.join()
-        b.record(stream)
-        b.synchronize()
-        g2.sync()
-        st2, n2 = g2.stats_total()
-        assert n2 == n_e2e
-        e2e_ms = a.elapsed_time(b)
-        e2e_done = st2.commits + st2.commits_ro
-        extra["e2e"] = {"value": e2e_done / (e2e_ms * 1e-3), "unit": UNIT,
-                        "h2d_bytes_per_step": ACCOUNTS * 4, "d2h_bytes_per_step": ACCOUNTS * 4,
-                        "api": "gstm_run_host_async (host buffers, pinned; copies pipelined with the "
-                               "neighbouring steps' transactions), gstm_join + CUDA events",
-                        "steps": n_e2e}
-        if not args.no_cgl:
-            extra["cgl"] = cgl_baseline(G, stream, T, seed0)
-            extra["stm_vbv"] = cgl_baseline(G, stream, T, seed0, mode="vbv")
-            table = [Variant("auto", "split"), Variant("tbv", "split"), Variant("hv", "split"),
-                     Variant("tbv", "paired"), Variant("hv", "paired", prelock=1),
-                     Variant("hv_backoff", "split"), Variant("hv_backoff", "paired", k_lock=1),
-                     Variant("fgl", "split"), Variant("fgl", "paired"),
-                     # FGL launches one CUDA thread per STM thread; also give the
-                     # hand-locking ceiling the concurrency the STM grid runs at
-                     # (16 warps per SM), its measured best
-                     Variant("fgl", "split", max_threads=512 * torch.cuda.get_device_properties(dev).multi_processor_count)]
-            extra["variants"] = variant_table(G, stream, flush, T, K, seed0,
-                                              [v for v in table if v.name != var.name])
-            fgl = [v for k, v in extra["variants"].items() if k.startswith("fgl")]
-            if fgl:
-                extra["fgl"] = max(fgl, key=lambda v: v["value"])
-        peaks, peak_src = measured_peaks()
-        extra["roofline"] = roofline(var, mode_used, tot, t_ms, args.steps, peaks, peak_src)
-        extra["roofline_l2"] = roofline_l2(G, var, mode_used, tot, t_ms, args.steps)
-        if world == 1 and not args.no_cpu:
-            extra["cpu_baseline"] = cpu_baseline(T, K, SEED)
-
+    tot = from_vector(vec[:NVEC])
+    balance_ok = int(vec[NVEC]) == world * ACCOUNTS * 1000
     done = tot["commits"] + tot["commits_ro"]
+    value = done / (t_ms * 1e-3)
+
+    if rank == 0 and not args.host_selftest:
+        extra.update(bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, tot, value, world,
+                                 detail))
     if rank == 0:
-        value = done / (t_ms * 1e-3)
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": config(args, f"{var.name} (mode used: {mode_used})"),
+            "config": config(args), "variant": f"{var_name} (mode used: {mode_used})",
             "abort_ratio": tot["aborts"] / max(1.0, tot["aborts"] + done),
-            "stats": {k: int(v) for k, v in tot.items()},
             "invariant_total_balance_ok": bool(balance_ok),
-            "clock_slot": int(st_tot.clock_slot),      # probed g_clock line
-            "clocks": clocks,
-            "gpu_launches": 3 * args.steps,
-            "wall_s_timed_region": wall,
+            "clocks": clocks, "gpu_launches": 3 * args.steps, "wall_s_timed_region": wall,
         }
-        if "cgl" in extra:
-            line["speedup_vs_cgl"] = value / world / extra["cgl"]["value"]
+        if comm:
+            line["comm"] = comm
+        if args.host_selftest:
+            line["selftest"] = "fake device steps (bench.py --host-selftest): host logic only, not a measurement"
+            line["stats"] = {k: int(v) for k, v in tot.items() if k in ("commits", "commits_ro", "aborts")}
         line.update(extra)
+        if detail:
+            sys.stderr.write("BENCH_DETAIL " + json.dumps(detail) + "\n")
         print(json.dumps(line), flush=True)
-    g.close()
+    if g is not None:
+        g.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
     return 0
 
 
+def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, tot, value, world, detail):
+    """Rank 0, after the timed region: e2e through the C ABI with host
+    buffers, CGL/FGL, the roofline, the other configs, the CPU baseline."""
+    import numpy as np
+    import torch
+    extra = {}
+    # e2e through the pipelined host-buffer call (gstm_run_host_async):
+    # every step copies its 4 MiB of balances in from pinned host memory
+    # and its result out, on the library's copy streams, overlapping the
+    # neighbouring steps' transactions (DESIGN.md §7.1); one CUDA-event
+    # pair around all steps, joined onto the launching stream; the same
+    # handle as the kernel-only measurement (its g_clock line was probed
+    # once, DESIGN.md §6.5)
+    pin_in = torch.full((ACCOUNTS,), 1000, dtype=torch.int32).pin_memory()
+    pin_out = torch.empty(ACCOUNTS, dtype=torch.int32).pin_memory()
+    h_in = pin_in.numpy().view(np.uint32)
+    h_out = pin_out.numpy().view(np.uint32)
+    for w in range(2):                                    # warm-up
+        g.run_host_async("bank", h_in, h_out, T, K, seed0 + w)
+    g.sync()
+    g.reset_stats_total()
+    n_e2e = max(3, min(args.steps, 10))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for k in range(n_e2e):
+        flush.fill_(float(k))
+        g.run_host_async("bank", h_in, h_out, T, K, seed0 + 7 + k)
+    g.join()
+    b.record(stream)
+    b.synchronize()
+    g.sync()
+    st2, n2 = g.stats_total()
+    assert n2 == n_e2e
+    e2e_ms = a.elapsed_time(b)
+    extra["e2e"] = {"value": (st2.commits + st2.commits_ro) / (e2e_ms * 1e-3), "unit": UNIT,
+                    "h2d_bytes_per_step": ACCOUNTS * 4, "d2h_bytes_per_step": ACCOUNTS * 4,
+                    "api": "gstm_run_host_async (pinned host buffers, copies pipelined with the neighbouring "
+                           "steps), gstm_join + CUDA events", "steps": n_e2e}
+    if not args.no_cgl:
+        mk = lambda m: Variant(m).handle(G, stream)                              # noqa: E731
+        cgl = cgl_rate(G, mk, "bank", T, K, seed0)
+        detail["bank_cgl"] = cgl
+        extra["cgl"] = {"value": cgl["value"], "unit": UNIT, "threads": cgl["threads"],
+                        "backoff_ns": cgl["backoff_ns"], "kernel": "cgl_kernel<BankWL>"}
+        extra["speedup_vs_cgl"] = value / world / cgl["value"]
+        table = [Variant("auto", "split"), Variant("tbv", "split"), Variant("hv", "split"),
+                 Variant("tbv", "paired"), Variant("hv", "paired", prelock=1),
+                 Variant("hv_backoff", "split"), Variant("hv_backoff", "paired", k_lock=1),
+                 Variant("fgl", "split"), Variant("fgl", "paired"),
+                 # FGL launches one CUDA thread per STM thread; also give the
+                 # hand-locking ceiling the concurrency the STM grid runs at
+                 # (16 warps per SM), its measured best
+                 Variant("fgl", "split", max_threads=512 * torch.cuda.get_device_properties(dev).multi_processor_count)]
+        detail["bank_variants"] = variant_table(G, stream, flush, T, K, seed0, [v for v in table if v.name != var.name])
+        detail["bank_stm_vbv"] = cgl_rate(G, lambda m: Variant("vbv").handle(G, stream), "bank", T, K, seed0,
+                                          mode="vbv")
+        fgl = [v for k, v in detail["bank_variants"].items() if k.startswith("fgl")]
+        if fgl:
+            best = max(fgl, key=lambda v: v["value"])
+            extra["fgl"] = {"value": best["value"], "unit": UNIT}
+        extra["auto_split"] = {"value": detail["bank_variants"]["auto/split"]["value"],
+                               "note": "the paper's STM-Optimized rule (P:252) on the paper's split layout"}
+    # the roofline of the headline kernel: the committed transactions' own
+    # op mix, measured on a scratch handle of the same layout (DESIGN.md §7.2)
+    paired = var.layout == "paired"
+    gp = g.params()
+    roof = op_mix_roof(G, R, stream, "bank", tot, mode_used, bool(var.prelock), gp.lock_pipeline > 0,
+                       ACCOUNTS, BITS, paired, T)
+    peaks = class_peaks(G, ACCOUNTS * 8, paired)            # paired: 8 B pairs; split: 4 B words + 4 B locks
+    maxf = max_formula(roof["ops_per_tx"], peaks)
+    ops = roof["ops_per_tx"]
+    extra["roofline"] = roofline_object(value / world, roof, maxf, ops["ld"] + ops["atom"] + ops["st"],
+                                        "launch duration = CUDA events on the launching stream around each step "
+                                        "(prepare + stm_kernel + finish; stm_kernel is 99.8% of it, "
+                                        "profiles/r01_bank_headline_launches.csv); traffic null: ncu DRAM bytes "
+                                        "come from a separate capture (profiles/), not from this run")
+    detail["bank_roof"] = {k: v for k, v in roof.items() if k != "program"}
+    detail["bank_class_peaks"] = peaks
+    if not args.no_configs:
+        only = [c for c in args.only_configs.split(",") if c] or list(CONFIGS)
+        cfgs = {}
+        for name in only:
+            t0 = time.perf_counter()
+            cfgs[name], detail[f"config_{name}"] = run_config(G, R, stream, flush, name, SEED + 31)
+            cfgs[name]["wall_s"] = round(time.perf_counter() - t0, 2)
+        extra["configs"] = cfgs
+    if world == 1 and not args.no_cpu:
+        extra["cpu_baseline"] = cpu_baseline(T, K, SEED)
+    return extra
+
+
 # ---------------------------------------------------------------------------
 # native arm, key-partitioned hash table (SURVEY §8e)
 # ---------------------------------------------------------------------------
-HT_BUCKETS, HT_THREADS, HT_K, HT_KEYS, HT_BITS = 1 << 20, 1 << 22, 4, 1 << 22, 22
-
-
 def ht_walk_count(heap, B, M):
     """Nodes reachable from the B bucket heads (vectorised chain walk) and
     the number of distinct keys among them (verification, after timing)."""
@@ -563,8 +799,11 @@ def run_native_ht(args):
     args.gpus = world
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    comm = None
     if world > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
         dist.init_process_group("nccl", device_id=dev)
+        comm = {"backend": "nccl", "nranks": dist.get_world_size()}
     from paper_conf_cgo_xuwglgq14_b200 import build as B
     if rank == 0 or world == 1:
         B.build()
@@ -580,23 +819,19 @@ def run_native_ht(args):
     stream = torch.cuda.Stream(device=dev)
     torch.cuda.set_stream(stream)
 
-    def handle():
-        g = G.Gstm(words, HT_BITS)
-        g.set_workload_defaults("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90,
-                                shard_bits=world.bit_length() - 1, shard=rank, k_lock=args.k_lock,
-                                prelock_vbv=prelock)
-        g.set_mode(mode)
-        g.set_stream(stream)
-        g.init_heap("ht")
-        return g
-
-    g = handle()
+    g = G.Gstm(words, HT_BITS)
+    g.set_workload_defaults("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90,
+                            shard_bits=world.bit_length() - 1, shard=rank, k_lock=args.k_lock,
+                            prelock_vbv=prelock)
+    g.set_mode(mode)
+    g.set_stream(stream)
+    g.init_heap("ht")
     flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)
     seed0 = shard_seed(rank)
     if world > 1:
         dist.barrier()
     step_ms, st_tot, wall, clocks = timed_steps(g, stream, flush, T, K, seed0, args.steps, args.warmup, local,
-                                                wl="ht")
+                                                wl="ht", reinit=True)
     if world > 1:
         dist.barrier()
     t_ms = float(sum(step_ms))
@@ -606,8 +841,8 @@ def run_native_ht(args):
     ok_local = float(nodes == distinct == last.commits)
     vec, (t_ms, wall) = reduce_over_ranks(list(stats_vector(st_tot)) + [nodes, ok_local], 0.0, t_ms, wall,
                                           world, dist, dev)
-    tot = from_vector(vec[:16])
-    keys_total, ok_ranks = int(vec[16]), int(vec[17])
+    tot = from_vector(vec[:NVEC])
+    keys_total, ok_ranks = int(vec[NVEC]), int(vec[NVEC + 1])
     extra = {}
     if rank == 0:
         h_in = np.zeros(words, dtype=np.uint32)
@@ -617,38 +852,26 @@ def run_native_ht(args):
         # e2e through the pipelined host-buffer call on the measured handle:
         # each step copies in its empty table (the step's input) and copies
         # out the filled one; copies overlap the neighbouring steps (§7.1)
-        g2 = g
-        g2.run_host_async("ht", hi, ho, T, K, seed0)
-        g2.sync()
-        g2.reset_stats_total()
+        g.run_host_async("ht", hi, ho, T, K, seed0)
+        g.sync()
+        g.reset_stats_total()
         n_e2e = max(3, min(args.steps, 5))
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         for k in range(n_e2e):
-            g2.run_host_async("ht", hi, ho, T, K, seed0 + 7 + k)
-        g2.join()
+            g.run_host_async("ht", hi, ho, T, K, seed0 + 7 + k)
+        g.join()
         b.record(stream)
         b.synchronize()
-        g2.sync()
-        st2, n2 = g2.stats_total()
+        g.sync()
+        st2, n2 = g.stats_total()
         assert n2 == n_e2e
         e2e_ms = a.elapsed_time(b)
-        e2e_done = st2.commits + st2.commits_ro
-        extra["e2e"] = {"value": e2e_done / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": words * 4,
-                        "d2h_bytes_per_step": words * 4, "steps": n_e2e,
+        extra["e2e"] = {"value": (st2.commits + st2.commits_ro) / (e2e_ms * 1e-3), "unit": UNIT,
+                        "h2d_bytes_per_step": words * 4, "d2h_bytes_per_step": words * 4, "steps": n_e2e,
                         "api": "gstm_run_host_async (pinned host buffers, pipelined copies), gstm_join + CUDA events"}
         extra["roofline"] = None
         extra["roofline_note"] = "the roofline object is reported for the bank headline (bench.py default)"
-        if world == 1 and not args.no_cpu:
-            import oracle as O
-            p = O.params("ht", ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90)
-            Ts = 1 << 20
-            heap = np.zeros(HT_BUCKETS + 2 * Ts * K, dtype=np.uint32)
-            t0 = time.perf_counter()
-            O.serial(p, heap, Ts, K, SEED)
-            dt = time.perf_counter() - t0
-            extra["cpu_baseline"] = {"value": Ts * K / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-                                     "sample": f"serial oracle, {Ts} threads x {K} HT operations, {dt:.2f} s"}
     done = tot["commits"] + tot["commits_ro"]
     if rank == 0:
         value = done / (t_ms * 1e-3)
@@ -659,16 +882,17 @@ def run_native_ht(args):
             "config": {"workload": "hash table insert/lookup (BASELINE configs[2]), key-partitioned over ranks",
                        "buckets_per_gpu": HT_BUCKETS, "threads_per_gpu": T, "tx_per_thread": K,
                        "lookup_pct": 90, "key_range": HT_KEYS, "lock_table_bits": HT_BITS,
-                       "variant": f"{mode}/split/k_lock={args.k_lock}"
-                                  + (f"/prelock={prelock}" if mode_used in ("hv", "hv_backoff") else "")
-                                  + f" (mode used: {mode_used})",
                        "partition": f"{world} shard(s): rank g owns keys with mix64 top {world.bit_length() - 1} bits = g",
                        "l2": "flushed (256 MiB write) between timed steps"},
+            "variant": f"{mode}/split/k_lock={args.k_lock}"
+                       + (f"/prelock={prelock}" if mode_used in ("hv", "hv_backoff") else "")
+                       + f" (mode used: {mode_used})",
             "abort_ratio": tot["aborts"] / max(1.0, tot["aborts"] + done),
-            "stats": {k: int(v) for k, v in tot.items()},
             "invariant_keys_ok": ok_ranks == world, "keys_in_tables_last_step": keys_total,
             "clocks": clocks, "gpu_launches": 3 * args.steps, "wall_s_timed_region": wall,
         }
+        if comm:
+            line["comm"] = comm
         line.update(extra)
         print(json.dumps(line), flush=True)
     g.close()
@@ -680,6 +904,10 @@ def run_native_ht(args):
 
 def main():
     args = parse()
+    if args.cpu_oracle_leg:
+        return cpu_oracle_leg(args.cpu_oracle_leg)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return self_launch(args)
     if args.impl == "reference":
         return run_reference(args)
     if args.workload == "ht":

@@ -169,6 +169,13 @@ typedef struct {
                                  /*    round of an execution may be pipelined, so this  */
                                  /*    is <= the executions that reached TXCommit's     */
                                  /*    lock step (Q15, Q37)                             */
+    /* log sizes summed over the COMMITTED executions of the STM modes (0 for
+     * CGL/FGL/VBV): the per-transaction op counts of the op-mix roof
+     * */
+    uint64_t reads_update;       /* read-set entries (memory reads) of update commits  */
+    uint64_t reads_ro;           /* read-set entries of read-only commits              */
+    uint64_t writes_update;      /* write-set entries of update commits                */
+    uint64_t locks_update;       /* lock-log entries (locks taken) of update commits   */
 } gstm_stats_t;
 
 /* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */
@@ -318,10 +325,34 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant);
 /* Roofline microbenchmark: kind 0 random atom.or, 1
  * same-address atom.add.u64, 2 random ld.relaxed, 3 random st.relaxed, 4
- * dependent atom.or chain, 5 warp-aggregated clock increments; over a table
+ * dependent atom.or chain, 5 warp-aggregated clock increments, 6/7/8 random
+ * 8-byte atom.or / ld / st (the paired layout's accesses); over a table
  * of table_bytes (power of two) with `threads` threads (multiple of 256).
  * *ops_per_s = operations per second; *ms = kernel time. */
 int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
+
+/* Op-mix roofline microbenchmark: n_tx conflict-free
+ * "transactions" on the handle's own memory (its layout, lock table and
+ * g_clock line), each the exact memory operations Algorithm 3 issues for one
+ * transaction of a workload, in its dependency order, without the STM logic.
+ * prog (prog_words uint32): prog[0] = number of programs P (1..4), | 0x100
+ * for record addressing (then prog[1] = records R, prog[2] = stride S: slot j
+ * of thread t is word (t mod R)*S + j mod S -- with R threads, each record's
+ * transactions form one serial chain, the contention roof of k-means), then per
+ * program: weight (the P weights sum to 65536), n_phases (<= 96), and
+ * n_phases phase words kind | count << 8 | slot0 << 16.  The ops of a phase
+ * are independent; each phase's addresses depend on the previous phase's
+ * results (one round trip per phase).  Op j of a phase touches word slot
+ * slot0 + j of the transaction: a random word in [0, words), the same word in
+ * every phase.  kind: 1 value load, 2 version-lock load, 3 lock atom.or, 4
+ * value store, 5 lock store (on the paired layout 1-5 are 8-byte accesses to
+ * the word's pair), 6 warp-aggregated atom.add on g_clock (count ignored),
+ * 7 release fence, 8 acquire fence.  threads (multiple of block, block a
+ * multiple of 32 <= 256) sets the occupancy.  Synchronous; CLOBBERS the
+ * heap, the lock table and the clock (which are reset: a new version epoch).
+ * *tx_per_s = transactions per second; *ms (may be NULL) = kernel time. */
+int gstm_ubench_mix(gstm_t* h, uint64_t words, const uint32_t* prog, uint32_t prog_words, uint64_t n_tx,
+                    uint32_t threads, uint32_t block, double* tx_per_s, double* ms);
 
 #ifdef __cplusplus
 }

@@ -268,6 +268,10 @@ static void fill_stats(gstm_stats_t* out, const unsigned long long* s, double ms
     out->attempts = s[S_ATTEMPTS];
     out->errors = s[S_ERRORS];
     out->pipelined_rounds = s[S_PIPELINED];
+    out->reads_update = s[S_RD_UPD];
+    out->reads_ro = s[S_RD_RO];
+    out->writes_update = s[S_WR_UPD];
+    out->locks_update = s[S_LK_UPD];
     out->elapsed_ms = ms;
     const double done = static_cast<double>(out->commits + out->commits_ro);
     out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
@@ -967,6 +971,18 @@ int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads
     if (rc == -1) { set_error("gstm_ubench: bad argument"); return GSTM_EINVAL; }
     if (rc) { set_error("gstm_ubench: CUDA failure %d", rc); return GSTM_ECUDA; }
     return GSTM_OK;
+}
+
+int gstm_ubench_mix(gstm_t* h, uint64_t words, const uint32_t* prog, uint32_t prog_words, uint64_t n_tx,
+                    uint32_t threads, uint32_t block, double* tx_per_s, double* ms)
+{
+    if (!h || !tx_per_s || words > h->heap_words) { set_error("gstm_ubench_mix: bad argument"); return GSTM_EINVAL; }
+    const int rc = ubench_mix(meta_of(h), h->paired, words, prog, prog_words, n_tx, threads, block, h->stream,
+                              tx_per_s, ms);
+    if (rc == -1) { set_error("gstm_ubench_mix: bad program or launch shape"); return GSTM_EINVAL; }
+    if (rc) { set_error("gstm_ubench_mix: CUDA failure %d", rc); return GSTM_ECUDA; }
+    // the clobbered lock table and clock start a new version epoch
+    return gstm_reset_meta(h);
 }
 
 }  // extern "C"

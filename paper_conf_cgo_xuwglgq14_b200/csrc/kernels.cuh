@@ -14,6 +14,10 @@ enum {
     S_COMMITS = 0, S_COMMITS_RO, S_AB_OPACITY, S_AB_PREVBV, S_AB_TBV, S_AB_COMMITVBV, S_AB_LOCK,
     S_LOCK_RETRIES, S_POSTVAL, S_VBV, S_SPINS, S_ATTEMPTS, S_ERRORS,
     S_PIPELINED,           // pipelined lock rounds: at most one per execution
+    // log sizes of the COMMITTED executions (the algorithmic op counts of the
+    // op-mix roof): reads appended to the read-set by update /
+    // read-only commits, write-set entries and lock-log entries of update commits
+    S_RD_UPD, S_RD_RO, S_WR_UPD, S_LK_UPD,
     S_NSTATS
 };
 
@@ -77,6 +81,8 @@ cudaError_t launch_km_assign(const KParams& kp, uint32_t* cluster, cudaStream_t 
 cudaError_t launch_km_init_centroids(const Meta& m, uint64_t c0, uint64_t n, cudaStream_t s);
 cudaError_t launch_km_recenter(const Meta& m, uint32_t C, uint32_t D, uint32_t stride, cudaStream_t s);
 int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
+int ubench_mix(const Meta& m, bool paired, uint64_t words, const uint32_t* prog, uint32_t prog_words, uint64_t n_tx,
+               uint32_t threads, uint32_t block, cudaStream_t s, double* tx_per_s, double* ms);
 int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s);
 int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_words, uint32_t* locks, uint32_t lmask,
                         uint32_t* heap, uint32_t hmask, cudaStream_t s);

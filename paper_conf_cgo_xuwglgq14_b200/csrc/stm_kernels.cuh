@@ -257,6 +257,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     p.tx_result[tx_id] = result;
                 }
                 cnt.inc(S_COMMITS_RO);
+                cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
                 done = true;
             } else {
                 stage = 1;
@@ -322,6 +323,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 p.tx_result[tx_id] = result;
             }
             cnt.inc(S_COMMITS);
+            cnt.inc(S_RD_UPD, static_cast<uint32_t>(tx.nr));
+            cnt.inc(S_WR_UPD, static_cast<uint32_t>(tx.nw));
+            cnt.inc(S_LK_UPD, static_cast<uint32_t>(tx.nl));
             done = true;
         }
         if constexpr (POL == POL_BACKOFF) {
@@ -361,6 +365,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                             p.tx_result[tx_id] = result;
                         }
                         cnt.inc(S_COMMITS);
+                        cnt.inc(S_RD_UPD, static_cast<uint32_t>(tx.nr));
+                        cnt.inc(S_WR_UPD, static_cast<uint32_t>(tx.nw));
+                        cnt.inc(S_LK_UPD, static_cast<uint32_t>(tx.nl));
                         done = true;
                     } else if (r == C_LOCK) {
                         cnt.inc(S_LOCK_RETRIES);

@@ -8,9 +8,11 @@
 //   3  random st.relaxed.gpu.u32 over S bytes                     (write-back / release)
 //   4  dependent chain of random atom.or (one per thread in flight): latency
 //   5  same-address atom.add.u64 issued by one lane per warp      (aggregated clock)
+//   6-8  random atom.or.b64 / ld.u64 / st.u64 over S bytes        (paired layout)
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <cuda_runtime.h>
 #include "kernels.cuh"
 
@@ -61,6 +63,27 @@ __global__ void ubench_kernel(int kind, uint32_t* table, uint32_t mask, unsigned
         if (prim::lane_id() == 0)
             for (uint32_t k = 0; k < n_per_thread; ++k) acc += static_cast<uint32_t>(prim::atom_add_relaxed64(hot, 32ull));
         break;
+    // 8-byte versions (the paired layout's value|lock accesses)
+    case 6: {
+        unsigned long long* t64 = reinterpret_cast<unsigned long long*>(table);
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k)
+            acc += static_cast<uint32_t>(prim::atom_or_relaxed_u64(t64 + ((ub_hash(t, k) & mask) >> 1), 0ull));
+        break;
+    }
+    case 7: {
+        unsigned long long* t64 = reinterpret_cast<unsigned long long*>(table);
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k)
+            acc += static_cast<uint32_t>(prim::ld_relaxed_u64(t64 + ((ub_hash(t, k) & mask) >> 1)));
+        break;
+    }
+    case 8: {
+        unsigned long long* t64 = reinterpret_cast<unsigned long long*>(table);
+#pragma unroll 4
+        for (uint32_t k = 0; k < n_per_thread; ++k) prim::st_relaxed_u64(t64 + ((ub_hash(t, k) & mask) >> 1), k);
+        break;
+    }
     }
     if (acc == 0xdeadbeefu) sink[0] = acc;
 }
@@ -96,6 +119,148 @@ __global__ void clock_mix_probe_kernel(unsigned long long* word, uint32_t* locks
         acc += static_cast<uint32_t>(__shfl_sync(0xffffffffu, b, 0)) & 1u;
     }
     if (acc == 0xdeadbeefu) sink[0] = 1;
+}
+
+// ---------------------------------------------------------------------------
+// Op-mix roof: every thread runs conflict-free
+// "transactions" made of exactly the memory operations Algorithm 3 issues for
+// one transaction of a workload, in the same dependency order, with no STM
+// logic around them (no logs, no validation branches, no retries).  A
+// program is a list of phases; the ops of one phase are independent (issued
+// back to back), and every phase's addresses depend on the previous phase's
+// results, so each phase costs one memory round trip -- as in the kernel.
+// Word slot j of a transaction is the same random word in every phase (the
+// value load, the lock load, the lock atomic and the store of word j hit the
+// same lines the kernel would).  Up to kMixProgs programs are mixed per
+// transaction by weight (e.g. update vs read-only transactions in the
+// proportions the measured run committed).
+// ---------------------------------------------------------------------------
+constexpr int kMixProgs = 4, kMixPhases = 96;
+struct MixProg {
+    uint32_t n_prog;
+    uint32_t records, stride;            // records > 0: slot j of thread t = word (t mod records)*stride + j
+    uint32_t cum[kMixProgs];             // cumulative weights out of 65536
+    uint32_t n_ph[kMixProgs];
+    uint32_t ph[kMixProgs][kMixPhases];  // kind | count << 8 | slot0 << 16
+};
+enum { MIX_LD_V = 1, MIX_LD_L = 2, MIX_ATOM_L = 3, MIX_ST_V = 4, MIX_ST_L = 5, MIX_CLOCK = 6, MIX_FENCE_REL = 7,
+       MIX_ACQ = 8, MIX_KINDS };
+
+template <bool PAIR>
+__global__ void __launch_bounds__(256) ubench_mix_kernel(const MixProg P, const Meta m, uint64_t words, uint32_t n_per_thread,
+                                                         uint32_t* sink)
+{
+    const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    uint32_t acc = 0;
+    for (uint32_t k = 0; k < n_per_thread; ++k) {
+        const uint64_t x = gen::mix64(t * gen::kGamma + k);
+        const uint32_t r = static_cast<uint32_t>(x >> 48);
+        uint32_t prog = 0;
+        while (prog + 1 < P.n_prog && r >= P.cum[prog]) ++prog;
+        uint32_t dep = 0;
+        for (uint32_t ph = 0; ph < P.n_ph[prog]; ++ph) {
+            const uint32_t code = P.ph[prog][ph];
+            const uint32_t kind = code & 0xffu, cnt = (code >> 8) & 0xffu, s0 = code >> 16;
+            uint32_t nd = 0;
+            if (kind == MIX_CLOCK) {
+                const unsigned am = __activemask();
+                const int leader = __ffs(am) - 1;
+                unsigned long long b = 0;
+                if (static_cast<int>(prim::lane_id()) == leader) b = prim::atom_add_acquire64(m.clock, __popc(am));
+                nd = static_cast<uint32_t>(__shfl_sync(am, b, leader));
+            } else if (kind == MIX_FENCE_REL) {
+                prim::fence_release();
+            } else if (kind == MIX_ACQ) {
+                prim::fence_acquire();
+            } else {
+#pragma unroll 8
+                for (uint32_t j = 0; j < cnt; ++j) {
+                    const uint32_t w = P.records
+                        ? static_cast<uint32_t>((t % P.records) * P.stride + ((s0 + j + dep) % P.stride))
+                        : static_cast<uint32_t>(gen::bounded(gen::draw(x, s0 + j) ^ dep, words));
+                    if constexpr (PAIR) {
+                        unsigned long long* pp = m.pair_ptr(w);
+                        if (kind == MIX_LD_V || kind == MIX_LD_L) nd ^= static_cast<uint32_t>(prim::ld_relaxed_u64(pp));
+                        else if (kind == MIX_ATOM_L) nd ^= static_cast<uint32_t>(prim::atom_or_relaxed_u64(pp, 0ull));
+                        else prim::st_relaxed_u64(pp, dep);
+                    } else {
+                        if (kind == MIX_LD_V) nd ^= prim::ld_relaxed(m.val_ptr(w));
+                        else if (kind == MIX_LD_L) nd ^= prim::ld_relaxed(m.lock_ptr(m.lock_of(w)));
+                        else if (kind == MIX_ATOM_L) nd ^= prim::atom_or_relaxed(m.lock_ptr(m.lock_of(w)), 0u);
+                        else if (kind == MIX_ST_V) prim::st_relaxed(m.val_ptr(w), dep);
+                        else prim::st_relaxed(m.lock_ptr(m.lock_of(w)), dep & ~1u);
+                    }
+                }
+            }
+            // the next phase's addresses depend on this phase's results (one
+            // round trip per phase); stores and fences leave dep unchanged
+            dep ^= nd & 0x1u;
+        }
+        acc += dep;
+    }
+    if (acc == 0xdeadbeefu) sink[0] = acc;
+}
+
+int ubench_mix(const Meta& m, bool paired, uint64_t words, const uint32_t* prog, uint32_t prog_words, uint64_t n_tx,
+               uint32_t threads, uint32_t block, cudaStream_t s, double* tx_per_s, double* ms_out)
+{
+    if (!prog || !tx_per_s || !words || words > (1ull << 32) || threads == 0 || block == 0 || block > 256 ||
+        block % 32 || threads % block || prog_words < 1)
+        return -1;
+    MixProg P;
+    memset(&P, 0, sizeof(P));
+    P.n_prog = prog[0] & 0xffu;
+    if (P.n_prog < 1 || P.n_prog > kMixProgs) return -1;
+    uint32_t pos = 1, cum = 0;
+    if (prog[0] & 0x100u) {              // record addressing: prog[1] = records, prog[2] = stride
+        if (prog_words < 3 || !prog[1] || !prog[2] || uint64_t(prog[1]) * prog[2] > words) return -1;
+        P.records = prog[1];
+        P.stride = prog[2];
+        pos = 3;
+    }
+    for (uint32_t q = 0; q < P.n_prog; ++q) {
+        if (pos + 2 > prog_words) return -1;
+        cum += prog[pos];
+        P.cum[q] = cum;
+        P.n_ph[q] = prog[pos + 1];
+        pos += 2;
+        if (P.n_ph[q] > kMixPhases || pos + P.n_ph[q] > prog_words) return -1;
+        for (uint32_t k = 0; k < P.n_ph[q]; ++k) {
+            const uint32_t kind = prog[pos + k] & 0xffu;
+            if (kind == 0 || kind >= MIX_KINDS) return -1;
+            P.ph[q][k] = prog[pos + k];
+        }
+        pos += P.n_ph[q];
+    }
+    if (cum != 65536u) return -1;
+    const uint32_t per = static_cast<uint32_t>((n_tx + threads - 1) / threads);
+    uint32_t* sink = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    int rc = 0;
+    if (cudaMalloc(&sink, 64) != cudaSuccess) return -2;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    const unsigned grid = threads / block;
+    auto run = [&]() {
+        if (paired) ubench_mix_kernel<true><<<grid, block, 0, s>>>(P, m, words, per, sink);
+        else ubench_mix_kernel<false><<<grid, block, 0, s>>>(P, m, words, per, sink);
+    };
+    run();                                            // warm-up
+    cudaEventRecord(e0, s);
+    run();
+    cudaEventRecord(e1, s);
+    if (cudaEventSynchronize(e1) != cudaSuccess || cudaGetLastError() != cudaSuccess) {
+        rc = -3;
+    } else {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        *tx_per_s = static_cast<double>(per) * threads / (ms * 1e-3);
+        if (ms_out) *ms_out = ms;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    return rc;
 }
 
 // Returns the index of the candidate (word = base + k*stride_words) with
@@ -171,7 +336,7 @@ out:
 // increments per second, i.e. 32 per atomic), or a negative error.
 int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms_out)
 {
-    if (kind < 0 || kind > 5 || threads == 0 || threads % 256 || table_bytes < 128 ||
+    if (kind < 0 || kind > 8 || threads == 0 || threads % 256 || table_bytes < 128 ||
         (table_bytes & (table_bytes - 1)))
         return -1;
     const uint32_t per = static_cast<uint32_t>((n_ops + threads - 1) / threads);

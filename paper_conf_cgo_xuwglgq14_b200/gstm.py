@@ -39,6 +39,7 @@ EXPORTS = [
     "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
     "gstm_lock_log", "gstm_ubench", "gstm_km_recenter", "gstm_run_host_async", "gstm_join", "gstm_sync",
+    "gstm_ubench_mix",
 ]
 
 
@@ -70,6 +71,8 @@ class gstm_stats_t(C.Structure):
         ("clock_end", C.c_uint64), ("elapsed_ms", C.c_double), ("tx_per_s", C.c_double),
         ("abort_ratio", C.c_double), ("status", C.c_int32), ("mode_used", C.c_int32),
         ("clock_slot", C.c_int32), ("pipelined_rounds", C.c_uint64),
+        ("reads_update", C.c_uint64), ("reads_ro", C.c_uint64), ("writes_update", C.c_uint64),
+        ("locks_update", C.c_uint64),
     ]
 
     def as_dict(self) -> dict:
@@ -127,6 +130,7 @@ def lib():
             "gstm_script": (i32, [V, i32, i32, V, i32, V, i32]),
             "gstm_lock_log": (i32, [V, i32, V, i32]),
             "gstm_ubench": (i32, [i32, u64, u64, u32, P(C.c_double), P(C.c_double)]),
+            "gstm_ubench_mix": (i32, [V, u64, V, u32, u64, u32, u32, P(C.c_double), P(C.c_double)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -396,6 +400,17 @@ def gstm_lock_log(entries, variant: int = 0) -> np.ndarray:
     out = np.zeros(256, dtype=np.uint32)
     n = _check(lib().gstm_lock_log(_ptr(e), e.size, _ptr(out), variant), "gstm_lock_log")
     return out[:n].copy()
+
+
+def gstm_ubench_mix(h, words: int, prog, n_tx: int, threads: int, block: int = 256):
+    """Op-mix roof (include/gstm.h): returns (tx/s, ms).  Clobbers the
+    handle's heap, lock table and clock."""
+    pr = np.ascontiguousarray(np.asarray(prog, dtype=np.uint32))
+    tps = C.c_double(0)
+    ms = C.c_double(0)
+    _check(lib().gstm_ubench_mix(h, words, _ptr(pr), pr.size, n_tx, threads, block, C.byref(tps), C.byref(ms)),
+           "gstm_ubench_mix")
+    return tps.value, ms.value
 
 
 def gstm_ubench(kind: int, table_bytes: int, n_ops: int, threads: int):

@@ -107,8 +107,10 @@ def test_km_assign_exact_when_64bit_sum_would_wrap():
         cent[2 * t], cent[2 * t + 1] = wrap, near
         d_wrap = sum((a - b) ** 2 for a, b in zip(f, wrap))
         assert d_wrap % (1 << 64) < 3000 ** 2 < d_wrap
-        exact = [sum((a - int(b)) ** 2 for a, b in zip(f, row)) for row in cent.tolist()]
-        want[int(np.argmin(exact))] += 1
+    rows = cent.tolist()
+    for t in range(T):                              # exact argmin (first minimum), Python integers
+        exact = [sum((int(a) - int(b)) ** 2 for a, b in zip(feats[t], row)) for row in rows]
+        want[min(range(Cn), key=lambda c: (exact[c], c))] += 1
     assert want[1::2].sum() == T                    # every point's nearest is a "near" row
     heap = init.copy()
     c0 = O.km_centroids(op)

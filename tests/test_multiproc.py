@@ -133,27 +133,81 @@ def test_two_rank_key_partitioned_ht_gloo():
     assert not set(got[0][2]) & set(got[1][2])                   # disjoint shards
 
 
-def test_bench_roofline_object_is_the_contract_and_the_cost_model():
-    """bench.py's `roofline` object (CPU-only arithmetic): contract keys, the
-    algorithmic sector model of DESIGN.md §7.2 (paired bank update = 2 pair
-    loads + 2 atom.or.b64 + 2 pair stores = 6 x 32 B; read-only = 2 loads;
-    split TBV update 10 sectors, + 2 pre-lock VBV loads for HV), and
-    achieved = bytes per launch / launch time."""
+def test_bench_roofline_object_is_the_contract():
+    """bench.py's `roofline` object (CPU-only arithmetic): the contract keys,
+    achieved and peak in algorithmic L2 sector bytes (32 B per access of the
+    committed transactions' own op mix), frac = achieved tx/s over the measured
+    op-mix roof, and the SURVEY §8(d) max-formula figure beside it."""
     import sys
     sys.path.insert(0, ROOT)
     import bench
-    tot = {"commits": 1_000_000, "commits_ro": 250_000}
-    r = bench.roofline(bench.Variant("hv", "paired"), "hv", tot, t_ms=2.0, steps=2,
-                       peaks={"hbm_gbs": 6000.0}, peak_src="test", traffic=123)
+    roof = {"roof_tx_per_s": 2.0e10, "threads": 75776, "round_trips_per_tx": 4.0}
+    peaks = {"ld": 2.8e11, "atom": 1.25e11, "st": 1.8e11, "clock": 4.9e10}
+    ops = {"ld": 2.0, "atom": 2.0, "st": 2.0, "clock": 1.0}
+    maxf = bench.max_formula(ops, peaks)
+    assert abs(maxf - 1 / max(2 / 2.8e11, 2 / 1.25e11, 2 / 1.8e11, 1 / 4.9e10)) < 1e-3
+    r = bench.roofline_object(1.0e10, roof, maxf, 6.0, "test")
     assert {"bound", "achieved", "peak", "unit", "frac", "traffic"} <= set(r)
-    assert r["bound"] == "hbm" and r["unit"] == "GB/s" and r["traffic"] == 123
-    assert r["bytes_per_unit"] == {"update_tx": 192, "read_only_tx": 64}
-    per_launch = (1_000_000 * 192 + 250_000 * 64) / 2
-    assert r["algorithmic_bytes_per_launch"] == per_launch
-    assert abs(r["achieved"] - per_launch / 1e-3 / 1e9) < 1e-9
-    assert abs(r["frac"] - r["achieved"] / 6000.0) < 1e-12
-    split_tbv = bench.roofline(bench.Variant("tbv", "split"), "tbv", tot, 2.0, 2, {}, "fallback", traffic=0)
-    assert split_tbv["bytes_per_unit"] == {"update_tx": 320, "read_only_tx": 128}
-    assert split_tbv["peak"] == 6650.0                  # the profiling guide's fallback
-    split_hv = bench.roofline(bench.Variant("hv", "split"), "hv", tot, 2.0, 2, {}, "fallback", traffic=0)
-    assert split_hv["bytes_per_unit"]["update_tx"] == 384
+    assert r["bound"] == "l2" and r["unit"] == "GB/s" and r["traffic"] is None
+    assert abs(r["achieved"] - 1.0e10 * 192 / 1e9) < 1e-6 and abs(r["peak"] - 2.0e10 * 192 / 1e9) < 1e-6
+    assert abs(r["frac"] - 0.5) < 1e-12 and abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-12
+    assert abs(r["frac_max_formula"] - 1.0e10 / maxf) < 1e-9
+
+
+def test_op_mix_programs_follow_algorithm_3():
+    """The op-mix roof's per-transaction programs (roofline.py) issue exactly
+    Algorithm 3's memory operations for the committed transactions' log sizes:
+    paired bank update = 2 pair loads, 2 atom.or (one pipelined round), the
+    clock, 2 pair stores (4 round trips); split TBV RA (4R/4W, 8 locks) = 4 +
+    4 loads, 8 sequential atomics (Q15), 4 write-back + 8 release stores, the
+    clock; HV adds the pre-lock VBV loads (A3.l71); read-only = reads only."""
+    from paper_conf_cgo_xuwglgq14_b200 import roofline as R
+    st = dict(commits=900, commits_ro=100, reads_update=1800, reads_ro=200, writes_update=1800, locks_update=1800)
+    p = R.programs_from_stats("bank", st, paired=True, mode="hv", prelock=False, pipelined=True)
+    ops = R.op_counts(p)
+    assert abs(ops["ld"] - 2.0) < 1e-3 and abs(ops["atom"] - 0.9 * 2) < 1e-3
+    assert abs(ops["st"] - 0.9 * 2) < 1e-3 and abs(ops["clock"] - 0.9) < 1e-3
+    assert abs(R.round_trips(p) - (0.9 * 4 + 0.1 * 1)) < 1e-3
+    st = dict(commits=10, commits_ro=0, reads_update=40, reads_ro=0, writes_update=40, locks_update=80)
+    p = R.programs_from_stats("ra", st, paired=False, mode="tbv", prelock=True, pipelined=False)
+    ops = R.op_counts(p)
+    assert ops == {"ld": 8.0, "atom": 8.0, "st": 12.0, "clock": 1.0}
+    assert R.round_trips(p) == 2 + 8 + 4 + 1 + 1            # loads, locks one by one, write-back, clock, release
+    ph = p[3:3 + p[2]]
+    atoms = [c for c in ph if c & 0xff == R.ATOM_L]
+    assert [(c >> 8) & 0xff for c in atoms] == [1] * 8 and [c >> 16 for c in atoms] == list(range(8))
+    p_hv = R.programs_from_stats("ra", st, paired=False, mode="hv", prelock=True, pipelined=False)
+    assert R.op_counts(p_hv)["ld"] == 12.0
+    # fractional mean reads (HT chains): two programs reproduce the mean exactly
+    st = dict(commits=0, commits_ro=4, reads_update=0, reads_ro=10, writes_update=0, locks_update=0)
+    p = R.programs_from_stats("ht", st, paired=False, mode="hv", prelock=False, pipelined=True)
+    assert p[0] == 2 and abs(R.op_counts(p)["ld"] - 2 * 2.5) < 1e-3
+    # record addressing (k-means: one serial chain per record)
+    st = dict(commits=5, commits_ro=0, reads_update=85, reads_ro=0, writes_update=85, locks_update=85)
+    p = R.programs_from_stats("km", st, paired=False, mode="hv", prelock=True, pipelined=False, records=(1024, 17))
+    assert p[0] == 1 | R.RECORDS and p[1:3] == [1024, 17]
+    assert R.op_counts(p)["atom"] == 17.0
+
+
+def test_bench_self_launches_n_ranks_with_gloo():
+    """`python bench.py --gpus 2` without a torchrun environment re-launches
+    itself as 2 ranks (torch.distributed.run); --host-selftest swaps the GPU
+    steps for fake counts so the host logic runs here on CPU with gloo: shard
+    seeds, barriers, the one SUM/MAX reduction, the aggregate value and the
+    communicator size in the JSON line."""
+    import json
+    import subprocess
+    import sys
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--host-selftest",
+                        "--steps", "4", "--warmup", "3"], capture_output=True, text=True, env=env, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout                          # rank 0 only
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["comm"] == {"backend": "gloo", "nranks": 2} and "selftest" in d
+    n = (1 << 20) * 16
+    assert d["stats"]["commits"] == 2 * (n - n // 16)         # SUM over ranks
+    assert abs(d["ms_per_step"] - 1.5) < 1e-9                 # MAX over ranks (rank 1: 1.5 ms per step)
+    assert abs(d["value"] - 2 * n / (4 * 1.5e-3)) < 1.0
+    assert d["invariant_total_balance_ok"]
