@@ -382,6 +382,7 @@ def op_mix_roof(G, R, stream, wl, st, mode, prelock, pipelined, words, bits, pai
     occupancies of gstm_ubench_mix on a scratch handle of the same layout and
     size (its g_clock line probed like the measured handle's)."""
     prog = R.programs_from_stats(wl, st, paired, mode, prelock, pipelined, records)
+    R.validate(prog, words)
     h = G.Gstm(words, bits, paired=paired)
     h.set_stream(stream)
     sweep = {}
@@ -641,8 +642,14 @@ def run_native(args):
     value = done / (t_ms * 1e-3)
 
     if rank == 0 and not args.host_selftest:
-        extra.update(bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, tot, value, world,
-                                 detail))
+        try:
+            extra.update(bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, tot, value,
+                                     world, detail))
+        except Exception as e:              # the headline line must still be printed
+            import traceback
+            traceback.print_exc()
+            extra["extras_error"] = f"{type(e).__name__}: {e}"
+            torch.cuda.synchronize()
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -753,8 +760,14 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
         cfgs = {}
         for name in only:
             t0 = time.perf_counter()
-            cfgs[name], detail[f"config_{name}"] = run_config(G, R, stream, flush, name, SEED + 31)
+            try:
+                cfgs[name], detail[f"config_{name}"] = run_config(G, R, stream, flush, name, SEED + 31)
+            except Exception as e:          # one config's failure must not lose the line
+                cfgs[name] = {"error": f"{type(e).__name__}: {e}"}
+                torch.cuda.synchronize()
             cfgs[name]["wall_s"] = round(time.perf_counter() - t0, 2)
+            sys.stderr.write(f"config {name}: {json.dumps(cfgs[name])}\n")
+            sys.stderr.flush()
         extra["configs"] = cfgs
     if world == 1 and not args.no_cpu:
         extra["cpu_baseline"] = cpu_baseline(T, K, SEED)

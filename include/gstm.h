@@ -339,7 +339,7 @@ int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads
  * for record addressing (then prog[1] = records R, prog[2] = stride S: slot j
  * of thread t is word (t mod R)*S + j mod S -- with R threads, each record's
  * transactions form one serial chain, the contention roof of k-means), then per
- * program: weight (the P weights sum to 65536), n_phases (<= 96), and
+ * program: weight (the P weights sum to 65536), n_phases (<= 160), and
  * n_phases phase words kind | count << 8 | slot0 << 16.  The ops of a phase
  * are independent; each phase's addresses depend on the previous phase's
  * results (one round trip per phase).  Op j of a phase touches word slot
@@ -347,7 +347,10 @@ int gstm_ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads
  * every phase.  kind: 1 value load, 2 version-lock load, 3 lock atom.or, 4
  * value store, 5 lock store (on the paired layout 1-5 are 8-byte accesses to
  * the word's pair), 6 warp-aggregated atom.add on g_clock (count ignored),
- * 7 release fence, 8 acquire fence.  threads (multiple of block, block a
+ * 7 release fence, 8 acquire fence (at most one clock phase per program).
+ * Warp-synchronous like the transaction kernel: the phases before the clock
+ * run per lane, then one warp-collective clock increment for the lanes that
+ * have one, then the phases after it.  threads (multiple of block, block a
  * multiple of 32 <= 256) sets the occupancy.  Synchronous; CLOBBERS the
  * heap, the lock table and the clock (which are reset: a new version epoch).
  * *tx_per_s = transactions per second; *ms (may be NULL) = kernel time. */

@@ -135,17 +135,64 @@ __global__ void clock_mix_probe_kernel(unsigned long long* word, uint32_t* locks
 // transaction by weight (e.g. update vs read-only transactions in the
 // proportions the measured run committed).
 // ---------------------------------------------------------------------------
-constexpr int kMixProgs = 4, kMixPhases = 96;
+constexpr int kMixProgs = 4, kMixPhases = 160;
 struct MixProg {
     uint32_t n_prog;
     uint32_t records, stride;            // records > 0: slot j of thread t = word (t mod records)*stride + j
     uint32_t cum[kMixProgs];             // cumulative weights out of 65536
     uint32_t n_ph[kMixProgs];
+    uint32_t clk[kMixProgs];             // index of the program's CLOCK phase (n_ph: none; at most one)
     uint32_t ph[kMixProgs][kMixPhases];  // kind | count << 8 | slot0 << 16
 };
 enum { MIX_LD_V = 1, MIX_LD_L = 2, MIX_ATOM_L = 3, MIX_ST_V = 4, MIX_ST_L = 5, MIX_CLOCK = 6, MIX_FENCE_REL = 7,
        MIX_ACQ = 8, MIX_KINDS };
 
+template <bool PAIR>
+__device__ __forceinline__ uint32_t mix_phases(const MixProg& P, const Meta& m, uint64_t words, uint64_t t, uint64_t x,
+                                               uint32_t prog, uint32_t from, uint32_t to, uint32_t dep)
+{
+    for (uint32_t ph = from; ph < to; ++ph) {
+        const uint32_t code = P.ph[prog][ph];
+        const uint32_t kind = code & 0xffu, cnt = (code >> 8) & 0xffu, s0 = code >> 16;
+        uint32_t nd = 0;
+        if (kind == MIX_FENCE_REL) {
+            prim::fence_release();
+        } else if (kind == MIX_ACQ) {
+            prim::fence_acquire();
+        } else {
+#pragma unroll 8
+            for (uint32_t j = 0; j < cnt; ++j) {
+                const uint32_t w = P.records
+                    ? static_cast<uint32_t>((t % P.records) * P.stride + ((s0 + j + dep) % P.stride))
+                    : static_cast<uint32_t>(gen::bounded(gen::draw(x, s0 + j) ^ dep, words));
+                if constexpr (PAIR) {
+                    unsigned long long* pp = m.pair_ptr(w);
+                    if (kind == MIX_LD_V || kind == MIX_LD_L) nd ^= static_cast<uint32_t>(prim::ld_relaxed_u64(pp));
+                    else if (kind == MIX_ATOM_L) nd ^= static_cast<uint32_t>(prim::atom_or_relaxed_u64(pp, 0ull));
+                    else prim::st_relaxed_u64(pp, dep);
+                } else {
+                    if (kind == MIX_LD_V) nd ^= prim::ld_relaxed(m.val_ptr(w));
+                    else if (kind == MIX_LD_L) nd ^= prim::ld_relaxed(m.lock_ptr(m.lock_of(w)));
+                    else if (kind == MIX_ATOM_L) nd ^= prim::atom_or_relaxed(m.lock_ptr(m.lock_of(w)), 0u);
+                    else if (kind == MIX_ST_V) prim::st_relaxed(m.val_ptr(w), dep);
+                    else prim::st_relaxed(m.lock_ptr(m.lock_of(w)), dep & ~1u);
+                }
+            }
+        }
+        // the next phase's addresses depend on this phase's results (one
+        // round trip per phase); stores and fences leave dep unchanged
+        dep ^= nd & 0x1u;
+    }
+    return dep;
+}
+
+// Warp-synchronous like the transaction kernel (stm_kernels.cuh): every
+// transaction starts at a warp barrier; the phases before the clock (body,
+// validation, locks, write-back) run per lane; then ONE warp-collective
+// clock increment for the lanes whose program has one (warp_stamp, A3.l83);
+// then the phases after it (release).  Without the barriers lanes that ran a
+// shorter program drift into later transactions and split the warp into
+// groups that each pay their own clock atomic.
 template <bool PAIR>
 __global__ void __launch_bounds__(256) ubench_mix_kernel(const MixProg P, const Meta m, uint64_t words, uint32_t n_per_thread,
                                                          uint32_t* sink)
@@ -153,49 +200,23 @@ __global__ void __launch_bounds__(256) ubench_mix_kernel(const MixProg P, const 
     const uint64_t t = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
     uint32_t acc = 0;
     for (uint32_t k = 0; k < n_per_thread; ++k) {
+        __syncwarp();
         const uint64_t x = gen::mix64(t * gen::kGamma + k);
         const uint32_t r = static_cast<uint32_t>(x >> 48);
         uint32_t prog = 0;
         while (prog + 1 < P.n_prog && r >= P.cum[prog]) ++prog;
-        uint32_t dep = 0;
-        for (uint32_t ph = 0; ph < P.n_ph[prog]; ++ph) {
-            const uint32_t code = P.ph[prog][ph];
-            const uint32_t kind = code & 0xffu, cnt = (code >> 8) & 0xffu, s0 = code >> 16;
-            uint32_t nd = 0;
-            if (kind == MIX_CLOCK) {
-                const unsigned am = __activemask();
-                const int leader = __ffs(am) - 1;
-                unsigned long long b = 0;
-                if (static_cast<int>(prim::lane_id()) == leader) b = prim::atom_add_acquire64(m.clock, __popc(am));
-                nd = static_cast<uint32_t>(__shfl_sync(am, b, leader));
-            } else if (kind == MIX_FENCE_REL) {
-                prim::fence_release();
-            } else if (kind == MIX_ACQ) {
-                prim::fence_acquire();
-            } else {
-#pragma unroll 8
-                for (uint32_t j = 0; j < cnt; ++j) {
-                    const uint32_t w = P.records
-                        ? static_cast<uint32_t>((t % P.records) * P.stride + ((s0 + j + dep) % P.stride))
-                        : static_cast<uint32_t>(gen::bounded(gen::draw(x, s0 + j) ^ dep, words));
-                    if constexpr (PAIR) {
-                        unsigned long long* pp = m.pair_ptr(w);
-                        if (kind == MIX_LD_V || kind == MIX_LD_L) nd ^= static_cast<uint32_t>(prim::ld_relaxed_u64(pp));
-                        else if (kind == MIX_ATOM_L) nd ^= static_cast<uint32_t>(prim::atom_or_relaxed_u64(pp, 0ull));
-                        else prim::st_relaxed_u64(pp, dep);
-                    } else {
-                        if (kind == MIX_LD_V) nd ^= prim::ld_relaxed(m.val_ptr(w));
-                        else if (kind == MIX_LD_L) nd ^= prim::ld_relaxed(m.lock_ptr(m.lock_of(w)));
-                        else if (kind == MIX_ATOM_L) nd ^= prim::atom_or_relaxed(m.lock_ptr(m.lock_of(w)), 0u);
-                        else if (kind == MIX_ST_V) prim::st_relaxed(m.val_ptr(w), dep);
-                        else prim::st_relaxed(m.lock_ptr(m.lock_of(w)), dep & ~1u);
-                    }
-                }
-            }
-            // the next phase's addresses depend on this phase's results (one
-            // round trip per phase); stores and fences leave dep unchanged
-            dep ^= nd & 0x1u;
+        const uint32_t clk = P.clk[prog], n = P.n_ph[prog];
+        uint32_t dep = mix_phases<PAIR>(P, m, words, t, x, prog, 0, clk, 0u);
+        __syncwarp();
+        const unsigned bm = __ballot_sync(prim::FULL, clk < n);
+        if (bm) {
+            const int leader = __ffs(bm) - 1;
+            unsigned long long b = 0;
+            if (static_cast<int>(prim::lane_id()) == leader) b = prim::atom_add_acquire64(m.clock, __popc(bm));
+            b = __shfl_sync(prim::FULL, b, leader);
+            dep ^= static_cast<uint32_t>(b) & 1u;
         }
+        if (clk < n) dep = mix_phases<PAIR>(P, m, words, t, x, prog, clk + 1, n, dep);
         acc += dep;
     }
     if (acc == 0xdeadbeefu) sink[0] = acc;
@@ -225,9 +246,14 @@ int ubench_mix(const Meta& m, bool paired, uint64_t words, const uint32_t* prog,
         P.n_ph[q] = prog[pos + 1];
         pos += 2;
         if (P.n_ph[q] > kMixPhases || pos + P.n_ph[q] > prog_words) return -1;
+        P.clk[q] = P.n_ph[q];
         for (uint32_t k = 0; k < P.n_ph[q]; ++k) {
             const uint32_t kind = prog[pos + k] & 0xffu;
             if (kind == 0 || kind >= MIX_KINDS) return -1;
+            if (kind == MIX_CLOCK) {
+                if (P.clk[q] != P.n_ph[q]) return -1;      // one clock increment per transaction
+                P.clk[q] = k;
+            }
             P.ph[q][k] = prog[pos + k];
         }
         pos += P.n_ph[q];

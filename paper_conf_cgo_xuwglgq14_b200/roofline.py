@@ -138,6 +138,35 @@ def programs_from_stats(wl: str, st, paired: bool, mode: str, prelock: bool, pip
     return mix(progs, records)
 
 
+MAX_PHASES = 160
+
+
+def validate(prog: list, words: int) -> None:
+    """The checks gstm_ubench_mix applies, with a message (GSTM_EINVAL
+    otherwise only says "bad program")."""
+    n, pos = prog[0] & 0xff, 1
+    if not 1 <= n <= 4:
+        raise ValueError(f"{n} programs (1..4)")
+    if prog[0] & RECORDS:
+        pos = 3
+        if prog[1] * prog[2] > words:
+            raise ValueError(f"records {prog[1]} x stride {prog[2]} > {words} words")
+    cum = 0
+    for q in range(n):
+        cum += prog[pos]
+        k = prog[pos + 1]
+        if k > MAX_PHASES:
+            raise ValueError(f"program {q}: {k} phases > {MAX_PHASES}")
+        for c in prog[pos + 2:pos + 2 + k]:
+            if not 1 <= (c & 0xff) <= 8:
+                raise ValueError(f"program {q}: bad phase kind {c & 0xff}")
+        if sum(1 for c in prog[pos + 2:pos + 2 + k] if c & 0xff == CLOCK) > 1:
+            raise ValueError(f"program {q}: more than one clock phase")
+        pos += 2 + k
+    if cum != 65536 or pos != len(prog):
+        raise ValueError(f"weights sum {cum}, {pos} of {len(prog)} words parsed")
+
+
 def op_counts(prog: list) -> dict:
     """Mean ops per transaction by class (the max-formula roof of SURVEY §8(d):
     roof = 1 / max_i(count_i / peak_i))."""
