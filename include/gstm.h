@@ -139,6 +139,11 @@ typedef struct {
                              /*    [t*k, t*k + k) (disjoint access sets: a unique,    */
                              /*    conflict-free result); needs        */
                              /*    n_threads * k <= n_words.  Default 0               */
+    uint32_t body_rounds;    /* STM modes: a lane whose transaction committed read-  */
+                             /*    only starts its next one in the same warp         */
+                             /*    iteration, up to this many bodies per iteration   */
+                             /*    (DESIGN.md §6.11); 0 or 1 = one body per          */
+                             /*    iteration.  Default 1 (HT: see DESIGN.md)         */
 } gstm_params_t;
 
 typedef struct {

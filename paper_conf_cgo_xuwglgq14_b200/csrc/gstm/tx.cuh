@@ -26,6 +26,17 @@
 #define GSTM_PV_ATTR __forceinline__
 #endif
 
+// a loop over a local-memory log: rolled in a compact Tx (kCompact), else
+// left to the compiler
+#define GSTM_LLOOP(...)                                        \
+    do {                                                       \
+        if constexpr (kCompact) {                              \
+            _Pragma("unroll 1") __VA_ARGS__                    \
+        } else {                                               \
+            __VA_ARGS__                                        \
+        }                                                      \
+    } while (0)
+
 namespace gstm {
 
 enum { MODE_HV = 1, MODE_TBV = 2 };
@@ -73,12 +84,19 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
 // SORTED = false: the lock log keeps encounter order (duplicates still
 // merged) -- the lock order of STM-HV-Backoff and of the unsorted
 // ablation; the paper's GPU-STM sorts.
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true>
+// COMPACT = true: loops over local-memory logs stay rolled (one copy of each,
+// `#pragma unroll 1`; validation loads 4 in flight) -- for kernels whose code
+// outgrows the instruction cache (HT: DESIGN.md §6.9); else the compiler
+// unrolls them (by 4) and validation keeps 8 loads in flight.
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false>
 struct Tx {
     // register-resident (unrolled) logs for small capacities unless the
     // workload asks for local memory (LOCAL: fewer registers, more warps)
     static constexpr bool kUnroll = !LOCAL && (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
     static constexpr int kRcap = RCAP, kWcap = WCAP, kLcap = LCAP;
+    static constexpr bool kCompact = COMPACT;
+    // value / lock-word loads validation keeps in flight with local-memory logs
+    static constexpr int kPvWidth = COMPACT ? 4 : 8;
 
     uint32_t r_addr[RCAP], r_val[RCAP];   // read-set  <addr,val>
     uint32_t w_addr[WCAP], w_val[WCAP];   // write-set <addr,val> (redo log)
@@ -184,7 +202,7 @@ struct Tx {
             }
             if (pos < nl && (l_ent[pos] >> 2) == id) { l_ent[pos] |= (e & 3u); return; }
             if (nl >= LCAP) { overflow = true; opaque = false; return; }
-            for (int k = nl; k > pos; --k) l_ent[k] = l_ent[k - 1];
+            GSTM_LLOOP(for (int k = nl; k > pos; --k) l_ent[k] = l_ent[k - 1];);
             l_ent[pos] = e;
             ++nl;
         }
@@ -203,9 +221,24 @@ struct Tx {
 #pragma unroll
             for (int k = 0; k < RCAP; ++k)
                 if (k < nr) ok &= (cur[k] == r_val[k]);
-        } else {
+        } else if constexpr (!kCompact) {
             for (int k = 0; k < nr; ++k)
                 ok &= (prim::ld_relaxed(m.val_ptr(r_addr[k])) == r_val[k]);
+        } else {
+            // compact: kPvWidth loads in flight per chunk, one rolled copy per
+            // call site (three sites in HV: A3.l71, l.76 and PostValidation's
+            // l.9 -- code size is what the HT kernel's instruction fetch pays
+            // for)
+#pragma unroll 1
+            for (int k0 = 0; k0 < nr; k0 += kPvWidth) {
+                uint32_t cur[kPvWidth];
+#pragma unroll
+                for (int j = 0; j < kPvWidth; ++j)
+                    if (k0 + j < nr) cur[j] = prim::ld_relaxed(m.val_ptr(r_addr[k0 + j]));
+#pragma unroll
+                for (int j = 0; j < kPvWidth; ++j)
+                    if (k0 + j < nr) ok &= (cur[j] == r_val[k0 + j]);
+            }
         }
         return ok;
     }
@@ -234,18 +267,18 @@ struct Tx {
                         again = true;                                // l.19 goto loop
                     }
             } else {
-                for (int k0 = 0; k0 < nr; k0 += 8) {                 // 8 lock loads in flight
-                    uint32_t vl[8];
+                GSTM_LLOOP(for (int k0 = 0; k0 < nr; k0 += kPvWidth) {   // kPvWidth lock loads in flight
+                    uint32_t vl[kPvWidth];
 #pragma unroll
-                    for (int j = 0; j < 8; ++j)
+                    for (int j = 0; j < kPvWidth; ++j)
                         if (k0 + j < nr) vl[j] = prim::ld_relaxed(m.lock_ptr(m.lock_of(r_addr[k0 + j])));
 #pragma unroll
-                    for (int j = 0; j < 8; ++j)
+                    for (int j = 0; j < kPvWidth; ++j)
                         if (k0 + j < nr && ((vl[j] & 1u) || (vl[j] >> 1) > snapshot)) {
                             newsnap = max(newsnap, vl[j] >> 1);
                             again = true;
                         }
-                }
+                });
             }
             snapshot = newsnap;
             if (!again) return true;                                 // l.20
@@ -365,9 +398,22 @@ struct Tx {
                 if (need[k]) newest = max(newest, vl[k] >> 1);
             check_version(m, newest, mode);                          // l.30-33 (Q35)
             reconverge();
+            if constexpr (kUnroll) {
 #pragma unroll
-            for (int k = 0; k < N; ++k)
-                if (need[k]) insert_lock((m.lock_of(a[k]) << 2) | 1u);   // l.34
+                for (int k = 0; k < N; ++k)
+                    if (need[k]) insert_lock((m.lock_of(a[k]) << 2) | 1u);   // l.34
+            } else {
+                // local-memory logs: one inlined copy of the (looping) insert
+#pragma unroll 1
+                for (int k = 0; k < N; ++k) {
+                    uint32_t ak = 0;
+                    bool nk = false;
+#pragma unroll
+                    for (int j = 0; j < N; ++j)
+                        if (j == k) { ak = a[j]; nk = need[j]; }
+                    if (nk) insert_lock((m.lock_of(ak) << 2) | 1u);  // l.34
+                }
+            }
         } else {
             uint32_t newest = 0;
 #pragma unroll
@@ -449,7 +495,7 @@ struct Tx {
             for (int k = 0; k < LCAP; ++k)
                 if (k < n_acq) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]);
         } else {
-            for (int k = 0; k < n_acq; ++k) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]);
+            GSTM_LLOOP(for (int k = 0; k < n_acq; ++k) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]););
         }
         n_acq = 0;
     }
@@ -600,13 +646,13 @@ struct Tx {
         }
         prim::fence_acquire();
         if (!ok) {
-            for (int k = 0; k < nl; ++k)                             // l.47: undo what we set
-                if (!(l_old[k] & 1u)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]);
+            GSTM_LLOOP(for (int k = 0; k < nl; ++k)                  // l.47: undo what we set
+                if (!(l_old[k] & 1u)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]););
             n_acq = 0;
             return false;
         }
-        for (int k = 0; k < nl; ++k)
-            if ((l_ent[k] & 1u) && (l_old[k] >> 1) > snapshot) passTBV = false;   // l.49-51
+        GSTM_LLOOP(for (int k = 0; k < nl; ++k)
+            if ((l_ent[k] & 1u) && (l_old[k] >> 1) > snapshot) passTBV = false;);   // l.49-51
         n_acq = nl;
         return true;
     }
@@ -644,7 +690,7 @@ struct Tx {
             for (int k = 0; k < WCAP; ++k)
                 if (k < nw) prim::st_relaxed(m.val_ptr(w_addr[k]), w_val[k]);
         } else {
-            for (int k = 0; k < nw; ++k) prim::st_relaxed(m.val_ptr(w_addr[k]), w_val[k]);
+            GSTM_LLOOP(for (int k = 0; k < nw; ++k) prim::st_relaxed(m.val_ptr(w_addr[k]), w_val[k]););
         }
         prim::fence_release();                                       // l.82
     }
@@ -680,8 +726,8 @@ struct Tx {
             for (int k = 0; k < LCAP; ++k)
                 if (k < nl) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
         } else {
-            for (int k = 0; k < nl; ++k)
-                prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]);
+            GSTM_LLOOP(for (int k = 0; k < nl; ++k)
+                prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), (l_ent[k] & 2u) ? (version << 1) : l_old[k]););
         }
         n_acq = 0;
     }

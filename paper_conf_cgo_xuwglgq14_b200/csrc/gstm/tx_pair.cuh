@@ -21,9 +21,9 @@
 
 namespace gstm {
 
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true>
-struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED> {
-    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED>;
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT>;
     using B::kUnroll;
     using B::r_addr;
     using B::r_val;

@@ -12,6 +12,8 @@
 // (gen.cuh), so an aborted transaction re-executes identically.
 #pragma once
 #include <cstdint>
+#include <type_traits>
+#include <utility>
 #include "gen.cuh"
 #include "prim.cuh"
 #include "tx.cuh"
@@ -32,6 +34,13 @@ struct WlParams {
 };
 
 // ---- contexts --------------------------------------------------------------
+// does the transaction type carry the warp-convergence mask (Tx, TxPair; not
+// TxVbv, whose lanes run independently)?
+template <class T, class = void>
+struct HasSyncMask : std::false_type {};
+template <class T>
+struct HasSyncMask<T, std::void_t<decltype(std::declval<T&>().sync_mask)>> : std::true_type {};
+
 template <class TX>
 struct StmCtx {
     TX& tx;
@@ -54,6 +63,18 @@ struct StmCtx {
     __device__ __forceinline__ void invalid() { tx.opaque = false; }
     // the transaction needs more log entries than compiled in: sticky error
     __device__ __forceinline__ void overflow() { tx.overflow = true; tx.opaque = false; }
+    // lanes of the warp that run this body together (stm_kernels.cuh,
+    // WL::kLockstep / kConvergent); 0 = unknown (then no warp-collective step)
+    __device__ __forceinline__ unsigned lockstep_mask() const
+    {
+        if constexpr (HasSyncMask<TX>::value) return tx.sync_mask;
+        else return 0u;
+    }
+    // the lanes that make the next read_batch call together (its reconverge)
+    __device__ __forceinline__ void set_sync_mask(unsigned m)
+    {
+        if constexpr (HasSyncMask<TX>::value) tx.sync_mask = m;
+    }
     static constexpr int kMaxChain = (TX::kRcap - 1) / 2;
 };
 
@@ -78,6 +99,8 @@ struct DirectCtx {
     __device__ __forceinline__ bool ok() const { return !bad; }
     __device__ __forceinline__ void invalid() { bad = true; }
     __device__ __forceinline__ void overflow() { bad = true; }
+    __device__ __forceinline__ unsigned lockstep_mask() const { return 0u; }
+    __device__ __forceinline__ void set_sync_mask(unsigned) {}
     static constexpr int kMaxChain = 1 << 30;
 };
 
@@ -249,8 +272,15 @@ struct BankWL {
 // heap = [heads B | key[M] | next[M]], node n (1..M) of tx_id = n-1; 0 = null.
 struct HtWL {
     static constexpr int MAXCHAIN = 24;
+    static constexpr bool kLockstep = true;     // chain walks in warp lockstep (body uses lockstep_mask)
     static constexpr int RCAP = 1 + 2 * MAXCHAIN, WCAP = 3, LCAP = RCAP + WCAP, FGL_LCAP = 1;
-    static constexpr int kMinBlocks = 2;
+    // code size is the HT kernel's limit (instruction fetch stalls, DESIGN.md
+    // §6.9): rolled log loops; 64 registers for 4 blocks (32 warps) per SM
+    static constexpr bool kCompact = true;
+#ifndef GSTM_HT_MINB
+#define GSTM_HT_MINB 4
+#endif
+    static constexpr int kMinBlocks = GSTM_HT_MINB;
     static constexpr int DESCR = 3;
     __host__ static bool check(const WlParams& p)
     {
@@ -283,20 +313,47 @@ struct HtWL {
     {
         uint32_t key, ins, bucket;
         key_of(p, x, key, ins, bucket);
-        if (key == 0) { c.overflow(); return; }        // no owned key drawn (never in practice)
         const uint64_t B = p.ht_buckets, M = p.T * p.K;
-        const uint32_t h0 = c.read(bucket);
-        if (!c.ok()) return;
-        uint32_t h = h0, found = 0;
-        for (int steps = 0; h != 0; ++steps) {
-            if (h > M) { c.invalid(); return; }
-            if (steps >= Ctx::kMaxChain) { c.overflow(); return; }
-            uint32_t a[2] = {static_cast<uint32_t>(B + h - 1), static_cast<uint32_t>(B + M + h - 1)}, v[2];
-            c.template read_batch<2>(a, v, 2);            // key[h], next[h]
-            if (!c.ok()) return;
-            if (v[0] == key) { found = 1; break; }
-            h = v[1];
+        // lanes that run their bodies together walk their chains in lockstep:
+        // one warp-collective step per chain node, so a step's loads, lock
+        // checks and log inserts are executed once for every walking lane
+        // instead of once per group of lanes that drifted apart (no lane
+        // leaves the loop before the warp agrees every walk is over)
+        const unsigned mask = c.lockstep_mask();
+        bool live = key != 0;
+        if (!live) c.overflow();                      // no owned key drawn (never in practice)
+        // one TXRead call site for the whole walk (step 0: the bucket head;
+        // step s > 0: key and next of the s-th node), so PostValidation and
+        // the lock spin are inlined once
+        uint32_t h0 = 0, h = 0, found = 0;
+        bool walking = live;
+        for (int steps = 0;; ++steps) {
+            if (walking && steps > 0 && h > M) { c.invalid(); walking = live = false; }
+            if (walking && steps > Ctx::kMaxChain) { c.overflow(); walking = live = false; }
+            const unsigned wm = mask ? __ballot_sync(mask, walking) : (walking ? 1u : 0u);
+            if (!wm) break;
+            if (walking) {
+                uint32_t a[2], v[2];
+                a[0] = steps ? static_cast<uint32_t>(B + h - 1) : bucket;          // key[h] / head
+                a[1] = static_cast<uint32_t>(B + M + h - 1);                      // next[h]
+                if (mask) c.set_sync_mask(wm);               // read_batch reconverges the walking lanes
+                c.template read_batch<2>(a, v, steps ? 2 : 1);
+                if (!c.ok()) {
+                    walking = live = false;
+                } else if (steps == 0) {
+                    h0 = h = v[0];
+                    walking = h != 0;
+                } else if (v[0] == key) {
+                    found = 1;
+                    walking = false;
+                } else {
+                    h = v[1];
+                    walking = h != 0;
+                }
+            }
         }
+        if (mask) c.set_sync_mask(0u);
+        if (!live) return;
         if (!ins) { result = found; return; }
         if (found) { result = 2; return; }
         const uint32_t n = static_cast<uint32_t>(1 + i * p.T + t);

@@ -38,6 +38,19 @@ struct Convergent { static constexpr bool value = false; };
 template <class WL>
 struct Convergent<WL, std::void_t<decltype(WL::kConvergent)>> { static constexpr bool value = WL::kConvergent; };
 
+// WL::kLockstep (optional): the body runs warp-collective steps over the
+// lanes that start bodies together (StmCtx::lockstep_mask, the HT chain walk)
+template <class WL, class = void>
+struct Lockstep { static constexpr bool value = false; };
+template <class WL>
+struct Lockstep<WL, std::void_t<decltype(WL::kLockstep)>> { static constexpr bool value = WL::kLockstep; };
+
+// WL::kCompact (optional): rolled log loops, 4-wide validation (Tx COMPACT)
+template <class WL, class = void>
+struct Compact { static constexpr bool value = false; };
+template <class WL>
+struct Compact<WL, std::void_t<decltype(WL::kCompact)>> { static constexpr bool value = WL::kCompact; };
+
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
@@ -127,7 +140,7 @@ struct Counters {
 __device__ __forceinline__ void flush_counters(Counters& cnt, unsigned long long* stats)
 {
     __syncwarp();
-#pragma unroll
+#pragma unroll 1
     for (int k = 0; k < S_NSTATS; ++k) {
         unsigned long long v = cnt.sh[k * kMaxBlock + threadIdx.x];
 #pragma unroll
@@ -196,8 +209,8 @@ template <class WL, int MODE, bool PAIR, int POL = POL_SORTED>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
     constexpr bool kSorted = POL == POL_SORTED;
-    using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted>,
-                                  Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted>>;
+    using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value>,
+                                  Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value>>;
     // The grid is persistent (host sizes it to what fits on the chip, or to
     // p.max_threads): lane g runs STM threads g, g+P, ... g+(Rs-1)P of the
     // static region [0, S = Rs*P), Rs = max(1, T/P - 1) rounds, with no
@@ -237,34 +250,61 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
         have_snap = false;
         PHASE_MARK(PH_BEGIN);
-        const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
-        bool done = false, skip = false;
-        const unsigned body_mask = Convergent<WL>::value ? __ballot_sync(FULL, act && stage == 0) : 0u;
-        if (act && stage == 0) {
-            cnt.inc(S_ATTEMPTS);
-            result = 0;
-            const uint64_t x = gen::tx_key(p.seed, t, i);
-            tx.begin(snap);                                           // TXBegin l.2-3
-            tx.sync_mask = body_mask;
-            StmCtx<TX> ctx{tx, m, MODE};
-            WL::body(ctx, p.w, x, t, i, result);                     // TXRead / TXWrite
-            if (!tx.opaque) {
-                if (tx.overflow) { cnt.inc(S_ERRORS); skip = true; }  // sticky ELOGOVF, give up this tx
-                else cnt.inc(S_AB_OPACITY);                          // Figure 1 / Q11
-            } else if (tx.read_only()) {                              // l.68: linearized at snapshot
-                if (p.tx_stamp) {
-                    p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
-                    p.tx_result[tx_id] = result;
+        bool done = false, aborted = false;
+        // Body rounds (p.body_rounds): a lane whose
+        // transaction committed read-only (A3.l68: no locks, no stamp) starts
+        // its next transaction in the same warp iteration, up to body_rounds
+        // bodies, so lanes of a mostly read-only workload (HT: 90% lookups) do
+        // not idle through the commit round of the warp's few update lanes.
+        // Every round uses the iteration's snapshot (a valid, older one: more
+        // validation at worst).  A lane that aborted, or holds an update to
+        // commit, sits out the later rounds.
+        bool cont = act && stage == 0;
+        // a lane's next transaction starts no earlier than where its last one
+        // was linearised (PostValidation may have raised that snapshot above
+        // the iteration's): per-thread real-time order
+        uint32_t lane_snap = snap;
+        for (uint32_t round = 0;; ++round) {
+            const bool run = cont && i < p.K;
+            if (round > 0 && (round >= p.body_rounds || !__any_sync(FULL, run))) break;
+            cont = false;
+            const unsigned body_mask =
+                (Convergent<WL>::value || Lockstep<WL>::value) ? __ballot_sync(FULL, run) : 0u;
+            if (run) {
+                const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
+                bool next = false;
+                cnt.inc(S_ATTEMPTS);
+                result = 0;
+                const uint64_t x = gen::tx_key(p.seed, t, i);
+                tx.begin(lane_snap);                                  // TXBegin l.2-3
+                tx.sync_mask = body_mask;
+                StmCtx<TX> ctx{tx, m, MODE};
+                WL::body(ctx, p.w, x, t, i, result);                 // TXRead / TXWrite
+                if (!tx.opaque) {
+                    if (tx.overflow) { cnt.inc(S_ERRORS); next = true; }  // sticky ELOGOVF, give up this tx
+                    else { cnt.inc(S_AB_OPACITY); aborted = true; }  // Figure 1 / Q11
+                } else if (tx.read_only()) {                          // l.68: linearized at snapshot
+                    if (p.tx_stamp) {
+                        p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
+                        p.tx_result[tx_id] = result;
+                    }
+                    cnt.inc(S_COMMITS_RO);
+                    cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
+                    next = true;
+                    cont = true;
+                    lane_snap = tx.snapshot;
+                } else {
+                    stage = 1;
+                    // STM-HV-Backoff: an execution that follows a lock abort goes
+                    // straight to the sequential step -- its parallel attempt
+                    // already failed
+                    tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
                 }
-                cnt.inc(S_COMMITS_RO);
-                cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
-                done = true;
-            } else {
-                stage = 1;
-                // STM-HV-Backoff: an execution that follows a lock abort goes
-                // straight to the sequential step -- its parallel attempt
-                // already failed
-                tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
+                if (next) {                                           // the next transaction of thread t
+                    ++i;
+                    backoff = 0;
+                    lock_aborts = 0;
+                }
             }
         }
         PHASE_MARK(PH_BODY);
@@ -303,11 +343,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     tries = 1;                                        // -> the sequential step below
                 } else if (p.k_lock && tries >= p.k_lock) {
                     stage = 0;
+                    aborted = true;
                     ++lock_aborts;
                     cnt.inc(S_AB_LOCK);
                 }
             } else {
                 stage = 0;
+                aborted = true;
                 cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
             }
         }
@@ -319,6 +361,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         if (got) {
             tx.release_and_update(m, stamp);                          // l.84
             if (p.tx_stamp) {
+                const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
                 p.tx_stamp[tx_id] = stamp - clock_begin;
                 p.tx_result[tx_id] = result;
             }
@@ -361,6 +404,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                         sl = static_cast<uint32_t>(clock_fetch_add(m.clock, 1u)) + 1u;   // l.83
                         tx.release_and_update(m, sl);                 // l.84
                         if (p.tx_stamp) {
+                            const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
                             p.tx_stamp[tx_id] = sl - clock_begin;
                             p.tx_result[tx_id] = result;
                         }
@@ -374,11 +418,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                         seq_failed = true;
                         if (p.k_lock && ++tries > p.k_lock) {
                             stage = 0;
+                            aborted = true;
                             ++lock_aborts;
                             cnt.inc(S_AB_LOCK);
                         }
                     } else {
                         stage = 0;
+                        aborted = true;
                         cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
                     }
                 }
@@ -389,12 +435,12 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             seq_fails = seq_failed ? seq_fails + 1u : 0u;
         }
         PHASE_MARK(PH_RELEASE);
-        if (done || skip) {
+        if (done) {
             stage = 0;
             ++i;
             backoff = 0;
             lock_aborts = 0;
-        } else if (p.backoff_ns && act && stage == 0) {
+        } else if (p.backoff_ns && aborted) {
             // exponential backoff after an abort (P:111 argues per-lane
             // delays cannot work under SIMT; lanes here sleep independently
             // under independent thread scheduling)

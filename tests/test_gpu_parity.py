@@ -318,6 +318,24 @@ def test_livelock_freedom_two_words(mode, k_lock, pipeline):
     assert st.commits == T * K
 
 
+@pytest.mark.parametrize("mode", ["hv", "tbv", "hv_backoff"])
+@pytest.mark.parametrize("wl,kw,T,K,bits", [
+    ("ht", dict(ht_buckets=1 << 12, ht_key_range=1 << 14, ht_lookup_pct=90), 1 << 14, 4, 14),
+    ("ht", dict(ht_buckets=64, ht_key_range=256, ht_lookup_pct=50), 2048, 4, 8),
+    ("bank", dict(n_words=1 << 10), 1 << 14, 4, 10),
+    ("ra", dict(n_reads=4, n_writes=4, n_words=1024), 256, 64, 10),
+])
+@pytest.mark.parametrize("rounds", [2, 8])
+def test_body_rounds_replay(mode, wl, kw, T, K, bits, rounds):
+    """body_rounds: lanes that commit read-only run their
+    next transaction in the same warp iteration, with the iteration's
+    snapshot.  Serializability (stamp-order replay, read-only transactions at
+    their snapshot) and each thread's program order must hold."""
+    g, gp, op, init = U.make(wl, T, K, bits, mode=mode, body_rounds=rounds, **kw)
+    U.run_verified(g, wl, op, init, T, K, 5 + rounds)
+    g.close()
+
+
 @pytest.mark.parametrize("paired", [False, True])
 @pytest.mark.parametrize("mode", ["hv", "tbv"])
 @pytest.mark.parametrize("pipeline", [1, 1000])
