@@ -258,12 +258,16 @@ int gstm_stats(gstm_t* h, gstm_stats_t* out);
  * the first error any of them reported. */
 int gstm_stats_total(gstm_t* h, gstm_stats_t* out, uint64_t* launches);
 int gstm_reset_stats_total(gstm_t* h);
-/* Per-phase time breakdown of the STM loop since gstm_reset_stats_total
- * (the paper's Figure 5 study): SM cycles summed over warps for
- * out[0] TXBegin/snapshot, [1] transaction body (reads, PostValidation, lock
- * spins), [2] lock acquisition + validation, [3] commit stamp, [4] write-back
- * and release, [5] loop/refill.  Non-zero only in a library built with
- * -DGSTM_PHASE_TIMING=1 (GSTM_DEFINES); writes min(n, 8) entries. */
+/* Execution-time breakdown of the STM kernels since gstm_reset_stats_total
+ * (the paper's Figure 5): SM cycles summed over every lane (each
+ * lane times its own path) in Figure 5's categories: out[0] native code,
+ * [1] transaction initialisation, [2] buffering (read/write/lock logging),
+ * [3] consistency checking (lock-word checks, spins, PostValidation, VBV),
+ * [4] acquiring/releasing locks, [5] committing (write-back, clock stamp),
+ * [6] aborted transactions (every cycle of an execution that aborted), [7]
+ * other (loop, refill, SIMT waiting outside a transaction).  Non-zero only in
+ * the "phase" build flavour (lib/libgstm_phase.so, -DGSTM_PHASE_TIMING=1);
+ * writes min(n, 16) entries. */
 int gstm_phase_cycles(gstm_t* h, uint64_t* out, int n);
 /* Verify mode (params.verify = 1): stamps[tx_id] = commit stamp - clock_begin
  * (1..C) for an update tx, or 0x80000000 | (snapshot - clock_begin) for a
@@ -322,11 +326,13 @@ int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per
  * with op 0 BEGIN, 1 READ, 2 WRITE, 3 COMMIT; out: n_ops x 4 words (format in
  * DESIGN.md §5.3).  mode: GSTM_MODE_HV or GSTM_MODE_TBV. */
 int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx);
-/* Insert entries (id<<2 | wr<<1 | rd) into a device lock log (variant 0:
- * register-resident, capacity 16; 1: local memory, capacity 256; both sorted
- * by id.  Variants 2 and 3: the same capacities in encounter
- * order, the lock order of GSTM_MODE_HV_BACKOFF / GSTM_MODE_HV_UNSORTED) and
- * return the resulting log in out; returns its length or a negative error. */
+/* Insert entries (id<<2 | wr<<1 | rd, id < 2^20) into a device lock log
+ * (variant 0: register-resident, capacity 16; 1: local memory, capacity 256;
+ * both sorted by id.  Variants 2 and 3: the same capacities in
+ * encounter order, the lock order of GSTM_MODE_HV_BACKOFF /
+ * GSTM_MODE_HV_UNSORTED.  Variants 4 and 5: the order-preserving hashed log
+ * of P:115 in local memory, capacity 16 / 256) and return the resulting log
+ * in out; returns its length or a negative error. */
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant);
 /* Roofline microbenchmark: kind 0 random atom.or, 1
  * same-address atom.add.u64, 2 random ld.relaxed, 3 random st.relaxed, 4

@@ -33,19 +33,34 @@ def nvcc() -> str:
     raise RuntimeError("nvcc not found")
 
 
-def _stale() -> bool:
-    if not os.path.exists(SO):
+# build flavours: lib/libgstm_<name>.so with extra defines (tests and tools
+# load them by name, gstm.lib(flavour)); "" is the product library
+FLAVOURS = {
+    "": [],
+    "strict": ["-DGSTM_STRICT_FENCES=1"],      # every fence the formal PTX model asks for
+    "hlog": ["-DGSTM_HLOG=1"],                 # order-preserving hashed lock logs
+    "phase": ["-DGSTM_PHASE_TIMING=1"],        # Figure 5 per-phase cycle counters
+}
+
+
+def so_path(flavour: str = "") -> str:
+    return os.path.join(LIBDIR, f"libgstm_{flavour}.so" if flavour else "libgstm.so")
+
+
+def _stale(so: str = SO) -> bool:
+    if not os.path.exists(so):
         return True
     deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS] + [os.path.join(ROOT, "include", "gstm.h"),
                                                                  os.path.abspath(__file__)]
-    return max(os.path.getmtime(d) for d in deps) > os.path.getmtime(SO)
+    return max(os.path.getmtime(d) for d in deps) > os.path.getmtime(so)
 
 
-def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = False) -> str:
-    if not force and not _stale():
-        return SO
+def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = False, flavour: str = "") -> str:
+    so = so_path(flavour)
+    if not force and not _stale(so):
+        return so
     os.makedirs(LIBDIR, exist_ok=True)
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(HERE, "build", flavour or "default")
     os.makedirs(objdir, exist_ok=True)
     objs = []
     procs = []
@@ -53,8 +68,10 @@ def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = Fals
         obj = os.path.join(objdir, src.replace(".cu", ".o"))
         cmd = [nvcc()] + ARCH + FLAGS + ["-I", os.path.join(ROOT, "include"), "-I", CSRC, "-c",
                                          os.path.join(CSRC, src), "-o", obj]
-        # e.g. GSTM_DEFINES="-DGSTM_STRICT_FENCES=1" (ablation builds; use --force)
-        cmd += os.environ.get("GSTM_DEFINES", "").split()
+        cmd += FLAVOURS[flavour]
+        # e.g. GSTM_DEFINES="-DGSTM_HT_MINB=3" (ablation builds of the product library; use --force)
+        if not flavour:
+            cmd += os.environ.get("GSTM_DEFINES", "").split()
         if ptxas_verbose:
             cmd += ["-Xptxas", "-v"]
         if verbose:
@@ -69,11 +86,15 @@ def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = Fals
         failed |= p.returncode != 0
     if failed:
         raise RuntimeError("nvcc failed")
-    tmp = SO + f".tmp{os.getpid()}"
+    tmp = so + f".tmp{os.getpid()}"
     cmd = [nvcc()] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs
     subprocess.check_call(cmd)
-    os.replace(tmp, SO)
-    return SO
+    os.replace(tmp, so)
+    return so
+
+
+def build_all(force: bool = False) -> list:
+    return [build(force=force, flavour=f) for f in FLAVOURS]
 
 
 if __name__ == "__main__":
@@ -81,5 +102,9 @@ if __name__ == "__main__":
     ap.add_argument("--force", action="store_true")
     ap.add_argument("--verbose", action="store_true")
     ap.add_argument("--ptxas", action="store_true")
+    ap.add_argument("--flavour", default="", choices=list(FLAVOURS) + ["all"])
     a = ap.parse_args()
-    print(build(force=a.force, verbose=a.verbose, ptxas_verbose=a.ptxas))
+    if a.flavour == "all":
+        print("\n".join(build_all(force=a.force)))
+    else:
+        print(build(force=a.force, verbose=a.verbose, ptxas_verbose=a.ptxas, flavour=a.flavour))

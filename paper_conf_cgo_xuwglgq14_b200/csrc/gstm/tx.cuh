@@ -37,7 +37,22 @@
         }                                                      \
     } while (0)
 
+// Figure 5 execution-time breakdown: build with
+// -DGSTM_PHASE_TIMING=1 (the "phase" library flavour).  Every lane times its
+// own path with clock64() and attributes the cycles to the paper's seven
+// categories -- native code, transaction initialisation, buffering (read/write
+// logging), consistency checking (lock-word checks, spins, PostValidation,
+// VBV), acquiring/releasing locks, committing (write-back, clock stamp) and
+// aborted transactions (every cycle of an execution that aborted) -- plus
+// "other" (loop, refill, SIMT waiting outside a transaction).
+#ifndef GSTM_PHASE_TIMING
+#define GSTM_PHASE_TIMING 0
+#endif
+
 namespace gstm {
+
+enum { PH_NATIVE = 0, PH_INIT, PH_BUFFER, PH_CONSIST, PH_LOCKS, PH_COMMIT, PH_TX_N, PH_ABORTED = PH_TX_N, PH_OTHER,
+       PH_N };
 
 enum { MODE_HV = 1, MODE_TBV = 2 };
 
@@ -88,7 +103,9 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
 // `#pragma unroll 1`; validation loads 4 in flight) -- for kernels whose code
 // outgrows the instruction cache (HT: DESIGN.md §6.9); else the compiler
 // unrolls them (by 4) and validation keeps 8 loads in flight.
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false>
+// HLOG = true (local-memory logs, sorted): the lock log is the order-preserving
+// hash table of P:115 instead of one sorted array.
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false, bool HLOG = false>
 struct Tx {
     // register-resident (unrolled) logs for small capacities unless the
     // workload asks for local memory (LOCAL: fewer registers, more warps)
@@ -97,11 +114,58 @@ struct Tx {
     static constexpr bool kCompact = COMPACT;
     // value / lock-word loads validation keeps in flight with local-memory logs
     static constexpr int kPvWidth = COMPACT ? 4 : 8;
+    // order-preserving hashed lock log: kHs home slots (load factor
+    // <= 1/2), then LCAP overflow slots (an entry never sits more than
+    // LCAP - 1 slots past its home); occupancy bitmap in registers
+    static constexpr bool kHlog = HLOG && SORTED && !kUnroll;
+    static constexpr int kHs = 2 * LCAP;
+    static constexpr int kTs = kHlog ? kHs + LCAP : LCAP;
+    static constexpr int kBw = kHlog ? (kTs + 31) / 32 : 1;
 
     uint32_t r_addr[RCAP], r_val[RCAP];   // read-set  <addr,val>
     uint32_t w_addr[WCAP], w_val[WCAP];   // write-set <addr,val> (redo log)
-    uint32_t l_ent[LCAP], l_old[LCAP];    // sorted lock log; old lock words
+    uint32_t l_ent[kTs], l_old[LCAP];     // sorted lock log (hashed: the table); old lock words
+    uint32_t occ[kBw];                    // hashed log: occupied slots
+    uint32_t id_shift = 12;               // hashed log: 32 - lock-table bits (home = id's top bits)
+    bool compacted;                       // hashed log: l_ent[0, nl) is the dense sorted log
     unsigned long long bloom;
+#if GSTM_PHASE_TIMING
+    uint32_t ph_acc[PH_TX_N];             // cycles of the current execution by category
+    unsigned long long ph_tot[PH_N];      // totals (aborted executions summed into PH_ABORTED)
+    int ph_cur = PH_OTHER;
+    long long ph_t = 0;
+    __device__ __forceinline__ void ph_init()
+    {
+        for (int k = 0; k < PH_TX_N; ++k) ph_acc[k] = 0u;
+        for (int k = 0; k < PH_N; ++k) ph_tot[k] = 0ull;
+        ph_cur = PH_OTHER;
+        ph_t = clock64();
+    }
+    // the lane enters category k: the cycles since the last switch go to the
+    // category it leaves
+    __device__ __forceinline__ void ph(int k)
+    {
+        const long long now = clock64();
+        if (ph_cur < PH_TX_N) ph_acc[ph_cur] += static_cast<uint32_t>(now - ph_t);
+        else ph_tot[ph_cur] += static_cast<unsigned long long>(now - ph_t);
+        ph_t = now;
+        ph_cur = k;
+    }
+    // the execution ended: committed -> its cycles by category; aborted ->
+    // all of them into PH_ABORTED
+    __device__ __forceinline__ void ph_end(bool committed)
+    {
+        ph(PH_OTHER);
+        for (int k = 0; k < PH_TX_N; ++k) {
+            ph_tot[committed ? k : static_cast<int>(PH_ABORTED)] += ph_acc[k];
+            ph_acc[k] = 0u;
+        }
+    }
+#else
+    __device__ __forceinline__ void ph_init() {}
+    __device__ __forceinline__ void ph(int) {}
+    __device__ __forceinline__ void ph_end(bool) {}
+#endif
     int nr, nw, nl, n_acq;
     uint32_t snapshot;
     bool opaque, passTBV, overflow;
@@ -122,7 +186,15 @@ struct Tx {
         overflow = false;
         snapshot = snap;                          // l.4
         sync_mask = 0u;
+        if constexpr (kHlog) {
+#pragma unroll
+            for (int k = 0; k < kBw; ++k) occ[k] = 0u;
+            compacted = false;
+        }
     }
+
+    // hashed log: ids are lock-table indices < 2^bits
+    __device__ __forceinline__ void set_id_bits(uint32_t bits) { id_shift = 32u - bits; }
 
     // Reconverge the lanes that run their bodies together after a rare,
     // per-lane path (a lock spin, PostValidation): without it the warp stays
@@ -164,11 +236,81 @@ struct Tx {
         ++nr;
     }
 
+    // ---- hashed log helpers: the occupancy bitmap stays in registers ------
+    __device__ __forceinline__ uint32_t occ_word(int w) const
+    {
+        uint32_t v = 0u;
+#pragma unroll
+        for (int k = 0; k < kBw; ++k)
+            if (k == w) v = occ[k];
+        return v;
+    }
+    __device__ __forceinline__ bool occ_test(int sl) const { return (occ_word(sl >> 5) >> (sl & 31)) & 1u; }
+    __device__ __forceinline__ void occ_set(int sl)
+    {
+#pragma unroll
+        for (int k = 0; k < kBw; ++k)
+            if (k == (sl >> 5)) occ[k] |= 1u << (sl & 31);
+    }
+
+    // ---- insert into the order-preserving hash table --------------
+    // Home slot = the id's top bits scaled to kHs slots (monotone in id); the
+    // occupied slots hold the entries in ascending id, each at or after its
+    // home.  An entry with id' > id can only sit at or after home(id), so the
+    // insert position is the first slot from home(id) that is empty or holds
+    // an id' >= id; the run of occupied slots from there shifts right by one
+    // (into the first empty slot).  Expected O(1) comparisons and moves
+    // instead of O(n) ("the number of comparison steps is reduced").
+    __device__ __forceinline__ void insert_lock_hashed(uint32_t e)
+    {
+        const uint32_t id = e >> 2;
+        int sl = id_shift >= 32u ? 0 : static_cast<int>(__umulhi(id << id_shift, static_cast<uint32_t>(kHs)));
+        bool occupied = occ_test(sl);
+        while (occupied && (l_ent[sl] >> 2) < id) occupied = occ_test(++sl);
+        if (occupied && (l_ent[sl] >> 2) == id) { l_ent[sl] |= (e & 3u); return; }   // Q4
+        if (nl >= LCAP) { overflow = true; opaque = false; return; }
+        int end = sl;                                        // first empty slot >= sl
+        if (occupied) {
+            int w = sl >> 5;
+            uint32_t free = ~occ_word(w) & (~0u << (sl & 31));
+            while (!free) free = ~occ_word(++w);
+            end = (w << 5) + __ffs(free) - 1;
+            GSTM_LLOOP(for (int k = end; k > sl; --k) l_ent[k] = l_ent[k - 1];);
+        }
+        occ_set(end);
+        l_ent[sl] = e;
+        ++nl;
+    }
+
+    // hashed log -> l_ent[0, nl) dense and ascending, for TXCommit (in place:
+    // the k-th occupied slot is at index >= k)
+    __device__ __forceinline__ void compact()
+    {
+        if constexpr (kHlog) {
+            if (compacted) return;
+            int j = 0;
+#pragma unroll
+            for (int w = 0; w < kBw; ++w) {
+                uint32_t b = occ[w];
+                while (b) {
+                    const int sl = (w << 5) + __ffs(b) - 1;
+                    b &= b - 1u;
+                    l_ent[j++] = l_ent[sl];
+                }
+            }
+            compacted = true;
+        }
+    }
+
     // ---- P:113-115, A3.l34/l38: sorted insert into the local lock log ----
     // Entries are id<<2 | wr<<1 | rd, ascending by id; a duplicate id only
     // ORs its bits (no new entry).
     __device__ __forceinline__ void insert_lock(uint32_t e)
     {
+        if constexpr (kHlog) {
+            insert_lock_hashed(e);
+            return;
+        }
         const uint32_t id = e >> 2;
         if constexpr (kUnroll) {
             int pos = 0;
@@ -323,13 +465,17 @@ struct Tx {
     __device__ __forceinline__ uint32_t read(const Meta& m, uint32_t a, int mode)
     {
         uint32_t v;
-        if (raw_lookup(a, v)) return v;                              // l.22-23
+        ph(PH_BUFFER);
+        if (raw_lookup(a, v)) { ph(PH_NATIVE); return v; }          // l.22-23
         v = prim::ld_relaxed(m.val_ptr(a));                            // l.24
         append_read(a, v);                                           // l.25
+        ph(PH_CONSIST);
         prim::fence_acquire();                                       // l.26
         const uint32_t vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));
         check_lock(m, a, vl, mode);                                  // l.27-33
+        ph(PH_BUFFER);
         insert_lock((m.lock_of(a) << 2) | 1u);                  // l.34
+        ph(PH_NATIVE);
         return v;                                                    // l.35
     }
 
@@ -352,6 +498,7 @@ struct Tx {
     {
         bool need[N];
         uint32_t vl[N];
+        ph(PH_BUFFER);
 #pragma unroll
         for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
 #pragma unroll
@@ -360,6 +507,7 @@ struct Tx {
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) append_read(a[k], v[k]);                    // l.25
+        ph(PH_CONSIST);
         prim::fence_acquire();                                       // l.26
 #pragma unroll
         for (int k = 0; k < N; ++k)
@@ -398,6 +546,7 @@ struct Tx {
                 if (need[k]) newest = max(newest, vl[k] >> 1);
             check_version(m, newest, mode);                          // l.30-33 (Q35)
             reconverge();
+            ph(PH_BUFFER);
             if constexpr (kUnroll) {
 #pragma unroll
                 for (int k = 0; k < N; ++k)
@@ -422,6 +571,7 @@ struct Tx {
             reconverge();
             check_version(m, newest, mode);                          // l.31-33
             reconverge();
+            ph(PH_BUFFER);
 #pragma unroll 1
             for (int k = 0; k < N; ++k) {
                 uint32_t ak = 0;
@@ -432,6 +582,7 @@ struct Tx {
                 if (nk) insert_lock((m.lock_of(ak) << 2) | 1u);
             }
         }
+        ph(PH_NATIVE);
     }
 
     // Batched TXRead of n words (n only known at run time; arrays in local
@@ -442,24 +593,35 @@ struct Tx {
                                               int mode)
     {
         uint32_t vl[kRcap];
+        ph(PH_BUFFER);
 #pragma unroll 8
         for (int k = 0; k < n; ++k)
             if (!skip[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));   // l.24
         for (int k = 0; k < n; ++k)
             if (!skip[k]) append_read(a[k], v[k]);                    // l.25
+        ph(PH_CONSIST);
         prim::fence_acquire();                                        // l.26
 #pragma unroll 8
         for (int k = 0; k < n; ++k)
             if (!skip[k]) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
         for (int k = 0; k < n; ++k)
             if (!skip[k]) {
+                ph(PH_CONSIST);
                 check_lock(m, a[k], vl[k], mode);                     // l.27-33
+                ph(PH_BUFFER);
                 insert_lock((m.lock_of(a[k]) << 2) | 1u);             // l.34
             }
+        ph(PH_NATIVE);
     }
 
     // ---- A3.l36-38 TXWrite(addr, val): upsert, bloom, sorted lock insert --
     __device__ __forceinline__ void write(const Meta& m, uint32_t a, uint32_t v)
+    {
+        ph(PH_BUFFER);
+        write_log(m, a, v);
+        ph(PH_NATIVE);
+    }
+    __device__ __forceinline__ void write_log(const Meta& m, uint32_t a, uint32_t v)
     {
         bool found = false;
         if (bloom & bloom_bit(a)) {
@@ -506,6 +668,7 @@ struct Tx {
     // makes lockstep retry livelock-free.
     __device__ __forceinline__ bool get_locks_and_tbv(const Meta& m)
     {
+        compact();
         n_acq = 0;
         bool ok = true;
         if constexpr (kUnroll) {
@@ -662,16 +825,24 @@ struct Tx {
     // (nothing held; retry, l.73-74), or an abort cause (nothing held).
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
+        ph(PH_BUFFER);
+        compact();
+        ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
+        ph(PH_LOCKS);
         bool got;
         if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
         else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18
-            if (!vbv(m)) { release_locks(m); return C_COMMITVBV; }   // l.76-78
+            ph(PH_CONSIST);
+            const bool ok = vbv(m);
+            ph(PH_LOCKS);
+            if (!ok) { release_locks(m); return C_COMMITVBV; }       // l.76-78
         }
+        ph(PH_COMMIT);
         // l.79 threadfence: the acquiring atomics already returned (each
         // atom.acquire waits for its result), so no write-back below can be
         // performed before the locks are held; the strict build adds the
@@ -720,6 +891,7 @@ struct Tx {
     // the acquiring atomic returned (reading Q16: == lock - 1).
     __device__ __forceinline__ void release_and_update(const Meta& m, uint32_t version)
     {
+        ph(PH_LOCKS);
         if (GSTM_STRICT_FENCES) prim::fence_release();
         if constexpr (kUnroll) {
 #pragma unroll

@@ -21,9 +21,10 @@
 
 namespace gstm {
 
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false>
-struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
-    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT>;
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false,
+          bool HLOG = false>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG>;
     using B::kUnroll;
     using B::r_addr;
     using B::r_val;
@@ -45,6 +46,8 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
     using B::append_read;
     using B::reconverge;
     using B::insert_lock;
+    using B::kCompact;
+    using B::ph;
 
     uint32_t l_val[LCAP];   // value each acquiring atom.or.b64 returned
 
@@ -130,12 +133,19 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
     __device__ __forceinline__ uint32_t read(const Meta& m, uint32_t a, int mode)
     {
         uint32_t v;
-        if (raw_lookup(a, v)) return v;                              // l.22-23
-        const unsigned long long pv = settle(m, a, prim::ld_relaxed_u64(m.pair_ptr(a)));   // l.24, l.27-29
+        ph(PH_BUFFER);
+        if (raw_lookup(a, v)) { ph(PH_NATIVE); return v; }          // l.22-23
+        unsigned long long pv = prim::ld_relaxed_u64(m.pair_ptr(a)); // l.24 (+ l.28)
+        ph(PH_CONSIST);
+        pv = settle(m, a, pv);                                       // l.27-29
         v = lo(pv);
+        ph(PH_BUFFER);
         append_read(a, v);                                           // l.25
+        ph(PH_CONSIST);
         check_version(m, hi(pv), mode);                              // l.30-33
+        ph(PH_BUFFER);
         insert_lock((a << 2) | 1u);                                  // l.34 (lock id = word)
+        ph(PH_NATIVE);
         return v;
     }
 
@@ -144,11 +154,13 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
     {
         bool need[N];
         unsigned long long pv[N];
+        ph(PH_BUFFER);
 #pragma unroll
         for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));
+        ph(PH_CONSIST);
         if constexpr (N <= 4) {
             // small batches (bank: 2), fully unrolled: ONE spin loop re-reads
             // every still-locked pair of the batch together (l.27-29), and ONE
@@ -181,6 +193,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
                 }
             check_version(m, newest << 1, mode);                      // l.30-33 (Q35)
             reconverge();
+            ph(PH_BUFFER);
 #pragma unroll
             for (int k = 0; k < N; ++k)
                 if (need[k]) insert_lock((a[k] << 2) | 1u);          // l.34
@@ -198,6 +211,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
             // one merged timestamp check per batch (tx.cuh read_batch)
             check_version(m, newest << 1, mode);
             reconverge();
+            ph(PH_BUFFER);
 #pragma unroll 1
             for (int k = 0; k < N; ++k) {
                 uint32_t ak = 0;
@@ -208,12 +222,14 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
                 if (nk) insert_lock((ak << 2) | 1u);
             }
         }
+        ph(PH_NATIVE);
     }
 
     __device__ __forceinline__ void read_many(const Meta& m, const uint32_t* a, uint32_t* v, const bool* skip, int n,
                                               int mode)
     {
         uint32_t vl[RCAP];
+        ph(PH_BUFFER);
 #pragma unroll 8
         for (int k = 0; k < n; ++k)
             if (!skip[k]) {
@@ -224,17 +240,22 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
         for (int k = 0; k < n; ++k)
             if (!skip[k]) {
                 if (vl[k] & 1u) {
+                    ph(PH_CONSIST);
                     const unsigned long long pv = settle(m, a[k], mk(v[k], vl[k]));
                     v[k] = lo(pv);
                     vl[k] = hi(pv);
+                    ph(PH_BUFFER);
                 }
                 append_read(a[k], v[k]);
             }
         for (int k = 0; k < n; ++k)
             if (!skip[k]) {
+                ph(PH_CONSIST);
                 check_version(m, vl[k], mode);
+                ph(PH_BUFFER);
                 insert_lock((a[k] << 2) | 1u);
             }
+        ph(PH_NATIVE);
     }
 
     // ---- A3.l62-66 VBV from the values in memory --------------------------
@@ -299,6 +320,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
     // ---- A3.l43-52 GetLocksAndTBV, sequential in ascending id -------------
     __device__ __forceinline__ bool get_locks_and_tbv(const Meta& m)
     {
+        B::compact();
         n_acq = 0;
         bool ok = true;
         if constexpr (kUnroll) {
@@ -441,16 +463,24 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
 
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
+        ph(PH_BUFFER);
+        B::compact();
+        ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
+        ph(PH_LOCKS);
         bool got;
         if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
         else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; }
-            if (!vbv_locked()) { release_locks(m); return C_COMMITVBV; }   // l.76-78
+            ph(PH_CONSIST);
+            const bool ok = vbv_locked();
+            ph(PH_LOCKS);
+            if (!ok) { release_locks(m); return C_COMMITVBV; }       // l.76-78
         }
+        ph(PH_COMMIT);
         return C_OK;
     }
 
@@ -463,6 +493,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT> {
     //      pairs get back exactly what the atomic returned --------------------
     __device__ __forceinline__ void release_and_update(const Meta& m, uint32_t version)
     {
+        ph(PH_COMMIT);                   // the value write-back IS the release store here (l.80-84)
         if constexpr (kUnroll) {
 #pragma unroll
             for (int k = 0; k < LCAP; ++k)

@@ -69,16 +69,20 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
 }
 
 // lock-log parity kernel: insert entries into a register-resident (variant 0)
-// or local-memory (variant 1) sorted lock log, or their encounter-order
-// counterparts (variants 2, 3: STM-HV-Backoff / unsorted ablation), and dump it.
-template <int LCAP, bool SORTED>
+// or local-memory (variant 1) sorted lock log, their encounter-order
+// counterparts (variants 2, 3: STM-HV-Backoff / unsorted ablation), or the
+// order-preserving hashed log of P:115 (variants 4, 5: capacity 16 / 256),
+// and dump it.
+template <int LCAP, bool SORTED, bool LOCAL = false, bool HLOG = false>
 __global__ void lock_log_kernel(const uint32_t* e, int n, uint32_t* out, int* out_n)
 {
     if (threadIdx.x || blockIdx.x) return;
-    using TX = Tx<1, 1, LCAP, false, SORTED>;
+    using TX = Tx<1, 1, LCAP, LOCAL, SORTED, false, HLOG>;
     TX tx;
     tx.begin(0);
+    tx.set_id_bits(20);                   // the test's lock ids are < 2^20
     for (int k = 0; k < n; ++k) tx.insert_lock(e[k]);
+    tx.compact();
     if constexpr (TX::kUnroll) {
 #pragma unroll
         for (int k = 0; k < LCAP; ++k)
@@ -104,7 +108,10 @@ cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* 
     case 0: lock_log_kernel<16, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
     case 1: lock_log_kernel<256, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
     case 2: lock_log_kernel<16, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
-    default: lock_log_kernel<256, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    case 3: lock_log_kernel<256, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    // the order-preserving hashed log of P:115 (local memory)
+    case 4: lock_log_kernel<16, true, true, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    default: lock_log_kernel<256, true, true, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
     }
     return cudaGetLastError();
 }

@@ -51,6 +51,16 @@ struct Compact { static constexpr bool value = false; };
 template <class WL>
 struct Compact<WL, std::void_t<decltype(WL::kCompact)>> { static constexpr bool value = WL::kCompact; };
 
+// WL::kHashedLog (optional; default GSTM_HLOG): local-memory lock logs are
+// the order-preserving hash table of P:115 (Tx HLOG)
+#ifndef GSTM_HLOG
+#define GSTM_HLOG 0
+#endif
+template <class WL, class = void>
+struct HashedLog { static constexpr bool value = GSTM_HLOG; };
+template <class WL>
+struct HashedLog<WL, std::void_t<decltype(WL::kHashedLog)>> { static constexpr bool value = WL::kHashedLog; };
+
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
@@ -163,33 +173,24 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
     return __shfl_sync(FULL, late, 0);
 }
 
-// Per-phase time breakdown of the transaction loop (the Figure 5 study of
-// P:329-333): build with -DGSTM_PHASE_TIMING=1; lane 0 of every
-// warp adds the SM cycles each phase of each iteration took (after a warp
-// barrier, so the time is the warp's) to meta[M_PHASE + k].
-#ifndef GSTM_PHASE_TIMING
-#define GSTM_PHASE_TIMING 0
-#endif
-enum { PH_BEGIN = 0, PH_BODY, PH_LOCK, PH_STAMP, PH_RELEASE, PH_LOOP, PH_N };
+// Per-category time breakdown (the Figure 5 study of P:329-333):
+// the "phase" build flavour (-DGSTM_PHASE_TIMING=1) times every lane's own
+// path in the paper's categories (tx.cuh PH_*, Tx::ph); at exit the per-lane
+// totals are summed per warp and added to meta[M_PHASE + k].
+template <class TX>
+__device__ __forceinline__ void flush_phases(TX& tx, unsigned long long* dst)
+{
 #if GSTM_PHASE_TIMING
-#define PHASE_DECL() unsigned long long ph_[PH_N] = {0, 0, 0, 0, 0, 0}; long long ph_t_ = clock64()
-#define PHASE_MARK(k)                                                        \
-    do {                                                                     \
-        __syncwarp();                                                        \
-        const long long now_ = clock64();                                    \
-        ph_[k] += static_cast<unsigned long long>(now_ - ph_t_);            \
-        ph_t_ = now_;                                                        \
-    } while (0)
-#define PHASE_FLUSH(dst)                                                     \
-    do {                                                                     \
-        if (prim::lane_id() == 0)                                            \
-            for (int k_ = 0; k_ < PH_N; ++k_) atomicAdd((dst) + k_, ph_[k_]); \
-    } while (0)
-#else
-#define PHASE_DECL() do {} while (0)
-#define PHASE_MARK(k) do {} while (0)
-#define PHASE_FLUSH(dst) do {} while (0)
+    tx.ph(PH_OTHER);
+#pragma unroll 1
+    for (int k = 0; k < PH_N; ++k) {
+        unsigned long long v = tx.ph_tot[k];
+#pragma unroll
+        for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+        if (prim::lane_id() == 0) atomicAdd(dst + k, v);
+    }
 #endif
+}
 
 // ---------------------------------------------------------------------------
 // STM kernel: GPU-STM with hierarchical validation (MODE_HV, "STM-HV-Sorting")
@@ -209,8 +210,9 @@ template <class WL, int MODE, bool PAIR, int POL = POL_SORTED>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
     constexpr bool kSorted = POL == POL_SORTED;
-    using TX = std::conditional_t<PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value>,
-                                  Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value>>;
+    using TX = std::conditional_t<
+        PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value, HashedLog<WL>::value>,
+        Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value, HashedLog<WL>::value>>;
     // The grid is persistent (host sizes it to what fits on the chip, or to
     // p.max_threads): lane g runs STM threads g, g+P, ... g+(Rs-1)P of the
     // static region [0, S = Rs*P), Rs = max(1, T/P - 1) rounds, with no
@@ -232,6 +234,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     GSTM_COUNTERS(cnt);
     TX tx;
     tx.reset_stats();
+    tx.set_id_bits(static_cast<uint32_t>(__popc(m.lock_mask)));   // lock ids < 2^bits (hashed log)
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
     uint32_t seq_fails = 0;   // POL_BACKOFF: consecutive failed sequential steps of this warp
     // stage 0: start (or re-execute) transaction (t, i); stage 1: its body
@@ -240,16 +243,16 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     int stage = 0;
     bool timed_out = false, have_snap = false;
     uint32_t lock_aborts = 0;   // lock aborts of the current transaction
-    PHASE_DECL();
+    tx.ph_init();
 
     while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
         const bool act = t < p.T;
+        tx.ph(!act ? PH_OTHER : stage == 1 ? PH_LOCKS : PH_INIT);
         // TXBegin l.4-5: a fresh clock read, or the clock value right after
         // this warp's own last commit (p.snapshot_reuse)
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
         have_snap = false;
-        PHASE_MARK(PH_BEGIN);
         bool done = false, aborted = false;
         // Body rounds (p.body_rounds): a lane whose
         // transaction committed read-only (A3.l68: no locks, no stamp) starts
@@ -275,15 +278,19 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 bool next = false;
                 cnt.inc(S_ATTEMPTS);
                 result = 0;
+                tx.ph(PH_INIT);
                 const uint64_t x = gen::tx_key(p.seed, t, i);
                 tx.begin(lane_snap);                                  // TXBegin l.2-3
                 tx.sync_mask = body_mask;
                 StmCtx<TX> ctx{tx, m, MODE};
+                tx.ph(PH_NATIVE);
                 WL::body(ctx, p.w, x, t, i, result);                 // TXRead / TXWrite
                 if (!tx.opaque) {
+                    tx.ph_end(false);
                     if (tx.overflow) { cnt.inc(S_ERRORS); next = true; }  // sticky ELOGOVF, give up this tx
                     else { cnt.inc(S_AB_OPACITY); aborted = true; }  // Figure 1 / Q11
                 } else if (tx.read_only()) {                          // l.68: linearized at snapshot
+                    tx.ph_end(true);
                     if (p.tx_stamp) {
                         p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
                         p.tx_result[tx_id] = result;
@@ -294,6 +301,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     cont = true;
                     lane_snap = tx.snapshot;
                 } else {
+                    tx.ph(PH_OTHER);                                  // waits for the warp's commit round
                     stage = 1;
                     // STM-HV-Backoff: an execution that follows a lock abort goes
                     // straight to the sequential step -- its parallel attempt
@@ -307,7 +315,6 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 }
             }
         }
-        PHASE_MARK(PH_BODY);
         // No lane may take a lock while another lane of its warp can still be
         // spinning on a lock in its read phase (A3.l27-29): under independent
         // thread scheduling the locker would then wait for the spinner at the
@@ -346,18 +353,19 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     aborted = true;
                     ++lock_aborts;
                     cnt.inc(S_AB_LOCK);
+                    tx.ph_end(false);
                 }
+                if (stage == 1) tx.ph(PH_OTHER);
             } else {
                 stage = 0;
                 aborted = true;
                 cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
+                tx.ph_end(false);
             }
         }
-        PHASE_MARK(PH_LOCK);
         unsigned gm;
         const uint32_t stamp = warp_stamp(m.clock, got, gm, next_snap);   // l.83
         if (gm) have_snap = true;
-        PHASE_MARK(PH_STAMP);
         if (got) {
             tx.release_and_update(m, stamp);                          // l.84
             if (p.tx_stamp) {
@@ -369,6 +377,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             cnt.inc(S_RD_UPD, static_cast<uint32_t>(tx.nr));
             cnt.inc(S_WR_UPD, static_cast<uint32_t>(tx.nw));
             cnt.inc(S_LK_UPD, static_cast<uint32_t>(tx.nl));
+            tx.ph_end(true);
             done = true;
         }
         if constexpr (POL == POL_BACKOFF) {
@@ -412,6 +421,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                         cnt.inc(S_RD_UPD, static_cast<uint32_t>(tx.nr));
                         cnt.inc(S_WR_UPD, static_cast<uint32_t>(tx.nw));
                         cnt.inc(S_LK_UPD, static_cast<uint32_t>(tx.nl));
+                        tx.ph_end(true);
                         done = true;
                     } else if (r == C_LOCK) {
                         cnt.inc(S_LOCK_RETRIES);
@@ -421,10 +431,14 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                             aborted = true;
                             ++lock_aborts;
                             cnt.inc(S_AB_LOCK);
+                            tx.ph_end(false);
+                        } else {
+                            tx.ph(PH_OTHER);
                         }
                     } else {
                         stage = 0;
                         aborted = true;
+                        tx.ph_end(false);
                         cnt.inc(r == C_PREVBV ? S_AB_PREVBV : (r == C_TBV ? S_AB_TBV : S_AB_COMMITVBV));
                     }
                 }
@@ -434,7 +448,6 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             seq_failed = __any_sync(FULL, seq_failed);
             seq_fails = seq_failed ? seq_fails + 1u : 0u;
         }
-        PHASE_MARK(PH_RELEASE);
         if (done) {
             stage = 0;
             ++i;
@@ -466,9 +479,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 i = 0;
             }
         }
-        PHASE_MARK(PH_LOOP);
     }
-    PHASE_FLUSH(p.meta + M_PHASE);
+    flush_phases(tx, p.meta + M_PHASE);
     cnt.inc(S_POSTVAL, tx.n_postval);
     cnt.inc(S_VBV, tx.n_vbv);
     cnt.inc(S_SPINS, tx.n_spin);

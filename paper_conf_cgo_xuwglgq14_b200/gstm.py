@@ -80,17 +80,25 @@ class gstm_stats_t(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
-_lib = None
+_libs: dict = {}
 
 
-def lib():
-    """Load libgstm.so (fails loudly if it was not built)."""
-    global _lib
-    if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise GstmError(f"{LIB_PATH} missing: run `python -m paper_conf_cgo_xuwglgq14_b200.build` "
-                            "(there is no CPU fallback)")
-        L = C.CDLL(LIB_PATH)
+def lib_path(flavour: str = "") -> str:
+    """lib/libgstm.so, or lib/libgstm_<flavour>.so for a build flavour
+    (build.FLAVOURS: "strict" PTX fences, "hlog" hashed lock logs, "phase"
+    Figure-5 phase timing)."""
+    return os.path.join(_HERE, "lib", f"libgstm_{flavour}.so" if flavour else "libgstm.so")
+
+
+def lib(flavour: str = ""):
+    """Load libgstm.so or a flavour of it (fails loudly if it was not built;
+    there is no CPU fallback)."""
+    if flavour not in _libs:
+        path = lib_path(flavour)
+        if not os.path.exists(path):
+            raise GstmError(f"{path} missing: run `python -m paper_conf_cgo_xuwglgq14_b200.build"
+                            f"{' --flavour ' + flavour if flavour else ''}` (there is no CPU fallback)")
+        L = C.CDLL(path)
         P, V = C.POINTER, C.c_void_p
         u32, u64, i32 = C.c_uint32, C.c_uint64, C.c_int
         sig = {
@@ -137,17 +145,17 @@ def lib():
             f = getattr(L, name)
             f.restype = res
             f.argtypes = args
-        _lib = L
-    return _lib
+        _libs[flavour] = L
+    return _libs[flavour]
 
 
-def last_error() -> str:
-    return lib().gstm_last_error().decode()
+def last_error(L=None) -> str:
+    return (L or lib()).gstm_last_error().decode()
 
 
-def _check(rc: int, what: str) -> int:
+def _check(rc: int, what: str, L=None) -> int:
     if rc < 0:
-        raise GstmError(f"{what}: {STATUS.get(rc, rc)}: {last_error()}")
+        raise GstmError(f"{what}: {STATUS.get(rc, rc)}: {last_error(L)}")
     return rc
 
 
@@ -160,41 +168,41 @@ def _ptr(a: np.ndarray):
 CREATE_PAIRED = 1
 
 
-def gstm_create(heap_words: int, lock_table_bits: int, flags: int = 0):
-    h = lib().gstm_create_ex(heap_words, lock_table_bits, flags) if flags else lib().gstm_create(heap_words,
-                                                                                                 lock_table_bits)
+def gstm_create(heap_words: int, lock_table_bits: int, flags: int = 0, L=None):
+    L = L or lib()
+    h = L.gstm_create_ex(heap_words, lock_table_bits, flags) if flags else L.gstm_create(heap_words, lock_table_bits)
     if not h:
-        raise GstmError(f"gstm_create: {last_error()}")
+        raise GstmError(f"gstm_create: {last_error(L)}")
     return h
 
 
-def gstm_destroy(h) -> None:
-    lib().gstm_destroy(h)
+def gstm_destroy(h, L=None) -> None:
+    (L or lib()).gstm_destroy(h)
 
 
-def gstm_default_params(workload) -> gstm_params_t:
+def gstm_default_params(workload, L=None) -> gstm_params_t:
     p = gstm_params_t()
-    _check(lib().gstm_default_params(_wl(workload), C.byref(p)), "gstm_default_params")
+    _check((L or lib()).gstm_default_params(_wl(workload), C.byref(p)), "gstm_default_params", L)
     return p
 
 
-def gstm_set_params(h, p: gstm_params_t) -> None:
-    _check(lib().gstm_set_params(h, C.byref(p)), "gstm_set_params")
+def gstm_set_params(h, p: gstm_params_t, L=None) -> None:
+    _check((L or lib()).gstm_set_params(h, C.byref(p)), "gstm_set_params", L)
 
 
-def gstm_set_mode(h, mode) -> None:
-    _check(lib().gstm_set_mode(h, _mode(mode)), "gstm_set_mode")
+def gstm_set_mode(h, mode, L=None) -> None:
+    _check((L or lib()).gstm_set_mode(h, _mode(mode)), "gstm_set_mode", L)
 
 
-def gstm_launch(h, workload, n_threads: int, tx_per_thread: int, seed: int) -> None:
-    _check(lib().gstm_launch(h, _wl(workload), n_threads, tx_per_thread, seed), "gstm_launch")
+def gstm_launch(h, workload, n_threads: int, tx_per_thread: int, seed: int, L=None) -> None:
+    _check((L or lib()).gstm_launch(h, _wl(workload), n_threads, tx_per_thread, seed), "gstm_launch", L)
 
 
-def gstm_stats(h, check: bool = True) -> gstm_stats_t:
+def gstm_stats(h, check: bool = True, L=None) -> gstm_stats_t:
     s = gstm_stats_t()
-    rc = lib().gstm_stats(h, C.byref(s))
+    rc = (L or lib()).gstm_stats(h, C.byref(s))
     if check:
-        _check(rc, "gstm_stats")
+        _check(rc, "gstm_stats", L)
     return s
 
 
@@ -209,18 +217,21 @@ def _mode(m) -> int:
 class Gstm:
     """Owning wrapper of a gstm_t handle."""
 
-    def __init__(self, heap_words: int, lock_table_bits: int, paired: bool = False):
+    def __init__(self, heap_words: int, lock_table_bits: int, paired: bool = False, flavour: str = ""):
         """paired=True: GSTM_CREATE_PAIRED layout (each word next to its
-        version lock; needs heap_words <= 2^lock_table_bits)."""
+        version lock; needs heap_words <= 2^lock_table_bits).  flavour: a
+        build flavour of the library (lib_path)."""
         self.h = None
-        self.h = gstm_create(heap_words, lock_table_bits, CREATE_PAIRED if paired else 0)
+        self._L = lib(flavour)
+        self.flavour = flavour
+        self.h = gstm_create(heap_words, lock_table_bits, CREATE_PAIRED if paired else 0, L=self._L)
         self.bits = lock_table_bits
         self.paired = paired
         self._attached = None
 
     def close(self) -> None:
         if self.h:
-            gstm_destroy(self.h)
+            gstm_destroy(self.h, L=self._L)
             self.h = None
 
     def __enter__(self):
@@ -238,7 +249,7 @@ class Gstm:
     # configuration
     def params(self) -> gstm_params_t:
         p = gstm_params_t()
-        _check(lib().gstm_get_params(self.h, C.byref(p)), "gstm_get_params")
+        _check(self._L.gstm_get_params(self.h, C.byref(p)), "gstm_get_params", self._L)
         return p
 
     def set_params(self, p: gstm_params_t | None = None, **kw) -> gstm_params_t:
@@ -248,102 +259,104 @@ class Gstm:
             if not hasattr(p, k):
                 raise KeyError(k)
             setattr(p, k, int(v))
-        gstm_set_params(self.h, p)
+        gstm_set_params(self.h, p, L=self._L)
         return p
 
     def set_workload_defaults(self, workload, **kw) -> gstm_params_t:
-        p = gstm_default_params(workload)
+        p = gstm_default_params(workload, L=self._L)
         return self.set_params(p, **kw)
 
     def set_mode(self, mode) -> None:
-        gstm_set_mode(self.h, mode)
+        gstm_set_mode(self.h, mode, L=self._L)
 
     def set_stream(self, stream) -> None:
         """stream: a torch.cuda.Stream, an int handle, or None (the handle's
         private stream).  torch's legacy default stream has handle 0; it is
         passed as cudaStreamLegacy (1) so work really lands on it."""
         if stream is None:
-            _check(lib().gstm_set_stream(self.h, None), "gstm_set_stream")
+            _check(self._L.gstm_set_stream(self.h, None), "gstm_set_stream", self._L)
             return
         ptr = int(getattr(stream, "cuda_stream", stream))
-        _check(lib().gstm_set_stream(self.h, C.c_void_p(ptr if ptr else 1)), "gstm_set_stream")
+        _check(self._L.gstm_set_stream(self.h, C.c_void_p(ptr if ptr else 1)), "gstm_set_stream", self._L)
 
     def attach_heap(self, tensor) -> None:
         """Use a torch CUDA tensor (int32/uint32 storage) as the heap."""
         if tensor is None:
-            _check(lib().gstm_attach_heap(self.h, None, 0), "gstm_attach_heap")
+            _check(self._L.gstm_attach_heap(self.h, None, 0), "gstm_attach_heap", self._L)
             self._attached = None
             return
         assert tensor.is_cuda and tensor.is_contiguous() and tensor.element_size() == 4
-        _check(lib().gstm_attach_heap(self.h, C.c_void_p(tensor.data_ptr()), tensor.numel()), "gstm_attach_heap")
+        _check(self._L.gstm_attach_heap(self.h, C.c_void_p(tensor.data_ptr()), tensor.numel()), "gstm_attach_heap", self._L)
         self._attached = tensor
 
     @property
     def heap_words(self) -> int:
-        return int(lib().gstm_heap_words(self.h))
+        return int(self._L.gstm_heap_words(self.h))
 
     # data
     def init_heap(self, workload) -> None:
-        _check(lib().gstm_init_heap(self.h, _wl(workload)), "gstm_init_heap")
+        _check(self._L.gstm_init_heap(self.h, _wl(workload)), "gstm_init_heap", self._L)
 
     def km_recenter(self) -> None:
         """End of a k-means iteration (params.km_assign = 1): centroids =
         floor means of their records, records zeroed (asynchronous)."""
-        _check(lib().gstm_km_recenter(self.h), "gstm_km_recenter")
+        _check(self._L.gstm_km_recenter(self.h), "gstm_km_recenter", self._L)
 
     def write_heap(self, a: np.ndarray, offset: int = 0) -> None:
         a = np.ascontiguousarray(a, dtype=np.uint32)
-        _check(lib().gstm_write_heap(self.h, _ptr(a), offset, a.size), "gstm_write_heap")
+        _check(self._L.gstm_write_heap(self.h, _ptr(a), offset, a.size), "gstm_write_heap", self._L)
 
     def read_heap(self, words: int | None = None, offset: int = 0) -> np.ndarray:
         n = self.heap_words - offset if words is None else words
         out = np.empty(n, dtype=np.uint32)
-        _check(lib().gstm_read_heap(self.h, _ptr(out), offset, n), "gstm_read_heap")
+        _check(self._L.gstm_read_heap(self.h, _ptr(out), offset, n), "gstm_read_heap", self._L)
         return out
 
     def read_locks(self, n: int | None = None) -> np.ndarray:
         n = (1 << self.bits) if n is None else n
         out = np.empty(n, dtype=np.uint32)
-        _check(lib().gstm_read_locks(self.h, _ptr(out), n), "gstm_read_locks")
+        _check(self._L.gstm_read_locks(self.h, _ptr(out), n), "gstm_read_locks", self._L)
         return out
 
     def read_clock(self) -> int:
         c = C.c_uint64(0)
-        _check(lib().gstm_read_clock(self.h, C.byref(c)), "gstm_read_clock")
+        _check(self._L.gstm_read_clock(self.h, C.byref(c)), "gstm_read_clock", self._L)
         return c.value
 
     def reset_meta(self) -> None:
-        _check(lib().gstm_reset_meta(self.h), "gstm_reset_meta")
+        _check(self._L.gstm_reset_meta(self.h), "gstm_reset_meta", self._L)
 
     def set_clock(self, value: int) -> None:
-        _check(lib().gstm_set_clock(self.h, value), "gstm_set_clock")
+        _check(self._L.gstm_set_clock(self.h, value), "gstm_set_clock", self._L)
 
     # hot path
     def launch(self, workload, n_threads: int, tx_per_thread: int, seed: int) -> None:
-        gstm_launch(self.h, workload, n_threads, tx_per_thread, seed)
+        gstm_launch(self.h, workload, n_threads, tx_per_thread, seed, L=self._L)
 
     def stats(self, check: bool = True) -> gstm_stats_t:
-        return gstm_stats(self.h, check)
+        return gstm_stats(self.h, check, L=self._L)
 
     def stats_total(self, check: bool = True):
         """(stats summed since reset_stats_total, number of launches)"""
         s = gstm_stats_t()
         n = C.c_uint64(0)
-        rc = lib().gstm_stats_total(self.h, C.byref(s), C.byref(n))
+        rc = self._L.gstm_stats_total(self.h, C.byref(s), C.byref(n))
         if check:
-            _check(rc, "gstm_stats_total")
+            _check(rc, "gstm_stats_total", self._L)
         return s, n.value
 
-    PHASES = ["begin", "body", "lock", "stamp", "release", "loop"]
+    # Figure 5's categories (P:329), in gstm_phase_cycles order
+    PHASES = ["native", "init", "buffering", "consistency", "locks", "commit", "aborted", "other"]
 
     def phase_cycles(self) -> dict:
-        """Figure-5-style breakdown (needs a GSTM_PHASE_TIMING build)."""
+        """Figure 5 breakdown: SM cycles summed over lanes per category since
+        reset_stats_total (needs the "phase" flavour: Gstm(..., flavour="phase"))."""
         out = np.zeros(8, dtype=np.uint64)
-        _check(lib().gstm_phase_cycles(self.h, _ptr(out), 8), "gstm_phase_cycles")
+        _check(self._L.gstm_phase_cycles(self.h, _ptr(out), 8), "gstm_phase_cycles", self._L)
         return {k: int(out[i]) for i, k in enumerate(self.PHASES)}
 
     def reset_stats_total(self) -> None:
-        _check(lib().gstm_reset_stats_total(self.h), "gstm_reset_stats_total")
+        _check(self._L.gstm_reset_stats_total(self.h), "gstm_reset_stats_total", self._L)
 
     def run(self, workload, n_threads: int, tx_per_thread: int, seed: int, check: bool = True) -> gstm_stats_t:
         self.launch(workload, n_threads, tx_per_thread, seed)
@@ -352,65 +365,67 @@ class Gstm:
     def read_tx_log(self, n: int):
         st = np.empty(n, dtype=np.uint32)
         rs = np.empty(n, dtype=np.uint32)
-        _check(lib().gstm_read_tx_log(self.h, _ptr(st), _ptr(rs), n), "gstm_read_tx_log")
+        _check(self._L.gstm_read_tx_log(self.h, _ptr(st), _ptr(rs), n), "gstm_read_tx_log", self._L)
         return st, rs
 
     def run_host(self, workload, heap_in: np.ndarray, heap_out: np.ndarray, n_threads: int,
                  tx_per_thread: int, seed: int) -> gstm_stats_t:
         s = gstm_stats_t()
         assert heap_in.dtype == np.uint32 and heap_out.dtype == np.uint32 and heap_in.size == heap_out.size
-        _check(lib().gstm_run_host(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
-                                   n_threads, tx_per_thread, seed, C.byref(s)), "gstm_run_host")
+        _check(self._L.gstm_run_host(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
+                                   n_threads, tx_per_thread, seed, C.byref(s)), "gstm_run_host", self._L)
         return s
 
     def run_host_async(self, workload, heap_in: np.ndarray, heap_out: np.ndarray, n_threads: int,
                        tx_per_thread: int, seed: int) -> None:
         """Enqueue copy-in, launch and copy-out; heap_out is valid after sync()."""
         assert heap_in.dtype == np.uint32 and heap_out.dtype == np.uint32 and heap_in.size == heap_out.size
-        _check(lib().gstm_run_host_async(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
-                                         n_threads, tx_per_thread, seed), "gstm_run_host_async")
+        _check(self._L.gstm_run_host_async(self.h, _wl(workload), _ptr(heap_in), _ptr(heap_out), heap_in.size,
+                                         n_threads, tx_per_thread, seed), "gstm_run_host_async", self._L)
 
     def join(self) -> int:
         """Make the handle's stream wait (device-side) for the last run_host_async copy-out."""
-        return _check(lib().gstm_join(self.h), "gstm_join")
+        return _check(self._L.gstm_join(self.h), "gstm_join", self._L)
 
     def sync(self) -> int:
-        return _check(lib().gstm_sync(self.h), "gstm_sync")
+        return _check(self._L.gstm_sync(self.h), "gstm_sync", self._L)
 
     # tests / measurement
     def descr_words(self, workload) -> int:
-        return _check(lib().gstm_descr_words(self.h, _wl(workload)), "gstm_descr_words")
+        return _check(self._L.gstm_descr_words(self.h, _wl(workload)), "gstm_descr_words", self._L)
 
     def dump_descr(self, workload, n_threads: int, tx_per_thread: int, seed: int, wpt: int | None = None):
         wpt = self.descr_words(workload) if wpt is None else wpt
         out = np.empty(n_threads * tx_per_thread * wpt, dtype=np.uint32)
-        _check(lib().gstm_dump_descr(self.h, _wl(workload), n_threads, tx_per_thread, seed, _ptr(out), wpt),
-               "gstm_dump_descr")
+        _check(self._L.gstm_dump_descr(self.h, _wl(workload), n_threads, tx_per_thread, seed, _ptr(out), wpt),
+               "gstm_dump_descr", self._L)
         return out.reshape(n_threads * tx_per_thread, wpt)
 
     def script(self, mode, ops, n_tx: int = 4, prelock_vbv: bool = True) -> np.ndarray:
         ops = np.ascontiguousarray(np.asarray(ops, dtype=np.uint32).reshape(-1, 4))
         out = np.zeros_like(ops)
-        _check(lib().gstm_script(self.h, _mode(mode), 1 if prelock_vbv else 0, _ptr(ops), ops.shape[0],
-                                 _ptr(out), n_tx), "gstm_script")
+        _check(self._L.gstm_script(self.h, _mode(mode), 1 if prelock_vbv else 0, _ptr(ops), ops.shape[0],
+                                 _ptr(out), n_tx), "gstm_script", self._L)
         return out
 
 
-def gstm_lock_log(entries, variant: int = 0) -> np.ndarray:
+def gstm_lock_log(entries, variant: int = 0, flavour: str = "") -> np.ndarray:
     e = np.ascontiguousarray(np.asarray(entries, dtype=np.uint32))
     out = np.zeros(256, dtype=np.uint32)
-    n = _check(lib().gstm_lock_log(_ptr(e), e.size, _ptr(out), variant), "gstm_lock_log")
+    L = lib(flavour)
+    n = _check(L.gstm_lock_log(_ptr(e), e.size, _ptr(out), variant), "gstm_lock_log", L)
     return out[:n].copy()
 
 
-def gstm_ubench_mix(h, words: int, prog, n_tx: int, threads: int, block: int = 256):
+def gstm_ubench_mix(h, words: int, prog, n_tx: int, threads: int, block: int = 256, L=None):
     """Op-mix roof (include/gstm.h): returns (tx/s, ms).  Clobbers the
     handle's heap, lock table and clock."""
     pr = np.ascontiguousarray(np.asarray(prog, dtype=np.uint32))
     tps = C.c_double(0)
     ms = C.c_double(0)
-    _check(lib().gstm_ubench_mix(h, words, _ptr(pr), pr.size, n_tx, threads, block, C.byref(tps), C.byref(ms)),
-           "gstm_ubench_mix")
+    L = L or lib()
+    _check(L.gstm_ubench_mix(h, words, _ptr(pr), pr.size, n_tx, threads, block, C.byref(tps), C.byref(ms)),
+           "gstm_ubench_mix", L)
     return tps.value, ms.value
 
 

@@ -20,17 +20,20 @@ def oracle_params(wl: str, gp: G.gstm_params_t) -> O.Params:
     return O.params(wl, **{f: getattr(gp, f) for f in WL_FIELDS})
 
 
-def make(wl: str, T: int, K: int, bits: int, mode="auto", heap_words=None, paired=False, **kw):
+def make(wl: str, T: int, K: int, bits: int, mode="auto", heap_words=None, paired=False, flavour="", **kw):
     """Create a handle sized for the workload, with verify on and the
     workload's device-side initial heap; returns (g, gp, op, init).
-    paired=True uses the GSTM_CREATE_PAIRED layout."""
+    paired=True uses the GSTM_CREATE_PAIRED layout; flavour selects a build
+    flavour of the library (build.FLAVOURS)."""
     gp = G.gstm_default_params(wl)
     for k, v in kw.items():
         setattr(gp, k, int(v))
     gp.verify = 1
     op = oracle_params(wl, gp)
     words = O.footprint(op, T, K) if heap_words is None else heap_words
-    g = G.Gstm(words, bits, paired=paired)
+    if flavour:
+        B.build(flavour=flavour)
+    g = G.Gstm(words, bits, paired=paired, flavour=flavour)
     g.set_params(gp)
     g.set_mode(mode)
     g.init_heap(wl)

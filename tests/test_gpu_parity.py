@@ -75,16 +75,24 @@ def test_init_heap_parity(wl):
     assert (g.read_heap() == O.init_heap(op, 100_003)).all()
 
 
-@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256), (2, 16), (3, 256)])
+@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256), (2, 16), (3, 256), (4, 16), (5, 256)])
 def test_lock_log_parity(variant, cap):
     """Encounter-time sorted lock log (P:113-115) on the device vs the oracle;
-    variants 2/3: the encounter-order log of STM-HV-Backoff (Q32)."""
+    variants 2/3: the encounter-order log of STM-HV-Backoff (Q32); 4/5: the
+    order-preserving hashed log of P:115 (same order as sorted(set)).  Id
+    ranges from 4 (every entry a duplicate of few ids) to 2^20 (spread), plus
+    ascending and clustered arrivals (long runs in the hashed table)."""
     rng = np.random.default_rng(variant)
     for trial in range(300):
         n = int(rng.integers(0, cap + 8))
         hi = int(rng.choice([4, 50, 1 << 20]))
-        e = (rng.integers(0, hi, n).astype(np.uint32) << 2) | rng.integers(1, 4, n).astype(np.uint32)
-        want = O.lock_log(e, sorted_log=variant < 2)
+        ids = rng.integers(0, hi, n)
+        if trial % 5 == 3:
+            ids = np.sort(ids)                               # ascending arrivals
+        if trial % 5 == 4:
+            ids = (1 << 19) + rng.integers(0, 3 * n + 1, n)  # one cluster of homes
+        e = (ids.astype(np.uint32) << 2) | rng.integers(1, 4, n).astype(np.uint32)
+        want = O.lock_log(e, sorted_log=variant not in (2, 3))
         if want.size > cap:
             with pytest.raises(G.GstmError):
                 G.gstm_lock_log(e, variant)
