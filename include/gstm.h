@@ -144,6 +144,10 @@ typedef struct {
                              /*    iteration, up to this many bodies per iteration   */
                              /*    (DESIGN.md §6.11); 0 or 1 = one body per          */
                              /*    iteration.  Default 1 (HT: see DESIGN.md)         */
+    uint32_t pipeline_max_locks; /* local-memory lock logs: the pipelined first round */
+                             /*    (lock_pipeline) is used only for logs of at most  */
+                             /*    this many locks (issued 8 atom.or at a time);     */
+                             /*    0 = 8.  Default 8                                 */
 } gstm_params_t;
 
 typedef struct {

@@ -200,6 +200,7 @@ static gstm_params_t default_params(int workload)
     p.snapshot_reuse = 1;
     p.lock_pipeline = 1;
     p.body_rounds = 1;
+    p.pipeline_max_locks = 8;
     if (workload == GSTM_WL_BANK) {
         p.n_words = 1ull << 20;
         // a transaction pipelines the first lock round of its first 4
@@ -683,6 +684,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.lock_pipeline = P.lock_pipeline;
     kp.max_threads = P.max_threads;
     kp.body_rounds = P.body_rounds ? P.body_rounds : 1u;
+    kp.pipeline_max_locks = P.pipeline_max_locks ? P.pipeline_max_locks : 8u;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));

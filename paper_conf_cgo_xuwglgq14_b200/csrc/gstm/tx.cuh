@@ -786,11 +786,12 @@ struct Tx {
     // out kChunk at a time (their results land in registers, then in the
     // local log), so a transaction with n locks pays ceil(n / kChunk) memory
     // round trips instead of n.  On a conflict every lock this round set is
-    // restored, as above.  Used only when the log fits one chunk (nl <=
-    // kChunk, e.g. an HT insert): with more locks, holding all of them while
-    // failing on one makes readers spin (measured on EB A=16 and KM's 17
-    // locks: -10% and -50%), and the sequential order that stops at the
-    // first held lock is faster.
+    // restored, as above.  The kernel uses it only for logs of at most
+    // params.pipeline_max_locks entries (default kChunk, e.g. an HT insert):
+    // with more locks, holding all of them while failing on one makes readers
+    // spin (measured on EB A=16 and KM's 17 locks: -10% and -50%), and the
+    // sequential order that stops at the first held lock is faster (DESIGN.md
+    // §6.4) -- except where one round trip per lock dominates (§7.4).
     static constexpr int kChunk = 8;
     __device__ __forceinline__ bool get_locks_and_tbv_pipelined_local(const Meta& m)
     {
@@ -833,7 +834,7 @@ struct Tx {
         ph(PH_LOCKS);
         bool got;
         if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
-        else got = (pipelined && nl <= kChunk) ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
+        else got = pipelined ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18

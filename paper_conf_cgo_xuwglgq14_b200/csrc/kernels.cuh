@@ -65,6 +65,7 @@ struct KParams {
     uint64_t max_threads;          // 0: one CUDA thread per STM thread; else cap (grid-stride)
     uint32_t paired;               // paired layout (value | lock per u64, tx_pair.cuh)
     uint32_t body_rounds;          // >= 1: bodies per warp iteration for lanes that commit read-only
+    uint32_t pipeline_max_locks;   // local-memory logs: pipeline the first round only up to this many locks
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);
