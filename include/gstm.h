@@ -335,8 +335,9 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
  * both sorted by id.  Variants 2 and 3: the same capacities in
  * encounter order, the lock order of GSTM_MODE_HV_BACKOFF /
  * GSTM_MODE_HV_UNSORTED.  Variants 4 and 5: the order-preserving hashed log
- * of P:115 in local memory, capacity 16 / 256) and return the resulting log
- * in out; returns its length or a negative error. */
+ * of P:115 in local memory, capacity 16 / 256.  Variant 6: sorted, in shared
+ * memory [entry][lane], capacity 64) and return the resulting log in
+ * out; returns its length or a negative error. */
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant);
 /* Roofline microbenchmark: kind 0 random atom.or, 1
  * same-address atom.add.u64, 2 random ld.relaxed, 3 random st.relaxed, 4

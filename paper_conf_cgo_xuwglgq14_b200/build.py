@@ -40,6 +40,7 @@ FLAVOURS = {
     "strict": ["-DGSTM_STRICT_FENCES=1"],      # every fence the formal PTX model asks for
     "hlog": ["-DGSTM_HLOG=1"],                 # order-preserving hashed lock logs
     "phase": ["-DGSTM_PHASE_TIMING=1"],        # Figure 5 per-phase cycle counters
+    "smem": ["-DGSTM_SMEM_LOGS=1"],            # bank / RA / KM logs in shared memory
 }
 
 

@@ -949,7 +949,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
 
 int gstm_lock_log(const uint32_t* entries, int n, uint32_t* out, int variant)
 {
-    if (!entries || !out || n < 0 || n > 4096 || variant < 0 || variant > 5) { set_error("gstm_lock_log: bad argument"); return GSTM_EINVAL; }
+    if (!entries || !out || n < 0 || n > 4096 || variant < 0 || variant > 6) { set_error("gstm_lock_log: bad argument"); return GSTM_EINVAL; }
     uint32_t *de = nullptr, *dout = nullptr;
     int* dn = nullptr;
     CUDA_TRY(cudaMalloc(&de, (n + 1) * 4));

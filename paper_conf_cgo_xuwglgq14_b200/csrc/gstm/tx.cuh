@@ -103,13 +103,38 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
 // `#pragma unroll 1`; validation loads 4 in flight) -- for kernels whose code
 // outgrows the instruction cache (HT: DESIGN.md §6.9); else the compiler
 // unrolls them (by 4) and validation keeps 8 loads in flight.
+// A per-thread log array: registers / local memory (SMEM = false), or the
+// literal organisation of P:117 in shared memory -- entry k of the 32 lanes of
+// a warp in 32 consecutive words, [entry][lane], so the lanes' accesses to
+// their k-th entries hit 32 different banks (SMEM = true; bind() sets the
+// lane's column).
+template <int CAP, bool SMEM>
+struct LogArr {
+    uint32_t a[CAP];
+    __device__ __forceinline__ uint32_t& operator[](int k) { return a[k]; }
+    __device__ __forceinline__ const uint32_t& operator[](int k) const { return a[k]; }
+    __device__ __forceinline__ void bind(uint32_t*) {}
+};
+template <int CAP>
+struct LogArr<CAP, true> {
+    uint32_t* p;                          // shared memory: this lane's column
+    __device__ __forceinline__ uint32_t& operator[](int k) { return p[k * 32]; }
+    __device__ __forceinline__ const uint32_t& operator[](int k) const { return p[k * 32]; }
+    __device__ __forceinline__ void bind(uint32_t* col) { p = col; }
+};
+
 // HLOG = true (local-memory logs, sorted): the lock log is the order-preserving
 // hash table of P:115 instead of one sorted array.
-template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false, bool HLOG = false>
+// SMEM = true: the read-, write- and lock-logs live in shared memory, per warp
+// [entry][lane]; the kernel binds them (bind_smem).
+template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false, bool HLOG = false,
+          bool SMEM = false>
 struct Tx {
     // register-resident (unrolled) logs for small capacities unless the
-    // workload asks for local memory (LOCAL: fewer registers, more warps)
-    static constexpr bool kUnroll = !LOCAL && (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
+    // workload asks for local memory (LOCAL: fewer registers, more warps) or
+    // shared memory (SMEM)
+    static constexpr bool kUnroll = !LOCAL && !SMEM && (RCAP <= 24 && WCAP <= 24 && LCAP <= 32);
+    static constexpr bool kSmem = SMEM;
     static constexpr int kRcap = RCAP, kWcap = WCAP, kLcap = LCAP;
     static constexpr bool kCompact = COMPACT;
     // value / lock-word loads validation keeps in flight with local-memory logs
@@ -117,14 +142,28 @@ struct Tx {
     // order-preserving hashed lock log: kHs home slots (load factor
     // <= 1/2), then LCAP overflow slots (an entry never sits more than
     // LCAP - 1 slots past its home); occupancy bitmap in registers
-    static constexpr bool kHlog = HLOG && SORTED && !kUnroll;
+    static constexpr bool kHlog = HLOG && SORTED && !kUnroll && !SMEM;
     static constexpr int kHs = 2 * LCAP;
     static constexpr int kTs = kHlog ? kHs + LCAP : LCAP;
     static constexpr int kBw = kHlog ? (kTs + 31) / 32 : 1;
 
-    uint32_t r_addr[RCAP], r_val[RCAP];   // read-set  <addr,val>
-    uint32_t w_addr[WCAP], w_val[WCAP];   // write-set <addr,val> (redo log)
-    uint32_t l_ent[kTs], l_old[LCAP];     // sorted lock log (hashed: the table); old lock words
+    LogArr<RCAP, SMEM> r_addr, r_val;     // read-set  <addr,val>
+    LogArr<WCAP, SMEM> w_addr, w_val;     // write-set <addr,val> (redo log)
+    LogArr<kTs, SMEM> l_ent;              // sorted lock log (hashed: the table)
+    LogArr<LCAP, SMEM> l_old;             // old lock words
+    // shared-memory logs: words per thread, and the binding of every log to
+    // this lane's column of its warp's [word][lane] region
+    static constexpr int kSmemWords = 2 * RCAP + 2 * WCAP + kTs + LCAP;
+    __device__ __forceinline__ void bind_smem(uint32_t* warp_region, int lane)
+    {
+        uint32_t* c = warp_region + lane;
+        r_addr.bind(c);
+        r_val.bind(c + 32 * RCAP);
+        w_addr.bind(c + 32 * (2 * RCAP));
+        w_val.bind(c + 32 * (2 * RCAP + WCAP));
+        l_ent.bind(c + 32 * (2 * RCAP + 2 * WCAP));
+        l_old.bind(c + 32 * (2 * RCAP + 2 * WCAP + kTs));
+    }
     uint32_t occ[kBw];                    // hashed log: occupied slots
     uint32_t id_shift = 12;               // hashed log: 32 - lock-table bits (home = id's top bits)
     bool compacted;                       // hashed log: l_ent[0, nl) is the dense sorted log

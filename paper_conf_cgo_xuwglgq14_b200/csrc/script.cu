@@ -72,13 +72,15 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
 // or local-memory (variant 1) sorted lock log, their encounter-order
 // counterparts (variants 2, 3: STM-HV-Backoff / unsorted ablation), or the
 // order-preserving hashed log of P:115 (variants 4, 5: capacity 16 / 256),
-// and dump it.
-template <int LCAP, bool SORTED, bool LOCAL = false, bool HLOG = false>
+// or the shared-memory log of P:117 (variant 6: capacity 64), and dump it.
+template <int LCAP, bool SORTED, bool LOCAL = false, bool HLOG = false, bool SMEM = false>
 __global__ void lock_log_kernel(const uint32_t* e, int n, uint32_t* out, int* out_n)
 {
+    using TX = Tx<1, 1, LCAP, LOCAL, SORTED, false, HLOG, SMEM>;
+    __shared__ uint32_t region[SMEM ? 32 * TX::kSmemWords : 1];
     if (threadIdx.x || blockIdx.x) return;
-    using TX = Tx<1, 1, LCAP, LOCAL, SORTED, false, HLOG>;
     TX tx;
+    if constexpr (SMEM) tx.bind_smem(region, 0);
     tx.begin(0);
     tx.set_id_bits(20);                   // the test's lock ids are < 2^20
     for (int k = 0; k < n; ++k) tx.insert_lock(e[k]);
@@ -111,7 +113,9 @@ cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* 
     case 3: lock_log_kernel<256, false><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
     // the order-preserving hashed log of P:115 (local memory)
     case 4: lock_log_kernel<16, true, true, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
-    default: lock_log_kernel<256, true, true, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    case 5: lock_log_kernel<256, true, true, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
+    // shared-memory logs, [entry][lane]
+    default: lock_log_kernel<64, true, false, false, true><<<1, 32, 0, s>>>(entries, n, out, out_n); break;
     }
     return cudaGetLastError();
 }

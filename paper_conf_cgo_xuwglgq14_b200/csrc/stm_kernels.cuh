@@ -61,6 +61,17 @@ struct HashedLog { static constexpr bool value = GSTM_HLOG; };
 template <class WL>
 struct HashedLog<WL, std::void_t<decltype(WL::kHashedLog)>> { static constexpr bool value = WL::kHashedLog; };
 
+// WL::kSmemLogs (optional; default GSTM_SMEM_LOGS for the workloads whose
+// logs fit: bank, RA, KM): logs in shared memory, [entry][lane] per warp
+// (Tx SMEM)
+#ifndef GSTM_SMEM_LOGS
+#define GSTM_SMEM_LOGS 0
+#endif
+template <class WL, class = void>
+struct SmemLogs { static constexpr bool value = false; };
+template <class WL>
+struct SmemLogs<WL, std::void_t<decltype(WL::kSmemLogs)>> { static constexpr bool value = WL::kSmemLogs; };
+
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
@@ -206,13 +217,27 @@ __device__ __forceinline__ void flush_phases(TX& tx, unsigned long long* dst)
 //                 committed
 //   POL_UNSORTED  ablation: encounter-order lock log with the parallel retry
 //                 of POL_SORTED -- exposed to the intra-warp livelock of P:63
+// the transaction type of a workload's STM kernel
+template <class WL, bool PAIR, int POL>
+using StmTx = std::conditional_t<
+    PAIR,
+    TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value,
+           HashedLog<WL>::value, SmemLogs<WL>::value>,
+    Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value, HashedLog<WL>::value,
+       SmemLogs<WL>::value>>;
+
+// dynamic shared memory of the STM kernel: the shared-memory logs, if any
+template <class WL, bool PAIR, int POL>
+constexpr size_t stm_smem_bytes(int block)
+{
+    using TX = StmTx<WL, PAIR, POL>;
+    return TX::kSmem ? static_cast<size_t>(block) * TX::kSmemWords * sizeof(uint32_t) : 0;
+}
+
 template <class WL, int MODE, bool PAIR, int POL = POL_SORTED>
 __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams p)
 {
-    constexpr bool kSorted = POL == POL_SORTED;
-    using TX = std::conditional_t<
-        PAIR, TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value, HashedLog<WL>::value>,
-        Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, kSorted, Compact<WL>::value, HashedLog<WL>::value>>;
+    using TX = StmTx<WL, PAIR, POL>;
     // The grid is persistent (host sizes it to what fits on the chip, or to
     // p.max_threads): lane g runs STM threads g, g+P, ... g+(Rs-1)P of the
     // static region [0, S = Rs*P), Rs = max(1, T/P - 1) rounds, with no
@@ -233,6 +258,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     unsigned long long* work = p.meta + M_WORK;
     GSTM_COUNTERS(cnt);
     TX tx;
+    if constexpr (TX::kSmem) {
+        // this warp's [word][lane] region of the block's shared-memory logs
+        extern __shared__ uint32_t gstm_smem_logs[];
+        tx.bind_smem(gstm_smem_logs + (threadIdx.x >> 5) * 32 * TX::kSmemWords, static_cast<int>(prim::lane_id()));
+    }
     tx.reset_stats();
     tx.set_id_bits(static_cast<uint32_t>(__popc(m.lock_mask)));   // lock ids < 2^bits (hashed log)
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
@@ -723,7 +753,7 @@ __global__ void descr_kernel(const KParams p, uint32_t* out, int wpt)
 // host launch templates (instantiated per workload in wl_*.cu)
 // ---------------------------------------------------------------------------
 template <class K>
-inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0)
+inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0, size_t smem = 0)
 {
     // SM count of the CURRENT device (cached per device: one process may
     // drive handles on several GPUs)
@@ -737,19 +767,25 @@ inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0)
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     }
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, 0) != cudaSuccess || per_sm < 1) per_sm = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, smem) != cudaSuccess || per_sm < 1) per_sm = 1;
     if (warps_per_sm > 0) per_sm = std::max(1, std::min(per_sm, warps_per_sm * 32 / block));
     return static_cast<uint64_t>(per_sm) * (sms > 0 ? sms : 148);
 }
 
 template <class K>
-inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s, int warps_per_sm = 0)
+inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s, int warps_per_sm = 0,
+                              size_t smem = 0)
 {
+    if (smem > 48 * 1024) {
+        const cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                   static_cast<int>(smem));
+        if (e != cudaSuccess) return e;
+    }
     uint64_t grid = (kp.T + block - 1) / block;
-    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block, kp.max_threads ? 0 : warps_per_sm));
+    grid = std::min<uint64_t>(grid, resident_blocks(kernel, block, kp.max_threads ? 0 : warps_per_sm, smem));
     if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
     if (grid == 0) return cudaSuccess;
-    kernel<<<static_cast<unsigned>(grid), block, 0, s>>>(kp);
+    kernel<<<static_cast<unsigned>(grid), block, smem, s>>>(kp);
     return cudaGetLastError();
 }
 
@@ -760,19 +796,24 @@ cudaError_t launch_wl(int kmode, const KParams& kp, int block, cudaStream_t s)
     if (kp.max_threads) grid = std::min<uint64_t>(grid, (kp.max_threads + block - 1) / block);   // concurrency cap
     if (grid == 0) return cudaSuccess;
     const dim3 g(static_cast<unsigned>(grid)), b(block);
+    constexpr int W = WarpsPerSM<WL>::value;
     switch (kmode) {
     case KMODE_HV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s, WarpsPerSM<WL>::value)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s, WarpsPerSM<WL>::value);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true>, kp, block, s, W, stm_smem_bytes<WL, true, POL_SORTED>(block))
+                         : launch_stm(stm_kernel<WL, MODE_HV, false>, kp, block, s, W, stm_smem_bytes<WL, false, POL_SORTED>(block));
     case KMODE_TBV:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s, WarpsPerSM<WL>::value)
-                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s, WarpsPerSM<WL>::value);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_TBV, true>, kp, block, s, W, stm_smem_bytes<WL, true, POL_SORTED>(block))
+                         : launch_stm(stm_kernel<WL, MODE_TBV, false>, kp, block, s, W, stm_smem_bytes<WL, false, POL_SORTED>(block));
     case KMODE_HV_BACKOFF:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_BACKOFF>, kp, block, s, WarpsPerSM<WL>::value)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_BACKOFF>, kp, block, s, WarpsPerSM<WL>::value);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_BACKOFF>, kp, block, s, W,
+                                      stm_smem_bytes<WL, true, POL_BACKOFF>(block))
+                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_BACKOFF>, kp, block, s, W,
+                                      stm_smem_bytes<WL, false, POL_BACKOFF>(block));
     case KMODE_HV_UNSORTED:
-        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_UNSORTED>, kp, block, s, WarpsPerSM<WL>::value)
-                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_UNSORTED>, kp, block, s, WarpsPerSM<WL>::value);
+        return kp.paired ? launch_stm(stm_kernel<WL, MODE_HV, true, POL_UNSORTED>, kp, block, s, W,
+                                      stm_smem_bytes<WL, true, POL_UNSORTED>(block))
+                         : launch_stm(stm_kernel<WL, MODE_HV, false, POL_UNSORTED>, kp, block, s, W,
+                                      stm_smem_bytes<WL, false, POL_UNSORTED>(block));
     case KMODE_VBV: vbv_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_CGL: cgl_kernel<WL><<<g, b, 0, s>>>(kp); break;
     case KMODE_FGL: fgl_kernel<WL><<<g, b, 0, s>>>(kp); break;

@@ -9,6 +9,8 @@
   every local-memory-log kernel (RA, HT, EB, KM).
 * "phase": the Figure 5 per-phase cycle counters:
   the instrumented kernel must stay serializable and account for its time.
+* "smem": the bank, RA and KM logs in shared memory, [entry][lane] per warp
+  (DESIGN.md §6.13).
 
 Same checks as test_gpu_parity.py: stamp-order replay bit-exact, brute force
 on tiny inputs, closed forms, livelock freedom on two words.
@@ -22,7 +24,7 @@ from paper_conf_cgo_xuwglgq14_b200 import gstm as G
 import gpu_util as U
 
 pytestmark = pytest.mark.gpu
-FLAVOURS = ["strict", "hlog", "phase"]
+FLAVOURS = ["strict", "hlog", "phase", "smem"]
 
 
 @pytest.fixture(scope="module", autouse=True)

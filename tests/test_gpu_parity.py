@@ -75,11 +75,12 @@ def test_init_heap_parity(wl):
     assert (g.read_heap() == O.init_heap(op, 100_003)).all()
 
 
-@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256), (2, 16), (3, 256), (4, 16), (5, 256)])
+@pytest.mark.parametrize("variant,cap", [(0, 16), (1, 256), (2, 16), (3, 256), (4, 16), (5, 256), (6, 64)])
 def test_lock_log_parity(variant, cap):
     """Encounter-time sorted lock log (P:113-115) on the device vs the oracle;
     variants 2/3: the encounter-order log of STM-HV-Backoff (Q32); 4/5: the
-    order-preserving hashed log of P:115 (same order as sorted(set)).  Id
+    order-preserving hashed log of P:115 (same order as sorted(set)); 6: the
+    shared-memory log of P:117.  Id
     ranges from 4 (every entry a duplicate of few ids) to 2^20 (spread), plus
     ascending and clustered arrivals (long runs in the hashed table)."""
     rng = np.random.default_rng(variant)

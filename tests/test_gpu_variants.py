@@ -185,3 +185,29 @@ def test_unsorted_without_crossing_orders_is_fine():
     g, gp, op, init = U.make("ra", T, K, 10, mode="hv_unsorted", n_reads=1, n_words=64, ra_kind=1)
     st, *_ = U.run_verified(g, "ra", op, init, T, K, 6)
     assert st.commits == T * K
+
+
+# ---------------------------------------------------------------------------
+# compute-sanitizer on tiny configurations of every kernel
+# ---------------------------------------------------------------------------
+@pytest.mark.slow
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer_clean(tool):
+    """memcheck (out-of-bounds / misaligned global, local and shared
+    accesses), racecheck (shared-memory hazards: the per-thread counter slots)
+    and synccheck (illegal __syncwarp / ballot masks: the lockstep and
+    reconverge masks) report nothing on tiny runs of every workload, mode and
+    layout, which also replay bit-exactly."""
+    import os
+    import shutil
+    import subprocess
+    import sys
+    exe = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "9", "--print-limit", "20",
+                        sys.executable, os.path.join(root, "tools", "sanitize_tiny.py")],
+                       capture_output=True, text=True, timeout=1500)
+    assert r.returncode == 0, (r.stdout[-3000:], r.stderr[-3000:])
+    assert "launches replayed" in r.stdout
+    out = r.stdout + r.stderr
+    assert "ERROR SUMMARY: 0 errors" in out or "(0 errors, 0 warnings)" in out, out[-2000:]

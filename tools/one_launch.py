@@ -34,7 +34,7 @@ def main():
     else:
         wl, words, bits, p, T, K, _, _ = bench.CONFIGS[a.config]
         g = G.Gstm(words, bits)
-        g.set_workload_defaults(wl, **p, **kv)
+        g.set_workload_defaults(wl, **dict(p, **kv))
     g.set_mode(a.mode)
     for k in range(a.launches):
         g.init_heap(wl)
