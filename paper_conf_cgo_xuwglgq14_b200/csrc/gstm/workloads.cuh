@@ -383,9 +383,21 @@ struct HtWL {
 };
 
 // ---- EigenBench-style: A accesses alternating read / write over H words ----
-struct EbWL {
-    static constexpr int MAXA = 64;
+// Compiled for A <= 16, <= 32 and <= 64 (the launch picks the smallest that
+// fits): the logs and the body's address arrays are sized by MAXA, so an A=16
+// transaction does not carry (and spill through L2) the frame of an A=64 one;
+// A <= 16 keeps its logs in shared memory (256 B per thread, DESIGN.md
+// §6.13) -- local-memory log traffic written through to L2 and evicted to HBM
+// by the streaming heap was most of EB's excess DRAM traffic (§7.4).
+#ifndef GSTM_EB16_SMEM
+#define GSTM_EB16_SMEM 1
+#endif
+template <int MAXA_, bool SMEM_>
+struct EbWLT {
+    static constexpr int MAXA = MAXA_;
     static constexpr int RCAP = MAXA / 2, WCAP = MAXA / 2, LCAP = MAXA, FGL_LCAP = MAXA;
+    static constexpr bool kSmemLogs = SMEM_ || (GSTM_SMEM_LOGS && MAXA <= 32);   // A=64: 256 KB per block
+    static constexpr bool kLocalLogs = true;   // never register-resident (A=32 unrolled: 2.4x slower)
     static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = 2 * MAXA;
     __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
@@ -434,6 +446,9 @@ struct EbWL {
         return static_cast<int>(2 * A);
     }
 };
+using EbWL = EbWLT<64, false>;            // descriptors, checks; A in (32, 64]
+using EbWL32 = EbWLT<32, false>;
+using EbWL16 = EbWLT<16, GSTM_EB16_SMEM>;
 
 // ---- k-means cluster update (STAMP kmeans' transactional step) -------------
 // record of cluster c = [count, sum_0 .. sum_{D-1}] at word c*stride (stride >= D+1;

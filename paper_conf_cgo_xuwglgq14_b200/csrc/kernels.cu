@@ -124,7 +124,10 @@ cudaError_t launch_tx(int workload, int kmode, const KParams& kp, int block, cud
     case WL_RA: return kp.w.ra_kind == 1 ? launch_wl<RaIncWL>(kmode, kp, block, s) : launch_wl<RaWL>(kmode, kp, block, s);
     case WL_BANK: return launch_wl<BankWL>(kmode, kp, block, s);
     case WL_HT: return launch_wl<HtWL>(kmode, kp, block, s);
-    case WL_EB: return launch_wl<EbWL>(kmode, kp, block, s);
+    case WL_EB:   // the smallest compiled access count that fits (workloads.cuh EbWLT)
+        return kp.w.n_accesses <= 16 ? launch_wl<EbWL16>(kmode, kp, block, s)
+             : kp.w.n_accesses <= 32 ? launch_wl<EbWL32>(kmode, kp, block, s)
+                                     : launch_wl<EbWL>(kmode, kp, block, s);
     case WL_KM: return launch_wl<KmWL>(kmode, kp, block, s);
     }
     return cudaErrorInvalidValue;

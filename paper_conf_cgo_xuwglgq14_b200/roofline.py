@@ -129,8 +129,16 @@ def programs_from_stats(wl: str, st, paired: bool, mode: str, prelock: bool, pip
     progs = []
     if cu:
         for w, s in _shape(wl, g("reads_update") / cu, g("writes_update") / cu, g("locks_update") / cu):
-            progs.append((cu * w, stm_program(s, paired, hv and prelock, pipelined)))
-    if cr:
+            q = stm_program(s, paired, hv and prelock, pipelined)
+            if records:
+                # contention roof: what a record's commits cannot overlap is the
+                # time its locks are held -- from the first lock atomic (A3.l45)
+                # to the release (l.84); the next transaction's reads and
+                # validation can run while the record is locked
+                first = next(k for k, c in enumerate(q) if c & 0xff == ATOM_L)
+                q = q[first:]
+            progs.append((cu * w, q))
+    if cr and not records:
         for w, s in _shape(wl, g("reads_ro") / cr, 0, 0):
             s.write_slots, s.locks = [], 0
             progs.append((cr * w, stm_program(s, paired, False, False)))

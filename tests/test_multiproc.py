@@ -187,6 +187,8 @@ def test_op_mix_programs_follow_algorithm_3():
     p = R.programs_from_stats("km", st, paired=False, mode="hv", prelock=True, pipelined=False, records=(1024, 17))
     assert p[0] == 1 | R.RECORDS and p[1:3] == [1024, 17]
     assert R.op_counts(p)["atom"] == 17.0
+    assert R.op_counts(p)["ld"] == 0.0                        # the lock-holding critical section only
+    assert p[3 + 2] & 0xff == R.ATOM_L
 
 
 def test_bench_self_launches_n_ranks_with_gloo():
