@@ -198,12 +198,13 @@ def op_counts(prog: list) -> dict:
 
 
 def round_trips(prog: list) -> float:
-    """Mean dependent memory phases per transaction (fences excluded)."""
+    """Mean dependent memory round trips per transaction: load, atomic and
+    clock phases (stores are fire-and-forget; fences are not accesses)."""
     n = prog[0] & 0xff
     pos = 3 if prog[0] & RECORDS else 1
     rt = 0.0
     for _ in range(n):
         w, k = prog[pos] / 65536.0, prog[pos + 1]
-        rt += w * sum(1 for c in prog[pos + 2:pos + 2 + k] if (c & 0xff) not in (FENCE_REL, FENCE_ACQ))
+        rt += w * sum(1 for c in prog[pos + 2:pos + 2 + k] if (c & 0xff) in (LD_V, LD_L, ATOM_L, CLOCK))
         pos += 2 + k
     return rt
