@@ -148,6 +148,12 @@ typedef struct {
                              /*    (lock_pipeline) is used only for logs of at most  */
                              /*    this many locks (issued 8 atom.or at a time);     */
                              /*    0 = 8.  Default 8                                 */
+    uint32_t lock_log_at_commit; /* 1: a read's lock enters the sorted lock log when   */
+                             /*    the transaction reaches TXCommit with a write-set */
+                             /*    instead of at the read (P:113's encounter time):  */
+                             /*    the same sorted log and acquisition order, no     */
+                             /*    sorting work for read-only transactions           */
+                             /*    (DESIGN.md §6.15).  Default 0                     */
 } gstm_params_t;
 
 typedef struct {

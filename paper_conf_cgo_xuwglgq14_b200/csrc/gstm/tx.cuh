@@ -206,6 +206,8 @@ struct Tx {
     __device__ __forceinline__ void ph_end(bool) {}
 #endif
     int nr, nw, nl, n_acq;
+    bool defer_rd = false;                // lock_log_at_commit: read locks inserted at TXCommit
+    bool deferred_done;
     uint32_t snapshot;
     bool opaque, passTBV, overflow;
     uint32_t n_postval, n_vbv, n_spin;    // per-thread statistics
@@ -220,6 +222,7 @@ struct Tx {
     __device__ __forceinline__ void begin(uint32_t snap)
     {
         nr = nw = nl = n_acq = 0;                 // l.2
+        deferred_done = false;
         bloom = 0ull;
         opaque = passTBV = true;                  // l.3
         overflow = false;
@@ -339,6 +342,24 @@ struct Tx {
             }
             compacted = true;
         }
+    }
+
+    // A3.l34 for a read: insert its lock now (encounter time), or --
+    // lock_log_at_commit (defer_rd) -- when the transaction reaches TXCommit
+    // with a write-set (insert_deferred_reads).  The sorted log is a function
+    // of the set of entries (insert order does not matter, Q4), so the
+    // acquisition order and the livelock-freedom argument are the same; a
+    // read-only transaction (HT lookups: 90%) skips the sorting it never uses.
+    __device__ __forceinline__ void insert_read_lock(uint32_t id)
+    {
+        if (!defer_rd) insert_lock((id << 2) | 1u);
+    }
+    __device__ __forceinline__ void insert_deferred_reads(const Meta& m)
+    {
+        if (!defer_rd || deferred_done) return;
+        deferred_done = true;
+#pragma unroll 1
+        for (int k = 0; k < nr; ++k) insert_lock((m.lock_of(r_addr[k]) << 2) | 1u);
     }
 
     // ---- P:113-115, A3.l34/l38: sorted insert into the local lock log ----
@@ -513,7 +534,7 @@ struct Tx {
         const uint32_t vl = prim::ld_relaxed(m.lock_ptr(m.lock_of(a)));
         check_lock(m, a, vl, mode);                                  // l.27-33
         ph(PH_BUFFER);
-        insert_lock((m.lock_of(a) << 2) | 1u);                  // l.34
+        insert_read_lock(m.lock_of(a));                               // l.34
         ph(PH_NATIVE);
         return v;                                                    // l.35
     }
@@ -589,7 +610,7 @@ struct Tx {
             if constexpr (kUnroll) {
 #pragma unroll
                 for (int k = 0; k < N; ++k)
-                    if (need[k]) insert_lock((m.lock_of(a[k]) << 2) | 1u);   // l.34
+                    if (need[k]) insert_read_lock(m.lock_of(a[k]));       // l.34
             } else {
                 // local-memory logs: one inlined copy of the (looping) insert
 #pragma unroll 1
@@ -599,7 +620,7 @@ struct Tx {
 #pragma unroll
                     for (int j = 0; j < N; ++j)
                         if (j == k) { ak = a[j]; nk = need[j]; }
-                    if (nk) insert_lock((m.lock_of(ak) << 2) | 1u);  // l.34
+                    if (nk) insert_read_lock(m.lock_of(ak));         // l.34
                 }
             }
         } else {
@@ -618,7 +639,7 @@ struct Tx {
 #pragma unroll
                 for (int j = 0; j < N; ++j)
                     if (j == k) { ak = a[j]; nk = need[j]; }
-                if (nk) insert_lock((m.lock_of(ak) << 2) | 1u);
+                if (nk) insert_read_lock(m.lock_of(ak));
             }
         }
         ph(PH_NATIVE);
@@ -648,7 +669,7 @@ struct Tx {
                 ph(PH_CONSIST);
                 check_lock(m, a[k], vl[k], mode);                     // l.27-33
                 ph(PH_BUFFER);
-                insert_lock((m.lock_of(a[k]) << 2) | 1u);             // l.34
+                insert_read_lock(m.lock_of(a[k]));                    // l.34
             }
         ph(PH_NATIVE);
     }
@@ -866,6 +887,7 @@ struct Tx {
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
         ph(PH_BUFFER);
+        insert_deferred_reads(m);
         compact();
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)

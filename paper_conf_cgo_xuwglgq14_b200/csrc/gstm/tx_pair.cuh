@@ -46,6 +46,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
     using B::append_read;
     using B::reconverge;
     using B::insert_lock;
+    using B::insert_read_lock;
     using B::kCompact;
     using B::ph;
 
@@ -144,7 +145,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
         ph(PH_CONSIST);
         check_version(m, hi(pv), mode);                              // l.30-33
         ph(PH_BUFFER);
-        insert_lock((a << 2) | 1u);                                  // l.34 (lock id = word)
+        insert_read_lock(a);                                         // l.34 (lock id = word)
         ph(PH_NATIVE);
         return v;
     }
@@ -196,7 +197,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
             ph(PH_BUFFER);
 #pragma unroll
             for (int k = 0; k < N; ++k)
-                if (need[k]) insert_lock((a[k] << 2) | 1u);          // l.34
+                if (need[k]) insert_read_lock(a[k]);                 // l.34
         } else {
             uint32_t newest = 0;
 #pragma unroll
@@ -219,7 +220,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
 #pragma unroll
                 for (int j = 0; j < N; ++j)
                     if (j == k) { ak = a[j]; nk = need[j]; }
-                if (nk) insert_lock((ak << 2) | 1u);
+                if (nk) insert_read_lock(ak);
             }
         }
         ph(PH_NATIVE);
@@ -253,7 +254,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
                 ph(PH_CONSIST);
                 check_version(m, vl[k], mode);
                 ph(PH_BUFFER);
-                insert_lock((a[k] << 2) | 1u);
+                insert_read_lock(a[k]);
             }
         ph(PH_NATIVE);
     }
@@ -464,6 +465,7 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
     {
         ph(PH_BUFFER);
+        B::insert_deferred_reads(m);
         B::compact();
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)

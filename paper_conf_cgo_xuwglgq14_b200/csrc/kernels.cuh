@@ -66,6 +66,7 @@ struct KParams {
     uint32_t paired;               // paired layout (value | lock per u64, tx_pair.cuh)
     uint32_t body_rounds;          // >= 1: bodies per warp iteration for lanes that commit read-only
     uint32_t pipeline_max_locks;   // local-memory logs: pipeline the first round only up to this many locks
+    uint32_t lock_log_at_commit;   // read locks enter the sorted lock log at TXCommit (Tx::insert_read_lock)
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);

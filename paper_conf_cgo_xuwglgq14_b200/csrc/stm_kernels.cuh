@@ -265,6 +265,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     }
     tx.reset_stats();
     tx.set_id_bits(static_cast<uint32_t>(__popc(m.lock_mask)));   // lock ids < 2^bits (hashed log)
+    tx.defer_rd = p.lock_log_at_commit != 0;
     uint32_t i = 0, iter = 0, backoff = 0, next_snap = 0, tries = 0, result = 0;
     uint32_t seq_fails = 0;   // POL_BACKOFF: consecutive failed sequential steps of this warp
     // stage 0: start (or re-execute) transaction (t, i); stage 1: its body

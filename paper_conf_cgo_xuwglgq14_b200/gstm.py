@@ -58,7 +58,7 @@ class gstm_params_t(C.Structure):
         ("lock_pipeline", C.c_uint32), ("max_threads", C.c_uint32), ("lock_shift", C.c_uint32),
         ("shard_bits", C.c_uint32), ("shard", C.c_uint32), ("km_stride", C.c_uint32),
         ("km_assign", C.c_uint32), ("l2_persist_locks", C.c_uint32), ("ra_partition", C.c_uint32),
-        ("body_rounds", C.c_uint32), ("pipeline_max_locks", C.c_uint32),
+        ("body_rounds", C.c_uint32), ("pipeline_max_locks", C.c_uint32), ("lock_log_at_commit", C.c_uint32),
     ]
 
 

@@ -345,6 +345,27 @@ def test_body_rounds_replay(mode, wl, kw, T, K, bits, rounds):
     g.close()
 
 
+@pytest.mark.parametrize("mode", ["hv", "tbv", "hv_backoff"])
+@pytest.mark.parametrize("wl,kw,T,K,bits,paired", [
+    ("ht", dict(ht_buckets=1 << 12, ht_key_range=1 << 14, ht_lookup_pct=90), 1 << 14, 4, 14, False),
+    ("ht", dict(ht_buckets=64, ht_key_range=256, ht_lookup_pct=30), 2048, 4, 8, False),
+    ("bank", dict(n_words=1 << 10), 1 << 14, 4, 10, False),
+    ("bank", dict(n_words=1 << 10), 1 << 14, 4, 10, True),
+    ("ra", dict(n_reads=4, n_writes=4, n_words=1024), 256, 64, 10, False),
+    ("ra", dict(n_reads=5, n_words=64, ra_kind=1), 512, 8, 6, True),
+    ("eb", dict(n_words=1 << 12, n_accesses=32), 4096, 2, 12, False),
+    ("km", dict(km_clusters=64, km_dims=16), 1 << 14, 2, 12, False),
+])
+def test_lock_log_at_commit_replay(mode, wl, kw, T, K, bits, paired):
+    """lock_log_at_commit: read locks enter the sorted log at
+    TXCommit instead of at the read -- the same log, so the same acquisition
+    order: serializable, livelock-free, every transaction commits."""
+    g, gp, op, init = U.make(wl, T, K, bits, mode=mode, paired=paired, lock_log_at_commit=1, **kw)
+    st, *_ = U.run_verified(g, wl, op, init, T, K, 13)
+    assert st.commits + st.commits_ro == T * K
+    g.close()
+
+
 @pytest.mark.parametrize("paired", [False, True])
 @pytest.mark.parametrize("mode", ["hv", "tbv"])
 @pytest.mark.parametrize("pipeline", [1, 1000])
