@@ -539,6 +539,56 @@ struct Tx {
         return v;                                                    // l.35
     }
 
+    // l.27-34 of a small batch (bank: 2; an HT chain step), fully unrolled:
+    // ONE spin loop re-reads every still-locked lock word of the batch together
+    // (l.27-29) and ONE timestamp check with the newest version (Q35): one copy
+    // of each rare path, so the lanes of a warp that take it take it together
+    // instead of one after the other
+    template <int N>
+    __device__ __forceinline__ void check_small(const Meta& m, const uint32_t (&a)[N], const bool (&need)[N],
+                                                uint32_t (&vl)[N], int mode)
+    {
+        uint32_t spins = 0;
+        bool locked = false;
+#pragma unroll
+        for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
+        while (locked) {
+            if (++spins > m.spin_cap) { opaque = false; break; }
+            if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
+#pragma unroll
+            for (int k = 0; k < N; ++k)
+                if (need[k] && (vl[k] & 1u)) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));   // l.28
+            locked = false;
+#pragma unroll
+            for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
+        }
+        n_spin += spins;
+        reconverge();
+        uint32_t newest = 0;
+#pragma unroll
+        for (int k = 0; k < N; ++k)
+            if (need[k]) newest = max(newest, vl[k] >> 1);
+        check_version(m, newest, mode);                          // l.30-33 (Q35)
+        reconverge();
+        ph(PH_BUFFER);
+        if constexpr (kUnroll) {
+#pragma unroll
+            for (int k = 0; k < N; ++k)
+                if (need[k]) insert_read_lock(m.lock_of(a[k]));       // l.34
+        } else {
+            // local-memory logs: one inlined copy of the (looping) insert
+#pragma unroll 1
+            for (int k = 0; k < N; ++k) {
+                uint32_t ak = 0;
+                bool nk = false;
+#pragma unroll
+                for (int j = 0; j < N; ++j)
+                    if (j == k) { ak = a[j]; nk = need[j]; }
+                if (nk) insert_read_lock(m.lock_of(ak));         // l.34
+            }
+        }
+    }
+
     // Batched TXRead of N words whose addresses are known together: the N
     // value loads (l.24) are issued back to back, one fence (l.26) orders all
     // of them before the N lock loads, then each read runs l.27-34 in order.
@@ -579,50 +629,7 @@ struct Tx {
                 else vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));
             }
         if constexpr (N <= 4) {
-            // small batches (bank: 2), fully unrolled: ONE spin loop re-reads
-            // every still-locked lock word of the batch together (l.27-29)
-            // and ONE timestamp check with the newest version (Q35): one copy
-            // of each rare path, so the lanes of a warp that take it take it
-            // together instead of one after the other
-            uint32_t spins = 0;
-            bool locked = false;
-#pragma unroll
-            for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
-            while (locked) {
-                if (++spins > m.spin_cap) { opaque = false; break; }
-                if (GSTM_SPIN_NS) __nanosleep(GSTM_SPIN_NS);
-#pragma unroll
-                for (int k = 0; k < N; ++k)
-                    if (need[k] && (vl[k] & 1u)) vl[k] = prim::ld_relaxed(m.lock_ptr(m.lock_of(a[k])));   // l.28
-                locked = false;
-#pragma unroll
-                for (int k = 0; k < N; ++k) locked |= need[k] && (vl[k] & 1u);
-            }
-            n_spin += spins;
-            reconverge();
-            uint32_t newest = 0;
-#pragma unroll
-            for (int k = 0; k < N; ++k)
-                if (need[k]) newest = max(newest, vl[k] >> 1);
-            check_version(m, newest, mode);                          // l.30-33 (Q35)
-            reconverge();
-            ph(PH_BUFFER);
-            if constexpr (kUnroll) {
-#pragma unroll
-                for (int k = 0; k < N; ++k)
-                    if (need[k]) insert_read_lock(m.lock_of(a[k]));       // l.34
-            } else {
-                // local-memory logs: one inlined copy of the (looping) insert
-#pragma unroll 1
-                for (int k = 0; k < N; ++k) {
-                    uint32_t ak = 0;
-                    bool nk = false;
-#pragma unroll
-                    for (int j = 0; j < N; ++j)
-                        if (j == k) { ak = a[j]; nk = need[j]; }
-                    if (nk) insert_read_lock(m.lock_of(ak));         // l.34
-                }
-            }
+            check_small<N>(m, a, need, vl, mode);
         } else {
             uint32_t newest = 0;
 #pragma unroll
