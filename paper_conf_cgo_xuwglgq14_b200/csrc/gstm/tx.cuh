@@ -26,6 +26,16 @@
 #define GSTM_PV_ATTR __forceinline__
 #endif
 
+// ablation switches: validation loads chunked 8-wide with
+// local-memory logs (measured slower on EB: off); binary-search position in
+// the sorted local lock log (EB A=64 +15%, KM +8%: on)
+#ifndef GSTM_VBV_CHUNKED
+#define GSTM_VBV_CHUNKED 0
+#endif
+#ifndef GSTM_LOG_BSEARCH
+#define GSTM_LOG_BSEARCH 1
+#endif
+
 // a loop over a local-memory log: rolled in a compact Tx (kCompact), else
 // left to the compiler
 #define GSTM_LLOOP(...)                                        \
@@ -397,8 +407,20 @@ struct Tx {
             int pos = 0;
             if constexpr (SORTED) {
                 // ascending arrival (a record's words, a stripe) appends in O(1)
-                if (nl > 0 && (l_ent[nl - 1] >> 2) < id) pos = nl;
-                while (pos < nl && (l_ent[pos] >> 2) < id) ++pos;
+                if (nl > 0 && (l_ent[nl - 1] >> 2) < id) {
+                    pos = nl;
+                } else if constexpr (GSTM_LOG_BSEARCH) {
+                    // binary search: log2(n) dependent log reads instead of
+                    // up to n (EB's 16-64 random locks)
+                    int hi = nl;
+                    while (pos < hi) {
+                        const int mid = (pos + hi) >> 1;
+                        if ((l_ent[mid] >> 2) < id) pos = mid + 1;
+                        else hi = mid;
+                    }
+                } else {
+                    while (pos < nl && (l_ent[pos] >> 2) < id) ++pos;
+                }
             } else {
                 while (pos < nl && (l_ent[pos] >> 2) != id) ++pos;   // encounter order: find or append
             }
@@ -423,9 +445,22 @@ struct Tx {
 #pragma unroll
             for (int k = 0; k < RCAP; ++k)
                 if (k < nr) ok &= (cur[k] == r_val[k]);
-        } else if constexpr (!kCompact) {
+        } else if constexpr (!kCompact && !GSTM_VBV_CHUNKED) {
             for (int k = 0; k < nr; ++k)
                 ok &= (prim::ld_relaxed(m.val_ptr(r_addr[k])) == r_val[k]);
+        } else if constexpr (!kCompact) {
+            // kPvWidth (8) loads in flight per chunk: a rolled loop would
+            // wait for each load before issuing the next (HBM-latency chains
+            // on EB's 2^26-word hot set)
+            for (int k0 = 0; k0 < nr; k0 += kPvWidth) {
+                uint32_t cur[kPvWidth];
+#pragma unroll
+                for (int j = 0; j < kPvWidth; ++j)
+                    if (k0 + j < nr) cur[j] = prim::ld_relaxed(m.val_ptr(r_addr[k0 + j]));
+#pragma unroll
+                for (int j = 0; j < kPvWidth; ++j)
+                    if (k0 + j < nr) ok &= (cur[j] == r_val[k0 + j]);
+            }
         } else {
             // compact: kPvWidth loads in flight per chunk, one rolled copy per
             // call site (three sites in HV: A3.l71, l.76 and PostValidation's
