@@ -639,13 +639,14 @@ struct Tx {
     // instruction cache).  The lock inserts go through one
     // rolled loop for the same reason.
     template <int N>
-    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode)
+    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode,
+                                               uint32_t skip = 0u)
     {
         bool need[N];
         uint32_t vl[N];
         ph(PH_BUFFER);
 #pragma unroll
-        for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
+        for (int k = 0; k < N; ++k) need[k] = (k < n) && !((skip >> k) & 1u) && !raw_lookup(a[k], v[k]);
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));    // l.24

@@ -151,13 +151,14 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
     }
 
     template <int N>
-    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode)
+    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int mode,
+                                               uint32_t skip = 0u)
     {
         bool need[N];
         unsigned long long pv[N];
         ph(PH_BUFFER);
 #pragma unroll
-        for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
+        for (int k = 0; k < N; ++k) need[k] = (k < n) && !((skip >> k) & 1u) && !raw_lookup(a[k], v[k]);
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) pv[k] = prim::ld_relaxed_u64(m.pair_ptr(a[k]));

@@ -153,12 +153,13 @@ struct TxVbv {
     }
 
     template <int N>
-    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int)
+    __device__ __forceinline__ void read_batch(const Meta& m, const uint32_t (&a)[N], uint32_t (&v)[N], int n, int,
+                                               uint32_t skip = 0u)
     {
         if (!opaque) return;
         bool need[N];
 #pragma unroll
-        for (int k = 0; k < N; ++k) need[k] = (k < n) && !raw_lookup(a[k], v[k]);
+        for (int k = 0; k < N; ++k) need[k] = (k < n) && !((skip >> k) & 1u) && !raw_lookup(a[k], v[k]);
 #pragma unroll
         for (int k = 0; k < N; ++k)
             if (need[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));

@@ -52,9 +52,9 @@ struct StmCtx {
     int mode;
     __device__ __forceinline__ uint32_t read(uint32_t a) { return tx.read(m, a, mode); }
     template <int N>
-    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n)
+    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n, uint32_t skip = 0u)
     {
-        tx.template read_batch<N>(m, a, v, n, mode);
+        tx.template read_batch<N>(m, a, v, n, mode, skip);      // skip: words the caller reads later (RAW)
     }
     __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
     {
@@ -88,11 +88,11 @@ struct DirectCtx {
     bool bad;
     __device__ __forceinline__ uint32_t read(uint32_t a) { return prim::ld_relaxed(m.val_ptr(a)); }
     template <int N>
-    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n)
+    __device__ __forceinline__ void read_batch(const uint32_t (&a)[N], uint32_t (&v)[N], int n, uint32_t skip = 0u)
     {
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (k < n) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
+            if (k < n && !((skip >> k) & 1u)) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
     }
     __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
     {
@@ -407,7 +407,55 @@ struct EbWLT {
     // §6.3); a read of a word this transaction wrote earlier is served from
     // the write-set in program order (A3.l22-23).
     template <class Ctx>
-    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t, uint64_t, uint32_t& result)
+    __device__ __forceinline__ static void body(Ctx& c, const WlParams& p, uint64_t x, uint64_t t, uint64_t i,
+                                                uint32_t& result)
+    {
+        if constexpr (MAXA <= 16) body_regs(c, p, x, result);
+        else body_local(c, p, x, result);
+    }
+    // A <= 16: the read and write addresses stay in registers (compile-time
+    // indices); the non-RAW reads go out as ONE read_batch (the RAW ones
+    // skipped, then served from the write-set in program order); no local
+    // memory (the local arrays of body_local were written through to L2 on
+    // every attempt)
+    template <class Ctx>
+    __device__ __forceinline__ static void body_regs(Ctx& c, const WlParams& p, uint64_t x, uint32_t& result)
+    {
+        constexpr int RM = MAXA / 2;
+        const int A = static_cast<int>(p.n_accesses);
+        uint32_t ra[RM], wa[RM], rv[RM];
+#pragma unroll
+        for (int r = 0; r < RM; ++r) {
+            ra[r] = 2 * r < A ? static_cast<uint32_t>(gen::bounded(gen::draw(x, 2 * r), p.n_words)) : 0u;
+            wa[r] = 2 * r + 1 < A ? static_cast<uint32_t>(gen::bounded(gen::draw(x, 2 * r + 1), p.n_words)) : 0u;
+        }
+        uint32_t rawm = 0;                            // read r follows a write of the same word
+#pragma unroll
+        for (int r = 0; r < RM; ++r)
+#pragma unroll
+            for (int w = 0; w < r; ++w)
+                if (2 * w + 1 < A && wa[w] == ra[r]) rawm |= 1u << r;
+        c.template read_batch<RM>(ra, rv, (A + 1) / 2, rawm);
+        if (!c.ok()) return;
+        uint32_t acc = 0;
+#pragma unroll 1
+        for (int j = 0; j < A; ++j) {
+            const int r = j >> 1;
+            uint32_t aj = 0, vj = 0;
+#pragma unroll
+            for (int k = 0; k < RM; ++k)
+                if (k == r) { aj = (j & 1) ? wa[k] : ra[k]; vj = rv[k]; }
+            if ((j & 1) == 0) {
+                acc += ((rawm >> r) & 1u) ? c.read(aj) : vj;
+                if (!c.ok()) return;
+            } else {
+                c.write(aj, acc + lo32(gen::draw(x, A + j)));
+            }
+        }
+        result = acc;
+    }
+    template <class Ctx>
+    __device__ __forceinline__ static void body_local(Ctx& c, const WlParams& p, uint64_t x, uint32_t& result)
     {
         const uint32_t A = p.n_accesses;
         uint32_t addr[MAXA], ra[MAXA / 2], rv[MAXA / 2];
