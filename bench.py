@@ -473,6 +473,9 @@ CONFIGS = {
     # name: (workload, heap words, lock bits, params, T, K, steps, note)
     "ra_c0": ("ra", 1024, 10, dict(n_reads=4, n_writes=4, n_words=1024), 256, 1024, 3,
               "BASELINE configs[0]: random array, 1K words, 256 threads, 4R+4W, 2^10 locks"),
+    "ra_paper": ("ra", 1 << 23, 20, dict(n_reads=4, n_writes=4, n_words=1 << 23), 1 << 20, 4, 5,
+                 "random array, paper-shaped (SURVEY 8(d) extra row; P:310, P:313): 8M words, 2^20 locks, "
+                 "2^20 threads x 4, 4R+4W"),
     "ht_c2": ("ht", HT_BUCKETS + 2 * HT_THREADS * HT_K, HT_BITS,
               dict(ht_buckets=HT_BUCKETS, ht_key_range=HT_KEYS, ht_lookup_pct=90), HT_THREADS, HT_K, 5,
               "BASELINE configs[2]: chained hash table, 2^20 buckets, 2^22 threads x 4, 90/10 lookup/insert, "
