@@ -489,6 +489,9 @@ CONFIGS = {
     "km_c4": ("km", 1024 * 17, 20, dict(km_clusters=1024, km_dims=16), 1 << 24, 1, 1,
               "BASELINE configs[4]: k-means cluster update, 16M points, 1024 centroids x 16 dims, record = 17 "
               "words, 2^20 locks"),
+    "km_rec_lock": ("km", 1024 * 32, 20, dict(km_clusters=1024, km_dims=16, km_stride=32, lock_shift=5), 1 << 24, 1,
+                    1, "BASELINE configs[4] with one version lock per k-means record (SURVEY f4): records padded "
+                    "to 32 words (128 B), lock stripe 2^5 words"),
 }
 
 
@@ -542,7 +545,7 @@ def run_config(G, R, stream, flush, name, seed):
                 "stm_tbv": {"value": res["tbv"][0], "abort_ratio": res["tbv"][1]},
                 "fgl": res["fgl"][0], "cgl": cgl["value"], "speedup_vs_cgl": v / cgl["value"],
                 "threads": T, "tx_per_thread": K, "steps": steps})
-    records = (1024, 17) if wl == "km" else None
+    records = (1024, kw.get("km_stride", 17)) if wl == "km" else None
     roof = op_mix_roof(G, R, stream, wl, st, "hv", bool(gp.prelock_vbv), first_round_pipelined(wl, gp, st),
                        words, bits, False, T, records=records)
     per_tx = roof["ops_per_tx"]

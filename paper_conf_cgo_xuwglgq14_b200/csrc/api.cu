@@ -99,8 +99,10 @@ static size_t g_l2_limit[kMaxDevices];
 
 static cudaError_t l2_limits(int dev, size_t* max_persist, size_t* max_window)
 {
+    static std::mutex mu;
     static size_t mp[kMaxDevices], mw[kMaxDevices];
     if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    std::lock_guard<std::mutex> g(mu);
     if (!mw[dev]) {
         cudaDeviceProp pr;
         cudaError_t e = cudaGetDeviceProperties(&pr, dev);

@@ -16,7 +16,11 @@
 //     atomic on the global clock (A3.l83 aggregated over the warp);
 //   * the snapshot (A3.l4) is read once per warp and broadcast.
 #include <algorithm>
+#include <atomic>
 #include <cstdint>
+#include <mutex>
+#include <set>
+#include <tuple>
 #include <type_traits>
 #pragma once
 #include "kernels.cuh"
@@ -757,13 +761,16 @@ template <class K>
 inline uint64_t resident_blocks(K kernel, int block, int warps_per_sm = 0, size_t smem = 0)
 {
     // SM count of the CURRENT device (cached per device: one process may
-    // drive handles on several GPUs)
-    static int sms_of[64];
+    // drive handles on several GPUs; a racing first query stores the same value)
+    static std::atomic<int> sms_of[64];
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64) {
-        if (!sms_of[dev]) cudaDeviceGetAttribute(&sms_of[dev], cudaDevAttrMultiProcessorCount, dev);
-        sms = sms_of[dev];
+        sms = sms_of[dev].load(std::memory_order_relaxed);
+        if (!sms) {
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            sms_of[dev].store(sms, std::memory_order_relaxed);
+        }
     } else {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     }
@@ -778,9 +785,19 @@ inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream
                               size_t smem = 0)
 {
     if (smem > 48 * 1024) {
-        const cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                   static_cast<int>(smem));
-        if (e != cudaSuccess) return e;
+        // opt in to > 48 KB of dynamic shared memory once per (kernel, device, size)
+        static std::mutex mu;
+        static std::set<std::tuple<const void*, int, size_t>> done;
+        int dev = 0;
+        cudaGetDevice(&dev);
+        const auto key = std::make_tuple(reinterpret_cast<const void*>(kernel), dev, smem);
+        std::lock_guard<std::mutex> g(mu);
+        if (!done.count(key)) {
+            const cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                       static_cast<int>(smem));
+            if (e != cudaSuccess) return e;
+            done.insert(key);
+        }
     }
     uint64_t grid = (kp.T + block - 1) / block;
     grid = std::min<uint64_t>(grid, resident_blocks(kernel, block, kp.max_threads ? 0 : warps_per_sm, smem));
