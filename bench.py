@@ -211,10 +211,9 @@ def cpu_baseline(T, K, seed, reps=5):
     out = json.loads(pinned.stdout.strip().splitlines()[-1])
     med = statistics.median(out["times_s"])
     return {"value": T * K / med, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"serial oracle (oracle/serial.c or_serial, gcc -O2, 1 thread, {how}) over one full step: "
-                      f"{T} threads x {K} tx = {T * K} bank transfers; median of {reps} runs "
-                      f"({min(out['times_s']):.3f}-{max(out['times_s']):.3f} s)",
-            "host_cores": os.cpu_count(), "cpu_model": cpu_model(), "affinity": out["affinity"]}
+            "sample": f"oracle/serial.c or_serial (-O2, 1 thread, {how}), one full step ({T * K} transfers), "
+                      f"median of {reps} ({min(out['times_s']):.3f}-{max(out['times_s']):.3f} s)",
+            "host_cores": os.cpu_count(), "cpu_model": cpu_model()}
 
 
 def run_reference(args):
@@ -416,8 +415,7 @@ def roofline_object(achieved_tx_s, roof, maxf, sectors_per_tx, note):
     return {"bound": "l2", "achieved": achieved_tx_s * b / 1e9, "peak": roof["roof_tx_per_s"] * b / 1e9,
             "unit": "GB/s", "frac": achieved_tx_s / roof["roof_tx_per_s"], "traffic": None,
             "roof_tx_per_s": roof["roof_tx_per_s"], "roof_threads": roof["threads"],
-            "roof_source": "measured: gstm_ubench_mix (the committed transactions' exact op mix, no conflicts, "
-                           "max over occupancy)",
+            "roof_source": "measured op-mix roof (gstm_ubench_mix, DESIGN.md 7.2)",
             "max_formula_tx_per_s": maxf, "frac_max_formula": achieved_tx_s / maxf,
             "bytes_per_tx": b, "round_trips_per_tx": roof["round_trips_per_tx"], "note": note}
 
@@ -495,6 +493,11 @@ CONFIGS = {
 }
 
 
+def sig(x: float, n: int = 4) -> float:
+    """x to n significant digits (keeps the JSON line short)."""
+    return float(f"{x:.{n}g}")
+
+
 def first_round_pipelined(wl, gp, st) -> bool:
     """Does the kernel issue a transaction's first lock round all at once
     ?  Register logs (bank) always may; local-memory logs only
@@ -510,7 +513,8 @@ def run_config(G, R, stream, flush, name, seed):
     import torch
     wl, words, bits, kw, T, K, steps, note = CONFIGS[name]
     reinit = wl == "ht"
-    out = {"workload": note}
+    out = {}
+    detail_extra = {"workload": note}
 
     def make(mode, **extra):
         g = G.Gstm(words, bits)
@@ -530,7 +534,8 @@ def run_config(G, R, stream, flush, name, seed):
             probes[cap] = g.run(wl, T, 1, seed + 5).tx_per_s
             g.close()
         extra["max_threads"] = max(probes, key=probes.get)
-        out["stm_concurrency_probe"] = probes
+        detail_extra["stm_concurrency_probe"] = probes
+        out["max_threads"] = extra["max_threads"]
     res = {}
     for mode in ("hv", "tbv", "fgl"):
         g = make(mode, **(extra if mode != "fgl" else {}))
@@ -541,27 +546,33 @@ def run_config(G, R, stream, flush, name, seed):
         torch.cuda.synchronize()
     cgl = cgl_rate(G, lambda m: make(m), wl, T, K, seed, reinit=reinit)
     v, ab, st, gp = res["hv"]
-    out.update({"stm": {"mode": "hv", "value": v, "abort_ratio": ab},
-                "stm_tbv": {"value": res["tbv"][0], "abort_ratio": res["tbv"][1]},
-                "fgl": res["fgl"][0], "cgl": cgl["value"], "speedup_vs_cgl": v / cgl["value"],
-                "threads": T, "tx_per_thread": K, "steps": steps})
+    # compact (the driver keeps the line): STM-HV rate and abort ratio, STM-TBV,
+    # FGL, CGL (tx/s), HV / CGL; the descriptions and probes go to stderr
+    out.update({"stm_hv": sig(v), "abort_hv": sig(ab), "stm_tbv": sig(res["tbv"][0]), "abort_tbv": sig(res["tbv"][1]),
+                "fgl": sig(res["fgl"][0]), "cgl": sig(cgl["value"]), "speedup_vs_cgl": sig(v / cgl["value"]),
+                "T": T, "K": K})
     records = (1024, kw.get("km_stride", 17)) if wl == "km" else None
     roof = op_mix_roof(G, R, stream, wl, st, "hv", bool(gp.prelock_vbv), first_round_pipelined(wl, gp, st),
                        words, bits, False, T, records=records)
     per_tx = roof["ops_per_tx"]
     sectors = per_tx["ld"] + per_tx["atom"] + per_tx["st"]
     peaks = class_peaks(G, words * 4 + (4 << bits), False)
-    out["roof"] = {"roof_tx_per_s": roof["roof_tx_per_s"], "frac": v / roof["roof_tx_per_s"],
-                   "threads": roof["threads"], "round_trips_per_tx": roof["round_trips_per_tx"],
-                   "max_formula_tx_per_s": max_formula(per_tx, peaks),
-                   "kind": "contention: 1024 records, one serial chain each" if records else "op mix, no conflicts"}
+    out["roof"] = sig(roof["roof_tx_per_s"])
+    out["frac"] = sig(v / roof["roof_tx_per_s"])
+    out["roof_kind"] = "contention" if records else "op_mix"
+    detail_extra["roof"] = {"threads": roof["threads"], "round_trips_per_tx": roof["round_trips_per_tx"],
+                            "max_formula_tx_per_s": max_formula(per_tx, peaks),
+                            "kind": "contention: 1024 records / lock-holding time" if records else
+                                    "op mix of the committed transactions, no conflicts"}
     if wl == "eb" and words * 4 > (128 << 20):
         # the hot set exceeds L2: SURVEY §8(d) counts every access of the
         # transaction as one 32 B HBM sector -- against the measured HBM peak
         hbm = float(measured_peaks()[0].get("hbm_gbs", 6650.0))
         gbs = v * 32.0 * sectors / 1e9
-        out["hbm"] = {"achieved_gbs": gbs, "peak_gbs": hbm, "frac": gbs / hbm, "bytes_per_tx": 32.0 * sectors}
-    detail = {"cgl": cgl, "roof": {k: v for k, v in roof.items() if k != "program"}, "class_peaks": peaks,
+        out["hbm_frac"] = sig(gbs / hbm)
+        detail_extra["hbm"] = {"achieved_gbs": gbs, "peak_gbs": hbm, "bytes_per_tx": 32.0 * sectors}
+    detail = {**detail_extra, "cgl": cgl, "roof_full": {k: v for k, v in roof.items() if k != "program"},
+              "class_peaks": peaks,
               "hv_stats": {k: getattr(st, k) for k in KEYS}}
     return out, detail
 
@@ -727,8 +738,7 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
     e2e_ms = a.elapsed_time(b)
     extra["e2e"] = {"value": (st2.commits + st2.commits_ro) / (e2e_ms * 1e-3), "unit": UNIT,
                     "h2d_bytes_per_step": ACCOUNTS * 4, "d2h_bytes_per_step": ACCOUNTS * 4,
-                    "api": "gstm_run_host_async (pinned host buffers, copies pipelined with the neighbouring "
-                           "steps), gstm_join + CUDA events", "steps": n_e2e}
+                    "api": "gstm_run_host_async (pinned host buffers, pipelined copies)", "steps": n_e2e}
     if not args.no_cgl:
         mk = lambda m: Variant(m).handle(G, stream)                              # noqa: E731
         cgl = cgl_rate(G, mk, "bank", T, K, seed0)
@@ -751,8 +761,7 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
         if fgl:
             best = max(fgl, key=lambda v: v["value"])
             extra["fgl"] = {"value": best["value"], "unit": UNIT}
-        extra["auto_split"] = {"value": detail["bank_variants"]["auto/split"]["value"],
-                               "note": "the paper's STM-Optimized rule (P:252) on the paper's split layout"}
+        extra["auto_split"] = sig(detail["bank_variants"]["auto/split"]["value"])   # STM-Optimized, split layout
     # the roofline of the headline kernel: the committed transactions' own
     # op mix, measured on a scratch handle of the same layout
     paired = var.layout == "paired"
@@ -763,10 +772,7 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
     maxf = max_formula(roof["ops_per_tx"], peaks)
     ops = roof["ops_per_tx"]
     extra["roofline"] = roofline_object(value / world, roof, maxf, ops["ld"] + ops["atom"] + ops["st"],
-                                        "launch duration = CUDA events on the launching stream around each step "
-                                        "(prepare + stm_kernel + finish; stm_kernel is 99.8% of it, "
-                                        "profiles/r01_bank_headline_launches.csv); traffic null: ncu DRAM bytes "
-                                        "come from a separate capture (profiles/), not from this run")
+                                        "CUDA events per step (stm_kernel 99.7% of it); traffic: ncu, profiles/")
     detail["bank_roof"] = {k: v for k, v in roof.items() if k != "program"}
     detail["bank_class_peaks"] = peaks
     if not args.no_configs:
@@ -779,7 +785,7 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
             except Exception as e:          # one config's failure must not lose the line
                 cfgs[name] = {"error": f"{type(e).__name__}: {e}"}
                 torch.cuda.synchronize()
-            cfgs[name]["wall_s"] = round(time.perf_counter() - t0, 2)
+            cfgs[name]["wall_s"] = round(time.perf_counter() - t0, 1)
             sys.stderr.write(f"config {name}: {json.dumps(cfgs[name])}\n")
             sys.stderr.flush()
         extra["configs"] = cfgs

@@ -367,6 +367,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
+            tx.insert_deferred_reads(m);                              // lock_log_at_commit: the full log first
             const bool pipelined = tries == 0 && lock_aborts < p.lock_pipeline &&
                                    (TX::kUnroll || tx.nl <= static_cast<int>(p.pipeline_max_locks));
             if (pipelined) cnt.inc(S_PIPELINED);
