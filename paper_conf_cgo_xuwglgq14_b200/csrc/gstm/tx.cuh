@@ -360,16 +360,20 @@ struct Tx {
     // of the set of entries (insert order does not matter, Q4), so the
     // acquisition order and the livelock-freedom argument are the same; a
     // read-only transaction (HT lookups: 90%) skips the sorting it never uses.
+    // (register-resident logs always insert at encounter time: a deferred
+    // pass would index them dynamically and move them to local memory)
     __device__ __forceinline__ void insert_read_lock(uint32_t id)
     {
-        if (!defer_rd) insert_lock((id << 2) | 1u);
+        if (kUnroll || !defer_rd) insert_lock((id << 2) | 1u);
     }
     __device__ __forceinline__ void insert_deferred_reads(const Meta& m)
     {
-        if (!defer_rd || deferred_done) return;
-        deferred_done = true;
+        if constexpr (!kUnroll) {
+            if (!defer_rd || deferred_done) return;
+            deferred_done = true;
 #pragma unroll 1
-        for (int k = 0; k < nr; ++k) insert_lock((m.lock_of(r_addr[k]) << 2) | 1u);
+            for (int k = 0; k < nr; ++k) insert_lock((m.lock_of(r_addr[k]) << 2) | 1u);
+        }
     }
 
     // ---- P:113-115, A3.l34/l38: sorted insert into the local lock log ----

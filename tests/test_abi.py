@@ -46,6 +46,18 @@ def test_library_is_sm100a_and_self_contained(so):
     assert "ATOMG.E.OR.64.STRONG.GPU" in paired and "LDG.E.64.STRONG.GPU" in paired
     # one MEMBAR (the l.82 release fence) in the paper layout, none paired
     assert split.count("MEMBAR") == 1 and paired.count("MEMBAR") == 0
+    # the bank kernels' logs stay in registers: no local-memory access at all
+    # (a dynamically indexed log pass once moved them to a 128 B stack frame)
+    for body in (split, paired):
+        assert "LDL" not in body and "STL" not in body
+    # the shared-memory log policy really uses shared memory: KM's
+    # and RA's HV kernels keep their logs in LDS/STS (RA: no local memory at
+    # all; KM keeps a few batch temporaries of its 17-word read on the stack)
+    for wl in ("4KmWL", "4RaWL"):
+        k = funcs[f"_ZN4gstm10stm_kernelINS_{wl}ELi1ELb0ELi0EEEvNS_7KParamsE"]
+        assert k.count("LDS") >= 16 and k.count("STS") >= 16
+    ra = funcs["_ZN4gstm10stm_kernelINS_4RaWLELi1ELb0ELi0EEEvNS_7KParamsE"]
+    assert "LDL" not in ra and "STL" not in ra
 
 
 def test_loads_and_host_only_calls(so):

@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--mode", default="hv")
     ap.add_argument("--launches", type=int, default=2)
     ap.add_argument("--set", nargs="*", default=[], help="gstm_params_t overrides k=v")
+    ap.add_argument("--paired", action="store_true", help="the paired layout (one lock per word)")
     a = ap.parse_args()
     B.build()
     from paper_conf_cgo_xuwglgq14_b200 import gstm as G
@@ -33,7 +34,9 @@ def main():
         wl, T, K = "bank", bench.THREADS, bench.TX_PER_THREAD
     else:
         wl, words, bits, p, T, K, _, _ = bench.CONFIGS[a.config]
-        g = G.Gstm(words, bits)
+        if a.paired:
+            bits = max(bits, (words - 1).bit_length())
+        g = G.Gstm(words, bits, paired=a.paired)
         g.set_workload_defaults(wl, **dict(p, **kv))
     g.set_mode(a.mode)
     for k in range(a.launches):
