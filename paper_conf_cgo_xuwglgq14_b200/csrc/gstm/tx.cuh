@@ -217,6 +217,7 @@ struct Tx {
 #endif
     int nr, nw, nl, n_acq;
     bool defer_rd = false;                // lock_log_at_commit: read locks inserted at TXCommit
+    bool pipelined_round = false;         // the last commit_acquire issued a pipelined first round
     bool deferred_done;
     uint32_t snapshot;
     bool opaque, passTBV, overflow;
@@ -931,11 +932,17 @@ struct Tx {
     // Commit steps up to the write-back (A3.l67-78).  Returns C_OK when all
     // locks are held and the read-set is valid, C_LOCK on a lock conflict
     // (nothing held; retry, l.73-74), or an abort cause (nothing held).
-    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
+    // want_pipe: this round may be the pipelined first round (§6.4); it is,
+    // for local-memory logs, only if the (complete) log has at most
+    // max_pipe_locks entries -- pipelined_round reports the decision
+    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool want_pipe = false,
+                                                  uint32_t max_pipe_locks = 8u)
     {
         ph(PH_BUFFER);
         insert_deferred_reads(m);
         compact();
+        const bool pipelined = want_pipe && (kUnroll || nl <= static_cast<int>(max_pipe_locks));
+        pipelined_round = pipelined;
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72

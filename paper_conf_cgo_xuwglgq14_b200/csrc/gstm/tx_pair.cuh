@@ -463,11 +463,17 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
         return true;
     }
 
-    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool pipelined = false)
+    // want_pipe: this round may be the pipelined first round (§6.4); it is,
+    // for local-memory logs, only if the (complete) log has at most
+    // max_pipe_locks entries -- pipelined_round reports the decision
+    __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool want_pipe = false,
+                                                  uint32_t max_pipe_locks = 8u)
     {
         ph(PH_BUFFER);
         B::insert_deferred_reads(m);
         B::compact();
+        const bool pipelined = want_pipe && (kUnroll || nl <= static_cast<int>(max_pipe_locks));
+        B::pipelined_round = pipelined;
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72

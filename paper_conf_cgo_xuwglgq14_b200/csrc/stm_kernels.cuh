@@ -367,11 +367,9 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
-            tx.insert_deferred_reads(m);                              // lock_log_at_commit: the full log first
-            const bool pipelined = tries == 0 && lock_aborts < p.lock_pipeline &&
-                                   (TX::kUnroll || tx.nl <= static_cast<int>(p.pipeline_max_locks));
-            if (pipelined) cnt.inc(S_PIPELINED);
-            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, pipelined);
+            const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline;
+            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks);
+            if (tx.pipelined_round) cnt.inc(S_PIPELINED);
             if (r == C_OK) {
                 got = true;
                 // l.79-82
