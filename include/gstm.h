@@ -336,6 +336,16 @@ int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per
  * with op 0 BEGIN, 1 READ, 2 WRITE, 3 COMMIT; out: n_ops x 4 words (format in
  * DESIGN.md §5.3).  mode: GSTM_MODE_HV or GSTM_MODE_TBV. */
 int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx);
+/* As gstm_script, with op 4 READ2 {4, slot, word a, word b}: a batched read
+ * of two words (the kernels' read_batch, reading Q35; out [value(a),
+ * value(b), snapshot, isOpaque | PostValidation ran << 1]) and the log
+ * storage of the transactions: log_policy 0 local memory (capacity 64 reads,
+ * 64 writes, 128 locks; = gstm_script), 1 register-resident, fully unrolled
+ * (8 / 8 / 16: the bank kernel's code), 2 shared memory [entry][lane] (16 /
+ * 16 / 32).  A transaction that exceeds its capacity reports
+ * isOpaque = 0 (log overflow). */
+int gstm_script_ex(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
+                   int log_policy);
 /* Insert entries (id<<2 | wr<<1 | rd, id < 2^20) into a device lock log
  * (variant 0: register-resident, capacity 16; 1: local memory, capacity 256;
  * both sorted by id.  Variants 2 and 3: the same capacities in

@@ -39,7 +39,7 @@ WL_RA, WL_BANK, WL_HT, WL_EB, WL_KM = 0, 1, 2, 3, 4
 WORKLOADS = {"ra": WL_RA, "bank": WL_BANK, "ht": WL_HT, "eb": WL_EB, "km": WL_KM}
 RO_FLAG = 0x80000000
 MODE_HV, MODE_TBV = 1, 2
-OP_BEGIN, OP_READ, OP_WRITE, OP_COMMIT = 0, 1, 2, 3
+OP_BEGIN, OP_READ, OP_WRITE, OP_COMMIT, OP_READ2 = 0, 1, 2, 3, 4   # OP_READ2: batched read (Q35)
 C_OK, C_OPACITY, C_PREVBV, C_TBV, C_COMMITVBV, C_READONLY = 0, 1, 2, 3, 4, 5
 
 

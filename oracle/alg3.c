@@ -143,7 +143,9 @@ static uint32_t TXRead(stm_t* g, tx_t* tx, uint64_t addr)
     do versionLock = g->g_lockTab[hash_addr(g, addr)];              /* l.27-28 */
     while ((versionLock & 1u) != 0);                                /* l.29 (Q8) */
     uint64_t version = versionLock >> 1;                            /* l.30 */
-    if (version > tx->snapshot) {                                   /* l.31 */
+    /* l.31; reading Q43: a transaction that is no longer opaque does not
+     * re-validate (Figure 1 breaks out at the first !isOpaque) */
+    if (tx->isOpaque && version > tx->snapshot) {
         if (g->mode == OR_MODE_HV) {
             if (!PostValidation(g, tx, version))                    /* l.32 */
                 tx->isOpaque = 0;                                   /* l.33 */
@@ -153,6 +155,49 @@ static uint32_t TXRead(stm_t* g, tx_t* tx, uint64_t addr)
     }
     lock_log_insert(tx->l_lockTab, &tx->n_locks, MAXLOG, (hash_addr(g, addr) << 2) | 1u); /* l.34 */
     return val;                                                     /* l.35 */
+}
+
+/* Reading Q35: a batched TXRead of two words whose
+ * addresses are known together -- l.22-25 for each word (RAW from the
+ * write-set, value load, append), one l.26 fence, l.27-30 for each word, then
+ * ONE timestamp check l.31-33 with the newest version of the batch (the
+ * outcome sequential TXReads reach: a read-set consistent at a snapshot >=
+ * every version read), then l.34 for each word.  Output: vals[2]. */
+static void TXRead2(stm_t* g, tx_t* tx, uint64_t a0, uint64_t a1, uint32_t* vals)
+{
+    uint64_t addr[2] = {a0, a1};
+    int need[2];
+    for (int i = 0; i < 2; ++i) {
+        need[i] = 1;
+        if (tx->bloom & bloom_bit(addr[i]))                         /* l.22 */
+            for (int k = 0; k < tx->n_writes; ++k)
+                if (tx->writes[k].addr == addr[i]) { vals[i] = tx->writes[k].val; need[i] = 0; break; } /* l.23 */
+        if (need[i]) {
+            vals[i] = g->heap[addr[i]];                             /* l.24 */
+            if (tx->n_reads < MAXLOG) {                             /* l.25 */
+                tx->reads[tx->n_reads].addr = addr[i]; tx->reads[tx->n_reads].val = vals[i]; tx->n_reads++;
+            }
+        }
+    }
+    /* l.26 threadfence() */
+    uint64_t newest = 0;
+    for (int i = 0; i < 2; ++i) {
+        if (!need[i]) continue;
+        uint32_t versionLock;
+        do versionLock = g->g_lockTab[hash_addr(g, addr[i])];       /* l.27-28 */
+        while ((versionLock & 1u) != 0);                            /* l.29 */
+        if ((versionLock >> 1) > newest) newest = versionLock >> 1; /* l.30 */
+    }
+    if (tx->isOpaque && newest > tx->snapshot) {                    /* l.31, once (Q35; Q43) */
+        if (g->mode == OR_MODE_HV) {
+            if (!PostValidation(g, tx, newest))                     /* l.32 */
+                tx->isOpaque = 0;                                   /* l.33 */
+        } else {
+            tx->isOpaque = 0;
+        }
+    }
+    for (int i = 0; i < 2; ++i)
+        if (need[i]) lock_log_insert(tx->l_lockTab, &tx->n_locks, MAXLOG, (hash_addr(g, addr[i]) << 2) | 1u); /* l.34 */
 }
 
 /* 36: TXWrite(addr, val) */
@@ -275,7 +320,8 @@ int or_alg3_script(int mode, int prelock_vbv, uint32_t bits,
         uint32_t op = ops[4 * k], slot = ops[4 * k + 1], addr = ops[4 * k + 2], val = ops[4 * k + 3];
         uint32_t* o = &out[4 * k];
         o[0] = o[1] = o[2] = o[3] = 0;
-        if (slot >= (uint32_t)n_tx || (op != OR_OP_BEGIN && op != OR_OP_COMMIT && addr >= words)) return -2 - k;
+        if (slot >= (uint32_t)n_tx || (op != OR_OP_BEGIN && op != OR_OP_COMMIT && addr >= words) ||
+            (op == OR_OP_READ2 && val >= words)) return -2 - k;
         tx_t* tx = &g_txs[slot];
         switch (op) {
         case OR_OP_BEGIN:
@@ -290,6 +336,14 @@ int or_alg3_script(int mode, int prelock_vbv, uint32_t bits,
         case OR_OP_WRITE:
             TXWrite(&g, tx, addr, val);
             break;
+        case OR_OP_READ2: {                 /* out: [val(addr), val(value field), snapshot, isOpaque | postval << 1] */
+            uint32_t v2[2];
+            tx->postval_ran = 0;
+            TXRead2(&g, tx, addr, val, v2);
+            o[0] = v2[0]; o[1] = v2[1]; o[2] = (uint32_t)tx->snapshot;
+            o[3] = (uint32_t)tx->isOpaque | ((uint32_t)tx->postval_ran << 1);
+            break;
+        }
         case OR_OP_COMMIT: {
             int cause; uint64_t stamp;
             tx->vbv_runs = 0;

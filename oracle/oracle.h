@@ -117,7 +117,8 @@ int or_replay(const or_params_t* p, uint32_t* heap, uint64_t words,
 
 /* ---------------- alg3.c: Algorithm 3 sequential model ------------------- */
 enum { OR_MODE_HV = 1, OR_MODE_TBV = 2 };
-enum { OR_OP_BEGIN = 0, OR_OP_READ = 1, OR_OP_WRITE = 2, OR_OP_COMMIT = 3 };
+enum { OR_OP_BEGIN = 0, OR_OP_READ = 1, OR_OP_WRITE = 2, OR_OP_COMMIT = 3,
+       OR_OP_READ2 = 4 /* batched TXRead of words (addr, value field), reading Q35 */ };
 /* Abort causes reported by COMMIT. */
 enum { OR_C_OK = 0, OR_C_OPACITY = 1, OR_C_PREVBV = 2, OR_C_TBV = 3,
        OR_C_COMMITVBV = 4, OR_C_READONLY = 5 };

@@ -921,13 +921,21 @@ int gstm_dump_descr(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per
 
 int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx)
 {
-    if (!h || !ops || !out || n_ops < 0 || n_tx < 1 || n_tx > 8 || (mode != GSTM_MODE_HV && mode != GSTM_MODE_TBV)) {
+    return gstm_script_ex(h, mode, prelock_vbv, ops, n_ops, out, n_tx, 0);
+}
+
+int gstm_script_ex(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
+                   int log_policy)
+{
+    if (!h || !ops || !out || n_ops < 0 || n_tx < 1 || n_tx > 8 || (mode != GSTM_MODE_HV && mode != GSTM_MODE_TBV) ||
+        log_policy < 0 || log_policy > 2) {
         set_error("gstm_script: bad argument");
         return GSTM_EINVAL;
     }
     for (int k = 0; k < n_ops; ++k) {
-        const uint32_t op = ops[4 * k], slot = ops[4 * k + 1], word = ops[4 * k + 2];
-        if (op > 3 || slot >= static_cast<uint32_t>(n_tx) || ((op == 1 || op == 2) && word >= h->heap_words)) {
+        const uint32_t op = ops[4 * k], slot = ops[4 * k + 1], word = ops[4 * k + 2], val = ops[4 * k + 3];
+        if (op > 4 || slot >= static_cast<uint32_t>(n_tx) || ((op == 1 || op == 2 || op == 4) && word >= h->heap_words) ||
+            (op == 4 && val >= h->heap_words)) {
             set_error("gstm_script: bad op %d", k);
             return GSTM_EINVAL;
         }
@@ -945,7 +953,7 @@ int gstm_script(gstm_t* h, int mode, int prelock_vbv, const uint32_t* ops, int n
     m.lock_shift = 0;
     m.vshift = m.lshift = h->paired ? 1u : 0u;
     if (e == cudaSuccess) e = cudaMemcpyAsync(dops, ops, n_ops * 16, cudaMemcpyHostToDevice, h->stream);
-    if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, h->stream);
+    if (e == cudaSuccess) e = launch_script(m, mode, prelock_vbv, dops, n_ops, dout, n_tx, log_policy, h->stream);
     if (e == cudaSuccess) e = cudaMemcpyAsync(out, dout, n_ops * 16, cudaMemcpyDeviceToHost, h->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
     cudaFree(dops);

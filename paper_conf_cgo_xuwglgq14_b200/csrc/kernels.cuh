@@ -78,7 +78,7 @@ cudaError_t launch_init_heap(int workload, uint32_t* heap, uint64_t words, int v
 cudaError_t launch_pack(uint32_t* plain, uint32_t* pairs, uint64_t words, int to_pairs, cudaStream_t s);
 cudaError_t launch_lock_halves(uint32_t* pairs, uint64_t words, uint32_t* out, cudaStream_t s);
 cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
-                          cudaStream_t s);
+                          int policy, cudaStream_t s);
 cudaError_t launch_lock_log(const uint32_t* entries, int n, uint32_t* out, int* out_n, int variant, cudaStream_t s);
 cudaError_t launch_km_assign(const KParams& kp, uint32_t* cluster, cudaStream_t s);
 cudaError_t launch_km_init_centroids(const Meta& m, uint64_t c0, uint64_t n, cudaStream_t s);

@@ -7,6 +7,7 @@
 //   READ   [value, isOpaque, snapshot, postvalidation ran]
 //   WRITE  [0, 0, 0, 0]
 //   COMMIT [ok, cause, stamp, vbv runs]
+//   READ2  [value(word), value(value field), snapshot, isOpaque | PostValidation ran << 1]
 #include <cstdint>
 #include "kernels.cuh"
 
@@ -18,8 +19,12 @@ template <class ScriptTx>
 __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out,
                               int n_tx)
 {
+    // shared-memory logs: transaction s takes column s of one [word][32] region
+    __shared__ uint32_t region[ScriptTx::kSmem ? 32 * ScriptTx::kSmemWords : 1];
     if (threadIdx.x || blockIdx.x) return;
     ScriptTx tx[kMaxScriptTx];
+    if constexpr (ScriptTx::kSmem)
+        for (int s = 0; s < kMaxScriptTx; ++s) tx[s].bind_smem(region, s);
     for (int k = 0; k < n_ops; ++k) {
         const uint32_t op = ops[4 * k], s = ops[4 * k + 1], a = ops[4 * k + 2], v = ops[4 * k + 3];
         uint32_t o[4] = {0, 0, 0, 0};
@@ -44,6 +49,17 @@ __global__ void script_kernel(const Meta m, int mode, int prelock, const uint32_
             case 2:  // WRITE
                 x.write(m, a, v);
                 break;
+            case 4: {  // READ2: batched read of words a and v (read_batch, reading Q35)
+                x.n_postval = 0;
+                const uint32_t aa[2] = {a, v};
+                uint32_t vv[2] = {0u, 0u};
+                x.template read_batch<2>(m, aa, vv, 2, mode);
+                o[0] = vv[0];
+                o[1] = vv[1];
+                o[2] = x.snapshot;
+                o[3] = (x.opaque ? 1u : 0u) | (x.n_postval ? 2u : 0u);
+                break;
+            }
             case 3: {  // COMMIT
                 x.n_vbv = 0;
                 if (!x.opaque) { o[1] = C_OPACITY; break; }
@@ -95,12 +111,26 @@ __global__ void lock_log_kernel(const uint32_t* e, int n, uint32_t* out, int* ou
     *out_n = tx.overflow ? -1 : tx.nl;
 }
 
+// policy 0: local-memory logs (Tx<64,64,128>); 1: register-resident logs,
+// the fully unrolled code the bank kernel runs (Tx<8,8,16>); 2: shared-memory
+// logs, [entry][lane] (Tx<16,16,32, SMEM>)
 cudaError_t launch_script(const Meta& m, int mode, int prelock, const uint32_t* ops, int n_ops, uint32_t* out, int n_tx,
-                          cudaStream_t s)
+                          int policy, cudaStream_t s)
 {
-    if (n_tx > kMaxScriptTx) return cudaErrorInvalidValue;
-    if (m.vshift) script_kernel<TxPair<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
-    else script_kernel<Tx<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    if (n_tx > kMaxScriptTx || policy < 0 || policy > 2) return cudaErrorInvalidValue;
+    if (m.vshift) {
+        if (policy == 1) script_kernel<TxPair<8, 8, 16>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+        else if (policy == 2)
+            script_kernel<TxPair<16, 16, 32, false, true, false, false, true>><<<1, 32, 0, s>>>(m, mode, prelock, ops,
+                                                                                              n_ops, out, n_tx);
+        else script_kernel<TxPair<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    } else {
+        if (policy == 1) script_kernel<Tx<8, 8, 16>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+        else if (policy == 2)
+            script_kernel<Tx<16, 16, 32, false, true, false, false, true>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops,
+                                                                                          out, n_tx);
+        else script_kernel<Tx<64, 64, 128>><<<1, 32, 0, s>>>(m, mode, prelock, ops, n_ops, out, n_tx);
+    }
     return cudaGetLastError();
 }
 

@@ -39,7 +39,7 @@ EXPORTS = [
     "gstm_stats_total", "gstm_reset_stats_total", "gstm_phase_cycles",
     "gstm_read_tx_log", "gstm_run_host", "gstm_descr_words", "gstm_dump_descr", "gstm_script",
     "gstm_lock_log", "gstm_ubench", "gstm_km_recenter", "gstm_run_host_async", "gstm_join", "gstm_sync",
-    "gstm_ubench_mix",
+    "gstm_ubench_mix", "gstm_script_ex",
 ]
 
 
@@ -137,6 +137,7 @@ def lib(flavour: str = ""):
             "gstm_descr_words": (i32, [V, i32]),
             "gstm_dump_descr": (i32, [V, i32, u64, u32, u64, V, u32]),
             "gstm_script": (i32, [V, i32, i32, V, i32, V, i32]),
+            "gstm_script_ex": (i32, [V, i32, i32, V, i32, V, i32, i32]),
             "gstm_lock_log": (i32, [V, i32, V, i32]),
             "gstm_ubench": (i32, [i32, u64, u64, u32, P(C.c_double), P(C.c_double)]),
             "gstm_ubench_mix": (i32, [V, u64, V, u32, u64, u32, u32, P(C.c_double), P(C.c_double)]),
@@ -401,11 +402,13 @@ class Gstm:
                "gstm_dump_descr", self._L)
         return out.reshape(n_threads * tx_per_thread, wpt)
 
-    def script(self, mode, ops, n_tx: int = 4, prelock_vbv: bool = True) -> np.ndarray:
+    def script(self, mode, ops, n_tx: int = 4, prelock_vbv: bool = True, log_policy: int = 0) -> np.ndarray:
+        """Scripted interleaving (gstm_script_ex); log_policy 0 local, 1
+        register-resident, 2 shared-memory logs."""
         ops = np.ascontiguousarray(np.asarray(ops, dtype=np.uint32).reshape(-1, 4))
         out = np.zeros_like(ops)
-        _check(self._L.gstm_script(self.h, _mode(mode), 1 if prelock_vbv else 0, _ptr(ops), ops.shape[0],
-                                 _ptr(out), n_tx), "gstm_script", self._L)
+        _check(self._L.gstm_script_ex(self.h, _mode(mode), 1 if prelock_vbv else 0, _ptr(ops), ops.shape[0],
+                                    _ptr(out), n_tx, log_policy), "gstm_script_ex", self._L)
         return out
 
 

@@ -22,11 +22,11 @@ def _built():
     U.ensure_built()
 
 
-def _script_both(mode, bits, heap0, clock0, ops, n_tx, prelock):
+def _script_both(mode, bits, heap0, clock0, ops, n_tx, prelock, policy=0):
     g = G.Gstm(heap0.size, bits, paired=True)
     g.write_heap(heap0)
     g.set_clock(clock0)
-    out_gpu = g.script(mode, ops, n_tx=n_tx, prelock_vbv=prelock)
+    out_gpu = g.script(mode, ops, n_tx=n_tx, prelock_vbv=prelock, log_policy=policy)
     heap_o = heap0.copy()
     locks_o = np.zeros(1 << bits, dtype=np.uint32)
     out_o, clk_o = O.alg3_script(mode, bits, heap_o, locks_o, clock0, ops, n_tx=n_tx, prelock_vbv=prelock)
@@ -53,18 +53,21 @@ def test_paired_script_paper_scenarios(sv):
 
 
 @pytest.mark.parametrize("mode", [G.MODE_HV, G.MODE_TBV])
-def test_paired_script_random_vs_oracle(mode):
+@pytest.mark.parametrize("policy", [0, 1, 2])
+def test_paired_script_random_vs_oracle(mode, policy):
+    """As the split-layout test: local, register-resident and shared-memory
+    logs, with batched reads (READ2, Q35)."""
     from test_oracle import encode_ops, random_script
-    rng = np.random.default_rng(77 + mode)
-    for trial in range(300):
+    rng = np.random.default_rng(77 + mode + 10 * policy)
+    for trial in range(200):
         bits = 4
         words = int(rng.integers(2, 17))
         n_tx = int(rng.integers(2, 5))
-        ops = encode_ops(random_script(rng, n_tx, words, 0))
+        ops = encode_ops(random_script(rng, n_tx, words, 0, batched=True, max_ops=4))
         heap0 = rng.integers(0, 50, words).astype(np.uint32)
         clock0 = int(rng.integers(0, 3))
         g, out_gpu, out_o, heap_o, locks_o, clk_o = _script_both(mode, bits, heap0, clock0, ops, n_tx,
-                                                                bool(trial % 2))
+                                                                bool(trial % 2), policy)
         assert out_gpu.tolist() == out_o.tolist(), trial
         assert (g.read_heap() == heap_o).all()
         assert (g.read_locks() == locks_o).all()

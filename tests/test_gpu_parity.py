@@ -104,11 +104,11 @@ def test_lock_log_parity(variant, cap):
 # ---------------------------------------------------------------------------
 # Algorithm 3 step-level parity: scripted interleavings on one device thread
 # ---------------------------------------------------------------------------
-def _script_both(mode, bits, heap0, clock0, ops, n_tx, prelock):
+def _script_both(mode, bits, heap0, clock0, ops, n_tx, prelock, policy=0):
     g = G.Gstm(heap0.size, bits)
     g.write_heap(heap0)
     g.set_clock(clock0)
-    out_gpu = g.script(mode, ops, n_tx=n_tx, prelock_vbv=prelock)
+    out_gpu = g.script(mode, ops, n_tx=n_tx, prelock_vbv=prelock, log_policy=policy)
     heap_o = heap0.copy()
     locks_o = np.zeros(1 << bits, dtype=np.uint32)
     out_o, clk_o = O.alg3_script(mode, bits, heap_o, locks_o, clock0, ops, n_tx=n_tx, prelock_vbv=prelock)
@@ -120,15 +120,16 @@ def _scenarios():
     return [(s, v) for s in load_scenarios() for v in s["variants"]]
 
 
+@pytest.mark.parametrize("policy", [0, 1, 2])
 @pytest.mark.parametrize("sv", _scenarios(), ids=lambda sv: f"{sv[0]['name']}-{sv[1]['mode']}-{int(sv[1]['prelock_vbv'])}")
-def test_script_paper_scenarios(sv):
+def test_script_paper_scenarios(sv, policy):
     from test_oracle import encode_ops
     s, v = sv
     mode = G.MODE_HV if v["mode"] == "HV" else G.MODE_TBV
     ops = encode_ops(s["ops"])
     heap0 = np.array(s["heap"], dtype=np.uint32)
     g, out_gpu, out_o, heap_o, locks_o, clk_o = _script_both(mode, s["bits"], heap0, s["clock0"], ops, 4,
-                                                            v["prelock_vbv"])
+                                                            v["prelock_vbv"], policy)
     assert out_gpu.tolist() == v["out"]                      # the paper-derived golden values
     assert out_gpu.tolist() == out_o.tolist()
     assert g.read_heap().tolist() == v["heap"]
@@ -139,17 +140,24 @@ def test_script_paper_scenarios(sv):
 
 @pytest.mark.parametrize("mode", [G.MODE_HV, G.MODE_TBV])
 @pytest.mark.parametrize("bits", [1, 2, 4])
-def test_script_random_vs_oracle(mode, bits):
+@pytest.mark.parametrize("policy", [0, 1, 2])
+def test_script_random_vs_oracle(mode, bits, policy):
+    """Random interleavings, op by op against Algorithm 3 (oracle/alg3.c),
+    including batched reads of two words (READ2: the kernels' read_batch with
+    the merged timestamp check of reading Q35), for every log storage the
+    kernels use: local memory (0), register-resident fully unrolled logs
+    (1: the bank kernel's code path, converged lock acquisition) and shared
+    memory [entry][lane] (2: P:117)."""
     from test_oracle import encode_ops, random_script
-    rng = np.random.default_rng(1000 + 10 * mode + bits)
+    rng = np.random.default_rng(1000 + 10 * mode + bits + 100 * policy)
     for trial in range(150):
         words = int(rng.integers(2, 9))
         n_tx = int(rng.integers(2, 5))
-        ops = encode_ops(random_script(rng, n_tx, words, 0))
+        ops = encode_ops(random_script(rng, n_tx, words, 0, batched=True, max_ops=4))
         heap0 = rng.integers(0, 50, words).astype(np.uint32)
         clock0 = int(rng.integers(0, 3))
         g, out_gpu, out_o, heap_o, locks_o, clk_o = _script_both(mode, bits, heap0, clock0, ops, n_tx,
-                                                                bool(trial % 2))
+                                                                bool(trial % 2), policy)
         assert out_gpu.tolist() == out_o.tolist(), trial
         assert (g.read_heap() == heap_o).all()
         assert (g.read_locks() == locks_o).all()

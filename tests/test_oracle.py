@@ -283,7 +283,7 @@ def test_replay_detects_lost_update():
 # --------------------------------------------------------------------------
 # Algorithm 3 model (alg3.c)
 # --------------------------------------------------------------------------
-_OPS = {"BEGIN": O.OP_BEGIN, "READ": O.OP_READ, "WRITE": O.OP_WRITE, "COMMIT": O.OP_COMMIT}
+_OPS = {"BEGIN": O.OP_BEGIN, "READ": O.OP_READ, "WRITE": O.OP_WRITE, "COMMIT": O.OP_COMMIT, "READ2": O.OP_READ2}
 
 
 def load_scenarios():
@@ -356,15 +356,18 @@ def test_lock_log_encounter_order():
         assert sorted(enc.tolist()) == O.lock_log(entries).tolist()
 
 
-def random_script(rng, n_tx, words, n_steps):
-    """Random interleaving of n_tx transactions; each tx: BEGIN, a few
-    READ/WRITE, COMMIT.  Returns the op list."""
+def random_script(rng, n_tx, words, n_steps, batched=False, max_ops=5):
+    """Random interleaving of n_tx transactions; each tx: BEGIN, 1..max_ops
+    READ/WRITE (and, batched=True, READ2: a batched read of two words, Q35),
+    COMMIT.  Returns the op list."""
     progs = []
     for s in range(n_tx):
         body = []
-        for _ in range(int(rng.integers(1, 6))):
+        for _ in range(int(rng.integers(1, max_ops + 1))):
             w = int(rng.integers(0, words))
-            if rng.random() < 0.55:
+            if batched and rng.random() < 0.3:
+                body.append(["READ2", s, w, int(rng.integers(0, words))])
+            elif rng.random() < 0.55:
                 body.append(["READ", s, w])
             else:
                 body.append(["WRITE", s, w, int(rng.integers(0, 1000))])
@@ -412,6 +415,18 @@ def check_opacity(init, ops, out, final_heap, clock0, final_clock):
                 st = state_at(o[2])
                 for rw, rv in tx["reads"]:
                     assert st[rw] == rv, (op, o)
+        elif kind == "READ2":
+            tx = txs[slot]
+            for w, v in ((op[2], o[0]), (op[3], o[1])):
+                if w in tx["writes"]:
+                    assert v == tx["writes"][w]
+                else:
+                    tx["reads"].append((w, v))
+            tx["snap"] = o[2]
+            if o[3] & 1:
+                st = state_at(o[2])
+                for rw, rv in tx["reads"]:
+                    assert st[rw] == rv, (op, o)
         elif kind == "WRITE":
             txs[slot]["writes"][op[2]] = op[3]
         else:
@@ -452,6 +467,47 @@ def test_alg3_random_scripts_are_opaque(mode, bits):
         assert not (locks & 1).any()          # no lock left held
         assert ((locks >> 1) <= clk).all()    # versions never exceed the clock
     assert commits > 100 and aborts > 10
+
+
+@pytest.mark.parametrize("mode", [O.MODE_HV, O.MODE_TBV])
+@pytest.mark.parametrize("bits", [1, 2, 4])
+def test_alg3_batched_reads_are_opaque(mode, bits):
+    """The batched TXRead of reading Q35 (OR_OP_READ2: value loads of both
+    words, then ONE timestamp check with the newest version) keeps opacity
+    under the independent checker, and a batch of two words that no
+    other transaction touches returns what two sequential TXReads return."""
+    rng = np.random.default_rng(500 + 100 * mode + bits)
+    commits = batched = 0
+    for trial in range(300):
+        words = int(rng.integers(2, 9))
+        n_tx = int(rng.integers(2, 5))
+        ops = random_script(rng, n_tx, words, 0, batched=True)
+        batched += sum(1 for op in ops if op[0] == "READ2")
+        init = rng.integers(0, 50, words).astype(np.uint32)
+        heap = init.copy()
+        locks = np.zeros(1 << bits, dtype=np.uint32)
+        out, clk = O.alg3_script(mode, bits, heap, locks, 0, encode_ops(ops), n_tx=n_tx,
+                                 prelock_vbv=bool(trial % 2))
+        commits += check_opacity(init.tolist(), ops, out, heap.tolist(), 0, clk)
+        assert not (locks & 1).any()
+    assert commits > 100 and batched > 200
+    # a lone transaction: READ2(a, b) == READ a; READ b (values, snapshot, opacity)
+    for trial in range(100):
+        words = 6
+        a, b = (int(x) for x in rng.integers(0, words, 2))
+        init = rng.integers(0, 50, words).astype(np.uint32)
+        w = int(rng.integers(0, words))
+        one = [["BEGIN", 0], ["WRITE", 0, w, 7], ["READ2", 0, a, b], ["COMMIT", 0]]
+        two = [["BEGIN", 0], ["WRITE", 0, w, 7], ["READ", 0, a], ["READ", 0, b], ["COMMIT", 0]]
+        outs = []
+        for script in (one, two):
+            heap = init.copy()
+            out, clk = O.alg3_script(mode, bits, heap, np.zeros(1 << bits, dtype=np.uint32), 3,
+                                     encode_ops(script), n_tx=1)
+            outs.append((out.tolist(), heap.tolist(), clk))
+        (o1, h1, c1), (o2, h2, c2) = outs
+        assert o1[2][:2] == [o2[2][0], o2[3][0]] and o1[2][2] == o2[3][2]
+        assert (o1[2][3] & 1) == o2[3][1] and o1[3] == o2[4] and h1 == h2 and c1 == c2
 
 
 def test_hv_aborts_no_more_than_tbv_on_false_conflicts():
