@@ -806,42 +806,6 @@ struct Tx {
         return ok;                                                   // l.52
     }
 
-    // Pipelined variant for a transaction's FIRST acquisition round (DESIGN.md
-    // §6.4): all atom.or are issued back to back (one memory round trip
-    // instead of n), then checked in ascending id.  On any conflict every
-    // lock this attempt set is restored and the next rounds fall back to the
-    // sequential sorted acquisition above, which carries the livelock-freedom
-    // argument.  Register-resident logs: every atom.or at once; local-memory
-    // logs (get_locks_and_tbv_pipelined_local): kChunk at a time.
-    __device__ __forceinline__ bool get_locks_and_tbv_pipelined(const Meta& m)
-    {
-        static_assert(kUnroll, "pipelined acquisition needs register-resident logs");
-        uint32_t vl[LCAP];
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl) vl[k] = prim::atom_or_relaxed(m.lock_ptr(l_ent[k] >> 2), 1u);   // l.45, all at once
-        prim::fence_acquire();
-        bool ok = true;
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl && (vl[k] & 1u)) ok = false;                  // l.46
-        if (!ok) {
-#pragma unroll
-            for (int k = 0; k < LCAP; ++k)                           // l.47: undo what we set
-                if (k < nl && !(vl[k] & 1u)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), vl[k]);
-            n_acq = 0;
-            return false;
-        }
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl) {
-                l_old[k] = vl[k];
-                if ((l_ent[k] & 1u) && (vl[k] >> 1) > snapshot) passTBV = false;   // l.49-51
-            }
-        n_acq = nl;
-        return true;
-    }
-
     // Register-resident logs: the pipelined first round and the sequential
     // sorted acquisition in ONE code path, so the lanes of a warp that make a
     // first attempt and those that retry after a lock abort share their memory

@@ -354,37 +354,6 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
         return ok;
     }
 
-    // first round of a fresh execution: all atom.or.b64 at once (§6.4)
-    __device__ __forceinline__ bool get_locks_and_tbv_pipelined(const Meta& m)
-    {
-        static_assert(kUnroll, "pipelined acquisition needs register-resident logs");
-        unsigned long long old[LCAP];
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl) old[k] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), 1ull << 32);
-        prim::fence_acquire();
-        bool ok = true;
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl && (hi(old[k]) & 1u)) ok = false;
-        if (!ok) {
-#pragma unroll
-            for (int k = 0; k < LCAP; ++k)
-                if (k < nl && !(hi(old[k]) & 1u)) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), old[k]);
-            n_acq = 0;
-            return false;
-        }
-#pragma unroll
-        for (int k = 0; k < LCAP; ++k)
-            if (k < nl) {
-                l_old[k] = hi(old[k]);
-                l_val[k] = lo(old[k]);
-                if ((l_ent[k] & 1u) && (hi(old[k]) >> 1) > snapshot) passTBV = false;
-            }
-        n_acq = nl;
-        return true;
-    }
-
     // Register-resident logs: the pipelined first round and the sequential
     // sorted acquisition in ONE code path (tx.cuh get_locks_and_tbv_converged):
     // round 0 issues entry 0 for every lane and every entry for a pipelined

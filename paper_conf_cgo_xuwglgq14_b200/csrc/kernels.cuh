@@ -86,7 +86,6 @@ cudaError_t launch_km_recenter(const Meta& m, uint32_t C, uint32_t D, uint32_t s
 int ubench(int kind, uint64_t table_bytes, uint64_t n_ops, uint32_t threads, double* ops_per_s, double* ms);
 int ubench_mix(const Meta& m, bool paired, uint64_t words, const uint32_t* prog, uint32_t prog_words, uint64_t n_tx,
                uint32_t threads, uint32_t block, cudaStream_t s, double* tx_per_s, double* ms);
-int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s);
 int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_words, uint32_t* locks, uint32_t lmask,
                         uint32_t* heap, uint32_t hmask, cudaStream_t s);
 

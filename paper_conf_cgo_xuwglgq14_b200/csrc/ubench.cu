@@ -88,18 +88,6 @@ __global__ void ubench_kernel(int kind, uint32_t* table, uint32_t mask, unsigned
     if (acc == 0xdeadbeefu) sink[0] = acc;
 }
 
-// Hot-spot probe for placing g_clock: every warp of a full-chip grid does
-// `n` warp-aggregated atom.add on one candidate word, like the commit path.
-__global__ void clock_probe_kernel(unsigned long long* word, uint32_t n, uint32_t* sink)
-{
-    // dependent chain: each increment waits for the previous one (latency
-    // under load, as on the commit path), not a pipelined throughput test
-    unsigned long long acc = 0;
-    if (prim::lane_id() == 0)
-        for (uint32_t k = 0; k < n; ++k) acc += prim::atom_add_acquire64(word, 8ull + (acc & 0x100000000000ull));
-    if (acc == 1ull) sink[0] = 1;
-}
-
 // Probe with the commit path's traffic mix: per warp round, 2 random
 // atom.or per lane on the lock table, 2 random loads per lane on the heap,
 // then one warp-aggregated increment of the candidate clock word.
@@ -318,36 +306,6 @@ int clock_calibrate_mix(unsigned long long* base, int n_candidates, int stride_w
         if (getenv("GSTM_CALIB_VERBOSE")) fprintf(stderr, "clock candidate %d (mix): %.4f ms\n", k, ms);
         if (ms < best_ms) { best_ms = ms; best = k; }
     }
-    cudaMemsetAsync(base, 0, static_cast<size_t>(n_candidates) * stride_words * 8, s);
-    cudaStreamSynchronize(s);
-out:
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
-    cudaFree(sink);
-    return best;
-}
-
-int clock_calibrate(unsigned long long* base, int n_candidates, int stride_words, cudaStream_t s)
-{
-    uint32_t* sink = nullptr;
-    cudaEvent_t e0 = nullptr, e1 = nullptr;
-    int best = -1;
-    float best_ms = 1e30f;
-    if (cudaMalloc(&sink, 64) != cudaSuccess) return -1;
-    cudaEventCreate(&e0);
-    cudaEventCreate(&e1);
-    for (int rep = 0; rep < 2; ++rep)
-        for (int k = 0; k < n_candidates; ++k) {
-            unsigned long long* w = base + static_cast<size_t>(k) * stride_words;
-            cudaEventRecord(e0, s);
-            clock_probe_kernel<<<148 * 4, 256, 0, s>>>(w, 32, sink);
-            cudaEventRecord(e1, s);
-            if (cudaEventSynchronize(e1) != cudaSuccess) { best = -1; goto out; }
-            float ms = 0.f;
-            cudaEventElapsedTime(&ms, e0, e1);
-            if (rep == 1 && getenv("GSTM_CALIB_VERBOSE")) fprintf(stderr, "clock candidate %d: %.4f ms\n", k, ms);
-            if (rep == 1 && ms < best_ms) { best_ms = ms; best = k; }
-        }
     cudaMemsetAsync(base, 0, static_cast<size_t>(n_candidates) * stride_words * 8, s);
     cudaStreamSynchronize(s);
 out:
