@@ -34,6 +34,8 @@ def main():
         "ld2_atom2_st2": [ph(R.LD_V, 2), ph(R.ATOM_L, 2), ph(R.ST_L, 2)],
         "bank_full": [ph(R.LD_V, 2), ph(R.ATOM_L, 2), ph(R.CLOCK), ph(R.ST_L, 2)],
         "clock_only": [ph(R.CLOCK)],
+        "atom2_clock_st2": [ph(R.ATOM_L, 2), ph(R.CLOCK), ph(R.ST_L, 2)],
+        "atom2_clock": [ph(R.ATOM_L, 2), ph(R.CLOCK)],
         "atom2": [ph(R.ATOM_L, 2)],
     }
     full = progs["bank_full"]
