@@ -154,6 +154,19 @@ typedef struct {
                              /*    the same sorted log and acquisition order, no     */
                              /*    sorting work for read-only transactions           */
                              /*    (DESIGN.md §6.15).  Default 0                     */
+    uint32_t serial_after;   /* contention manager (the adaptive    */
+                             /*    transaction scheduling P:313 and P:317 leave to   */
+                             /*    future work): a transaction whose executions      */
+                             /*    aborted >= serial_after times while g_clock       */
+                             /*    advanced by < serial_commits per abort (the whole */
+                             /*    GPU commits less than that per attempt) takes a   */
+                             /*    ticket; while tickets are outstanding no other    */
+                             /*    transaction starts, and the ticket holders run    */
+                             /*    one at a time in ticket order (FIFO), taking      */
+                             /*    their locks in one pipelined round.  Scheduling   */
+                             /*    only: every execution still validates and commits */
+                             /*    by Algorithm 3.  0 = off.  Default 0 (EB: 4)      */
+    uint32_t serial_commits; /*    see serial_after; 0 = 4.  Default 4                */
 } gstm_params_t;
 
 typedef struct {
@@ -191,6 +204,8 @@ typedef struct {
     uint64_t reads_ro;           /* read-set entries of read-only commits              */
     uint64_t writes_update;      /* write-set entries of update commits                */
     uint64_t locks_update;       /* lock-log entries (locks taken) of update commits   */
+    uint64_t serial_runs;        /* executions run as the serial-ticket owner          */
+                                 /*    (serial_after)                  */
 } gstm_stats_t;
 
 /* ---- lifecycle (STM_STARTUP / STM_SHUTDOWN) ------------------ */

@@ -37,7 +37,7 @@ static constexpr size_t kMetaBytes = 1024 * 1024; // metadata block (M_WORDS use
 // probability ~0.03%)
 static constexpr int kClockCandidates = 256;
 static constexpr int kClockStride = 288;           // ... 2304 B apart (crosses 256 B and 2 KiB address bits)
-static_assert(gstm::M_SEQ >= gstm::M_WORDS + kClockCandidates * kClockStride + 16 && gstm::M_SEQ * 8 + 128 <= kMetaBytes,
+static_assert(gstm::M_SEQ >= gstm::M_WORDS + kClockCandidates * kClockStride + 16 && gstm::M_SERIAL * 8 + 128 <= kMetaBytes,
               "STM-VBV sequence lock must sit on its own line after the clock candidates");
 
 struct gstm_handle {
@@ -203,6 +203,8 @@ static gstm_params_t default_params(int workload)
     p.lock_pipeline = 1;
     p.body_rounds = 1;
     p.pipeline_max_locks = 8;
+    p.serial_after = 0;
+    p.serial_commits = 4;
     if (workload == GSTM_WL_BANK) {
         p.n_words = 1ull << 20;
         // a transaction pipelines the first lock round of its first 4
@@ -280,6 +282,7 @@ static void fill_stats(gstm_stats_t* out, const unsigned long long* s, double ms
     out->reads_ro = s[S_RD_RO];
     out->writes_update = s[S_WR_UPD];
     out->locks_update = s[S_LK_UPD];
+    out->serial_runs = s[S_SERIAL];
     out->elapsed_ms = ms;
     const double done = static_cast<double>(out->commits + out->commits_ro);
     out->tx_per_s = ms > 0 ? done / (ms * 1e-3) : 0.0;
@@ -692,6 +695,8 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.body_rounds = P.body_rounds ? P.body_rounds : 1u;
     kp.pipeline_max_locks = P.pipeline_max_locks ? P.pipeline_max_locks : 8u;
     kp.lock_log_at_commit = P.lock_log_at_commit;
+    kp.serial_after = P.serial_after;
+    kp.serial_commits = P.serial_commits ? P.serial_commits : 4u;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));

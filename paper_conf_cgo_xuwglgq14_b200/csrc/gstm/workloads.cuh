@@ -139,6 +139,7 @@ struct RaWL {
 #define GSTM_RA_LOCAL_LOGS 1    // local-memory logs: 1.6x over the 128-register unrolled logs
 #endif
     static constexpr bool kLocalLogs = GSTM_RA_LOCAL_LOGS;
+    static constexpr bool kSerialGate = true;   // contention manager compiled in (stm_kernels.cuh §6.16)
 #ifndef GSTM_RA_MINB
 #define GSTM_RA_MINB 2
 #endif
@@ -195,6 +196,7 @@ struct RaIncWL {
     static constexpr int MAXR = 16;
     static constexpr int RCAP = MAXR, WCAP = MAXR, LCAP = MAXR, FGL_LCAP = MAXR;
     static constexpr bool kLocalLogs = GSTM_RA_LOCAL_LOGS;
+    static constexpr bool kSerialGate = true;   // contention manager compiled in (stm_kernels.cuh §6.16)
     static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = MAXR;
     __host__ static bool check(const WlParams& p)
@@ -288,6 +290,12 @@ struct HtWL {
     // code size is the HT kernel's limit (instruction fetch stalls, DESIGN.md
     // §6.9): rolled log loops; 64 registers for 4 blocks (32 warps) per SM
     static constexpr bool kCompact = true;
+#ifndef GSTM_HT_SMEM_HEAD
+#define GSTM_HT_SMEM_HEAD 0
+#endif
+    // logs: the first GSTM_HT_SMEM_HEAD entries in shared memory
+    static constexpr bool kSmemLogs = GSTM_HT_SMEM_HEAD > 0;
+    static constexpr int kSmemHead = GSTM_HT_SMEM_HEAD;
 #ifndef GSTM_HT_MINB
 #define GSTM_HT_MINB 4
 #endif
@@ -403,6 +411,7 @@ struct EbWLT {
     static constexpr int RCAP = MAXA / 2, WCAP = MAXA / 2, LCAP = MAXA, FGL_LCAP = MAXA;
     static constexpr bool kSmemLogs = SMEM_ || (GSTM_SMEM_LOGS && MAXA <= 32);   // A=64: 256 KB per block
     static constexpr bool kLocalLogs = true;   // never register-resident (A=32 unrolled: 2.4x slower)
+    static constexpr bool kSerialGate = true;   // contention manager compiled in (stm_kernels.cuh §6.16)
     static constexpr int kMinBlocks = 2;
     static constexpr int DESCR = 2 * MAXA;
     __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
@@ -521,6 +530,7 @@ struct KmWL {
 #define GSTM_KM_LOCAL_LOGS 1     // local-memory logs: 122 vs 254 registers, 2.5x faster
 #endif
     static constexpr bool kLocalLogs = GSTM_KM_LOCAL_LOGS;
+    static constexpr bool kSerialGate = true;   // contention manager compiled in (stm_kernels.cuh §6.16)
     static constexpr int kMinBlocks = GSTM_KM_LOCAL_LOGS ? 2 : 1;
     // 1024 records: 8 resident warps per SM is the measured optimum
     // (21.5 vs 17.9 M tx/s at 16)

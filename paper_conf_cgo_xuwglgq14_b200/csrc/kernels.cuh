@@ -18,6 +18,7 @@ enum {
     // op-mix roof): reads appended to the read-set by update /
     // read-only commits, write-set entries and lock-log entries of update commits
     S_RD_UPD, S_RD_RO, S_WR_UPD, S_LK_UPD,
+    S_SERIAL,              // executions run as the serial-ticket owner (contention manager)
     S_NSTATS
 };
 
@@ -41,6 +42,7 @@ enum {
     M_WORDS = 160,
     // after the 256 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
     M_SEQ = M_WORDS + 256 * 288 + 16,  // STM-VBV global sequence lock, own line
+    M_SERIAL = M_SEQ + 16,             // contention manager's ticket word {serving:32 | next:32}, own line
 };
 
 constexpr int kPhaseWords = 16;    // M_PHASE .. M_PHASE + 15
@@ -67,6 +69,8 @@ struct KParams {
     uint32_t body_rounds;          // >= 1: bodies per warp iteration for lanes that commit read-only
     uint32_t pipeline_max_locks;   // local-memory logs: pipeline the first round only up to this many locks
     uint32_t lock_log_at_commit;   // read locks enter the sorted lock log at TXCommit (Tx::insert_read_lock)
+    uint32_t serial_after;         // contention manager: aborts before a transaction may take a serial ticket (0 = off)
+    uint32_t serial_commits;       // ... only while the clock advanced by < serial_commits per abort
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);

@@ -76,12 +76,29 @@ struct SmemLogs { static constexpr bool value = false; };
 template <class WL>
 struct SmemLogs<WL, std::void_t<decltype(WL::kSmemLogs)>> { static constexpr bool value = WL::kSmemLogs; };
 
+// WL::kSmemHead (optional, with kSmemLogs): only the first kSmemHead entries
+// of each log in shared memory, the rest in local memory (LogArr hybrid,
+// DESIGN.md §6.17); 0 = every entry in shared memory
+template <class WL, class = void>
+struct SmemHead { static constexpr int value = 0; };
+template <class WL>
+struct SmemHead<WL, std::void_t<decltype(WL::kSmemHead)>> { static constexpr int value = WL::kSmemHead; };
+
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
 struct RunWriteback { static constexpr bool value = false; };
 template <class WL>
 struct RunWriteback<WL, std::void_t<decltype(WL::kRunWriteback)>> { static constexpr bool value = WL::kRunWriteback; };
+
+// WL::kSerialGate (optional): the contention manager (p.serial_after,
+// DESIGN.md §6.16) is compiled into this workload's STM kernels.  Bank and
+// HT (abort ratios 0.16 and 0.003) leave it out: it costs them 8-12
+// registers
+template <class WL, class = void>
+struct SerialGate { static constexpr bool value = false; };
+template <class WL>
+struct SerialGate<WL, std::void_t<decltype(WL::kSerialGate)>> { static constexpr bool value = WL::kSerialGate; };
 
 // WL::kWarpsPerSM (optional): resident STM warps per SM the persistent grid
 // stops at (0 = as many as fit).  More concurrent transactions than that
@@ -188,6 +205,80 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
     return __shfl_sync(FULL, late, 0);
 }
 
+// ---------------------------------------------------------------------------
+// Contention manager (p.serial_after != 0): the adaptive
+// transaction scheduling the paper leaves to future work.
+// One 64-bit word in the metadata block, M_SERIAL = {serving:32 | next:32},
+// is a ticket queue.  A transaction that keeps aborting while the whole GPU
+// commits little (g_clock advanced by < serial_commits per abort of its
+// own) takes a ticket; while any ticket is outstanding (next != serving) no
+// other transaction STARTS an execution -- one that has aborted before joins
+// the queue instead, so a serial phase, once the contention test opened it,
+// serves every transaction that was failing -- and the holders run one at a time
+// in ticket order, the owner (ticket == serving) taking its locks in one
+// pipelined round.  The executions already in flight drain (they commit or
+// abort within their bounded lock rounds), so the owner soon runs alone;
+// when its transaction is done it serves the next ticket.  This only decides
+// WHEN executions start: each one still runs Algorithm 3 in full (reads,
+// validation, sorted locks, stamp), so the results and the replay checks are
+// those of any other schedule.
+// ---------------------------------------------------------------------------
+struct SerialState {
+    uint32_t ticket = 0, serving = 0;
+    uint32_t n_ab = 0;        // aborted executions of the current transaction
+    uint32_t s_first = 0;     // snapshot of its first execution
+    bool has_ticket = false;
+    bool pending = false;     // the last poll saw tickets outstanding (warp-uniform)
+    __device__ __forceinline__ bool owner() const { return has_ticket && ticket == serving; }
+};
+
+// Only the FIRST lock round of an execution is pipelined, as for every
+// other transaction: a round after a failed one is the sequential sorted
+// acquisition, so the owner and an in-flight lane cannot defeat each other's
+// rounds forever (Q15, Q37).
+//
+// Called once per warp iteration by every lane; `fresh`: this lane would
+// start an execution of its current transaction (stage 0).  Returns whether
+// it may.  The ticket word is read when this warp takes or holds a ticket,
+// after a poll that saw tickets outstanding, and every 8th iteration
+// otherwise (a stale "none outstanding" only lets an execution start that
+// the owner then waits to drain).
+__device__ __forceinline__ bool serial_gate(const KParams& p, SerialState& ss, bool fresh, uint32_t snap,
+                                            uint32_t iter)
+{
+    unsigned long long* sw = p.meta + M_SERIAL;
+    const bool want = fresh && !ss.has_ticket &&
+                      ((ss.n_ab >= p.serial_after && snap - ss.s_first < p.serial_commits * ss.n_ab) ||
+                       (ss.pending && ss.n_ab >= 1u));
+    const unsigned wm = __ballot_sync(FULL, want);
+    const bool poll = wm || __any_sync(FULL, ss.has_ticket) || ss.pending || (iter & 7u) == 0u;
+    if (poll) {
+        unsigned long long w = 0;
+        if (prim::lane_id() == 0)
+            w = wm ? atomicAdd(sw, static_cast<unsigned long long>(__popc(wm))) : prim::ld_relaxed64(sw);
+        w = __shfl_sync(FULL, w, 0);
+        const uint32_t next = static_cast<uint32_t>(w) + __popc(wm);
+        ss.serving = static_cast<uint32_t>(w >> 32);
+        if (want) {
+            ss.ticket = static_cast<uint32_t>(w) + __popc(wm & prim::lanemask_lt());
+            ss.has_ticket = true;
+        }
+        ss.pending = next != ss.serving;
+    }
+    return ss.has_ticket ? ss.owner() : !ss.pending;
+}
+
+// the owner's transaction is done (committed or dropped): serve the next ticket
+__device__ __forceinline__ void serial_release(const KParams& p, SerialState& ss)
+{
+    if (ss.owner()) {
+        prim::fence_release();   // not needed for correctness (scheduling only); orders the owner's commit first
+        atomicAdd(p.meta + M_SERIAL, 1ull << 32);
+    }
+    ss.has_ticket = false;
+    ss.n_ab = 0;
+}
+
 // Per-category time breakdown (the Figure 5 study of P:329-333):
 // the "phase" build flavour (-DGSTM_PHASE_TIMING=1) times every lane's own
 // path in the paper's categories (tx.cuh PH_*, Tx::ph); at exit the per-lane
@@ -226,9 +317,9 @@ template <class WL, bool PAIR, int POL>
 using StmTx = std::conditional_t<
     PAIR,
     TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value,
-           HashedLog<WL>::value, SmemLogs<WL>::value>,
+           HashedLog<WL>::value, SmemLogs<WL>::value, SmemHead<WL>::value>,
     Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value, HashedLog<WL>::value,
-       SmemLogs<WL>::value>>;
+       SmemLogs<WL>::value, SmemHead<WL>::value>>;
 
 // dynamic shared memory of the STM kernel: the shared-memory logs, if any
 template <class WL, bool PAIR, int POL>
@@ -278,6 +369,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     int stage = 0;
     bool timed_out = false, have_snap = false;
     uint32_t lock_aborts = 0;   // lock aborts of the current transaction
+    SerialState ss;             // contention manager (p.serial_after)
+    const bool serial_on = SerialGate<WL>::value && p.serial_after != 0;
     tx.ph_init();
 
     while (__any_sync(FULL, t < p.T)) {
@@ -288,7 +381,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         // this warp's own last commit (p.snapshot_reuse)
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
         have_snap = false;
-        bool done = false, aborted = false;
+        bool done = false, aborted = false, fin = false, ran = false;
+        const bool may_start = serial_on ? serial_gate(p, ss, act && stage == 0 && i < p.K, snap, iter) : true;
         // Body rounds (p.body_rounds): a lane whose
         // transaction committed read-only (A3.l68: no locks, no stamp) starts
         // its next transaction in the same warp iteration, up to body_rounds
@@ -297,7 +391,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         // Every round uses the iteration's snapshot (a valid, older one: more
         // validation at worst).  A lane that aborted, or holds an update to
         // commit, sits out the later rounds.
-        bool cont = act && stage == 0;
+        bool cont = act && stage == 0 && may_start;
         // a lane's next transaction starts no earlier than where its last one
         // was linearised (PostValidation may have raised that snapshot above
         // the iteration's): per-thread real-time order
@@ -312,6 +406,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 const uint64_t tx_id = static_cast<uint64_t>(i) * p.T + t;
                 bool next = false;
                 cnt.inc(S_ATTEMPTS);
+                ran = true;
+                if (serial_on) {
+                    if (ss.n_ab == 0) ss.s_first = lane_snap;
+                    if (ss.has_ticket) cnt.inc(S_SERIAL);
+                }
                 result = 0;
                 tx.ph(PH_INIT);
                 const uint64_t x = gen::tx_key(p.seed, t, i);
@@ -333,7 +432,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     cnt.inc(S_COMMITS_RO);
                     cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
                     next = true;
-                    cont = true;
+                    cont = !(serial_on && ss.has_ticket);   // the serial owner hands over after one transaction
                     lane_snap = tx.snapshot;
                 } else {
                     tx.ph(PH_OTHER);                                  // waits for the warp's commit round
@@ -344,6 +443,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
                 }
                 if (next) {                                           // the next transaction of thread t
+                    fin = true;
                     ++i;
                     backoff = 0;
                     lock_aborts = 0;
@@ -367,8 +467,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
-            const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline;
-            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks);
+            // (the serial owner pipelines the first round of every execution,
+            // whatever its size: once the executions in flight drained it is
+            // the only one running, §6.16)
+            const bool owner = serial_on && ss.owner();
+            const bool want_pipe = tries == 0 && (lock_aborts < p.lock_pipeline || owner);
+            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe,
+                                            owner ? 0x7fffffffu : p.pipeline_max_locks);
             if (tx.pipelined_round) cnt.inc(S_PIPELINED);
             if (r == C_OK) {
                 got = true;
@@ -484,6 +589,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             seq_fails = seq_failed ? seq_fails + 1u : 0u;
         }
         if (done) {
+            fin = true;
             stage = 0;
             ++i;
             backoff = 0;
@@ -494,6 +600,16 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // under independent thread scheduling)
             backoff = backoff ? min(backoff * 2u, 64u * p.backoff_ns) : p.backoff_ns;
             __nanosleep(backoff);
+        }
+        if (serial_on) {
+            if (fin) serial_release(p, ss);
+            if (aborted) ++ss.n_ab;   // (an execution of the lane's NEXT transaction, if fin)
+            // a warp whose lanes were all held back sleeps before polling
+            // again (the warp holding the next ticket polls at once)
+            if (!__any_sync(FULL, ran || stage == 1)) {
+                const bool soon = ss.has_ticket && ss.ticket - ss.serving <= 1u;
+                if (!__any_sync(FULL, soon)) __nanosleep(1000);
+            }
         }
         // refill: lanes whose STM thread ran all K transactions take the next
         // one -- their next static thread, else one from the counter

@@ -59,6 +59,7 @@ class gstm_params_t(C.Structure):
         ("shard_bits", C.c_uint32), ("shard", C.c_uint32), ("km_stride", C.c_uint32),
         ("km_assign", C.c_uint32), ("l2_persist_locks", C.c_uint32), ("ra_partition", C.c_uint32),
         ("body_rounds", C.c_uint32), ("pipeline_max_locks", C.c_uint32), ("lock_log_at_commit", C.c_uint32),
+        ("serial_after", C.c_uint32), ("serial_commits", C.c_uint32),
     ]
 
 
@@ -73,7 +74,7 @@ class gstm_stats_t(C.Structure):
         ("abort_ratio", C.c_double), ("status", C.c_int32), ("mode_used", C.c_int32),
         ("clock_slot", C.c_int32), ("pipelined_rounds", C.c_uint64),
         ("reads_update", C.c_uint64), ("reads_ro", C.c_uint64), ("writes_update", C.c_uint64),
-        ("locks_update", C.c_uint64),
+        ("locks_update", C.c_uint64), ("serial_runs", C.c_uint64),
     ]
 
     def as_dict(self) -> dict:

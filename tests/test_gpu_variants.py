@@ -207,6 +207,8 @@ def test_compute_sanitizer_clean(tool):
     r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "9", "--print-limit", "20",
                         sys.executable, os.path.join(root, "tools", "sanitize_tiny.py")],
                        capture_output=True, text=True, timeout=1500)
+    if r.returncode != 0 and "closed on this pool" in r.stderr:
+        pytest.skip("compute-sanitizer is disabled on this GPU pool (" + r.stderr.strip()[:80] + ")")
     assert r.returncode == 0, (r.stdout[-3000:], r.stderr[-3000:])
     assert "launches replayed" in r.stdout
     out = r.stdout + r.stderr

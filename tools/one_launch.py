@@ -45,7 +45,8 @@ def main():
         n = max(1, st.commits + st.commits_ro)
         print(f"{a.config} {a.mode} launch {k}: {st.tx_per_s / 1e6:.1f} M tx/s, abort {st.abort_ratio:.3f}, "
               f"{st.elapsed_ms:.3f} ms; per tx: postval {st.postvalidations / n:.4f} vbv {st.vbv_runs / n:.4f} "
-              f"spins {st.spins / n:.4f} lock_retries {st.lock_retries / n:.4f} ro {st.commits_ro / n:.3f}", flush=True)
+              f"spins {st.spins / n:.4f} lock_retries {st.lock_retries / n:.4f} ro {st.commits_ro / n:.3f} "
+              f"serial {st.serial_runs}", flush=True)
     g.close()
 
 
