@@ -161,11 +161,13 @@ typedef struct {
                              /*    advanced by < serial_commits per abort (the whole */
                              /*    GPU commits less than that per attempt) takes a   */
                              /*    ticket; while tickets are outstanding no other    */
-                             /*    transaction starts, and the ticket holders run    */
-                             /*    one at a time in ticket order (FIFO), taking      */
-                             /*    their locks in one pipelined round.  Scheduling   */
-                             /*    only: every execution still validates and commits */
-                             /*    by Algorithm 3.  0 = off.  Default 0 (EB: 4)      */
+                             /*    transaction starts (one that aborted before joins */
+                             /*    the queue), and the holders run one at a time in  */
+                             /*    ticket order (FIFO), each IRREVOCABLY: in place,  */
+                             /*    under encounter-time version locks, stamped while */
+                             /*    it holds them all -- serialised like an A3 commit */
+                             /*    (gstm/tx_irr.cuh).  Kernels of EB, RA and KM only  */
+                             /*    (bank and HT ignore it).  0 = off.  Default 0     */
     uint32_t serial_commits; /*    see serial_after; 0 = 4.  Default 4                */
 } gstm_params_t;
 

@@ -21,7 +21,7 @@ SO = os.path.join(LIBDIR, "libgstm.so")
 SOURCES = ["api.cu", "kernels.cu", "script.cu", "ubench.cu",
            "wl_ra.cu", "wl_bank.cu", "wl_ht.cu", "wl_eb.cu", "wl_eb16.cu", "wl_eb32.cu", "wl_km.cu", "km.cu"]     # one TU per workload: parallel build
 HEADERS = ["kernels.cuh", "stm_kernels.cuh", "gstm/prim.cuh", "gstm/gen.cuh", "gstm/tx.cuh", "gstm/tx_pair.cuh",
-           "gstm/tx_vbv.cuh", "gstm/workloads.cuh"]
+           "gstm/tx_vbv.cuh", "gstm/tx_irr.cuh", "gstm/workloads.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr"]
 

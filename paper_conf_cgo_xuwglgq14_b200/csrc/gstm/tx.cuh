@@ -118,13 +118,7 @@ __device__ __forceinline__ unsigned long long bloom_bit(uint32_t w)
 // a warp in 32 consecutive words, [entry][lane], so the lanes' accesses to
 // their k-th entries hit 32 different banks (SMEM = true; bind() sets the
 // lane's column).
-//
-// HEAD > 0 (with SMEM): a hybrid -- entries [0, HEAD) in the shared-memory
-// column, the rest in a per-thread local array.  For logs whose capacity is
-// set by a rare worst case (HT: a 24-node chain, 49 reads) while a typical
-// transaction uses a few entries: the shared-memory head takes the log
-// traffic that local memory writes through to L2.
-template <int CAP, bool SMEM, int HEAD = 0>
+template <int CAP, bool SMEM>
 struct LogArr {
     uint32_t a[CAP];
     __device__ __forceinline__ uint32_t& operator[](int k) { return a[k]; }
@@ -132,30 +126,19 @@ struct LogArr {
     __device__ __forceinline__ void bind(uint32_t*) {}
 };
 template <int CAP>
-struct LogArr<CAP, true, 0> {
+struct LogArr<CAP, true> {
     uint32_t* p;                          // shared memory: this lane's column
     __device__ __forceinline__ uint32_t& operator[](int k) { return p[k * 32]; }
     __device__ __forceinline__ const uint32_t& operator[](int k) const { return p[k * 32]; }
     __device__ __forceinline__ void bind(uint32_t* col) { p = col; }
 };
-template <int CAP, int HEAD>
-struct LogArr<CAP, true, HEAD> {
-    static constexpr int H = HEAD < CAP ? HEAD : CAP;
-    uint32_t* p;                          // shared memory: this lane's column, entries [0, H)
-    uint32_t a[CAP > H ? CAP - H : 1];    // local memory: entries [H, CAP)
-    __device__ __forceinline__ uint32_t& operator[](int k) { return k < H ? p[k * 32] : a[k - H]; }
-    __device__ __forceinline__ const uint32_t& operator[](int k) const { return k < H ? p[k * 32] : a[k - H]; }
-    __device__ __forceinline__ void bind(uint32_t* col) { p = col; }
-};
-// shared-memory words per lane of a log of CAP entries
-__host__ __device__ constexpr int smem_entries(int cap, int head) { return head > 0 && head < cap ? head : cap; }
 
 // HLOG = true (local-memory logs, sorted): the lock log is the order-preserving
 // hash table of P:115 instead of one sorted array.
 // SMEM = true: the read-, write- and lock-logs live in shared memory, per warp
 // [entry][lane]; the kernel binds them (bind_smem).
 template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false, bool HLOG = false,
-          bool SMEM = false, int SHEAD = 0>
+          bool SMEM = false>
 struct Tx {
     // register-resident (unrolled) logs for small capacities unless the
     // workload asks for local memory (LOCAL: fewer registers, more warps) or
@@ -174,25 +157,22 @@ struct Tx {
     static constexpr int kTs = kHlog ? kHs + LCAP : LCAP;
     static constexpr int kBw = kHlog ? (kTs + 31) / 32 : 1;
 
-    LogArr<RCAP, SMEM, SHEAD> r_addr, r_val;     // read-set  <addr,val>
-    LogArr<WCAP, SMEM, SHEAD> w_addr, w_val;     // write-set <addr,val> (redo log)
-    LogArr<kTs, SMEM, SHEAD> l_ent;              // sorted lock log (hashed: the table)
-    LogArr<LCAP, SMEM, SHEAD> l_old;             // old lock words
+    LogArr<RCAP, SMEM> r_addr, r_val;     // read-set  <addr,val>
+    LogArr<WCAP, SMEM> w_addr, w_val;     // write-set <addr,val> (redo log)
+    LogArr<kTs, SMEM> l_ent;              // sorted lock log (hashed: the table)
+    LogArr<LCAP, SMEM> l_old;             // old lock words
     // shared-memory logs: words per thread, and the binding of every log to
-    // this lane's column of its warp's [word][lane] region (SHEAD > 0: the
-    // first SHEAD entries of each log)
-    static constexpr int kSr = smem_entries(RCAP, SHEAD), kSw = smem_entries(WCAP, SHEAD);
-    static constexpr int kSt = smem_entries(kTs, SHEAD), kSl = smem_entries(LCAP, SHEAD);
-    static constexpr int kSmemWords = 2 * kSr + 2 * kSw + kSt + kSl;
+    // this lane's column of its warp's [word][lane] region
+    static constexpr int kSmemWords = 2 * RCAP + 2 * WCAP + kTs + LCAP;
     __device__ __forceinline__ void bind_smem(uint32_t* warp_region, int lane)
     {
         uint32_t* c = warp_region + lane;
         r_addr.bind(c);
-        r_val.bind(c + 32 * kSr);
-        w_addr.bind(c + 32 * (2 * kSr));
-        w_val.bind(c + 32 * (2 * kSr + kSw));
-        l_ent.bind(c + 32 * (2 * kSr + 2 * kSw));
-        l_old.bind(c + 32 * (2 * kSr + 2 * kSw + kSt));
+        r_val.bind(c + 32 * RCAP);
+        w_addr.bind(c + 32 * (2 * RCAP));
+        w_val.bind(c + 32 * (2 * RCAP + WCAP));
+        l_ent.bind(c + 32 * (2 * RCAP + 2 * WCAP));
+        l_old.bind(c + 32 * (2 * RCAP + 2 * WCAP + kTs));
     }
     uint32_t occ[kBw];                    // hashed log: occupied slots
     uint32_t id_shift = 12;               // hashed log: 32 - lock-table bits (home = id's top bits)

@@ -22,9 +22,9 @@
 namespace gstm {
 
 template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false,
-          bool HLOG = false, bool SMEM = false, int SHEAD = 0>
-struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM, SHEAD> {
-    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM, SHEAD>;
+          bool HLOG = false, bool SMEM = false>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM>;
     using B::kUnroll;
     using B::r_addr;
     using B::r_val;

@@ -61,6 +61,9 @@ struct StmCtx {
         tx.read_many(m, a, v, skip, n, mode);
     }
     __device__ __forceinline__ void write(uint32_t a, uint32_t v) { tx.write(m, a, v); }
+    // the body's write addresses, in write order (a hint for the irrevocable
+    // owner, gstm/tx_irr.cuh; nothing to do here)
+    __device__ __forceinline__ void will_write(const uint32_t*, int, int) {}
     __device__ __forceinline__ bool ok() const { return tx.opaque; }
     // the body found its own view inconsistent (e.g. a chain pointer out of
     // range): only possible for a transaction that is about to abort
@@ -100,6 +103,7 @@ struct DirectCtx {
             if (!skip[k]) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
     }
     __device__ __forceinline__ void write(uint32_t a, uint32_t v) { prim::st_relaxed(m.val_ptr(a), v); ++nw; }
+    __device__ __forceinline__ void will_write(const uint32_t*, int, int) {}
     __device__ __forceinline__ bool ok() const { return !bad; }
     __device__ __forceinline__ void invalid() { bad = true; }
     __device__ __forceinline__ void overflow() { bad = true; }
@@ -290,12 +294,6 @@ struct HtWL {
     // code size is the HT kernel's limit (instruction fetch stalls, DESIGN.md
     // §6.9): rolled log loops; 64 registers for 4 blocks (32 warps) per SM
     static constexpr bool kCompact = true;
-#ifndef GSTM_HT_SMEM_HEAD
-#define GSTM_HT_SMEM_HEAD 0
-#endif
-    // logs: the first GSTM_HT_SMEM_HEAD entries in shared memory
-    static constexpr bool kSmemLogs = GSTM_HT_SMEM_HEAD > 0;
-    static constexpr int kSmemHead = GSTM_HT_SMEM_HEAD;
 #ifndef GSTM_HT_MINB
 #define GSTM_HT_MINB 4
 #endif
@@ -476,13 +474,20 @@ struct EbWLT {
         bool raw[MAXA / 2];
         for (uint32_t j = 0; j < A; ++j) addr[j] = static_cast<uint32_t>(gen::bounded(gen::draw(x, j), p.n_words));
         const uint32_t R = (A + 1) / 2;
+        // read r is read-after-write if an earlier write has its address; a
+        // 64-bit filter of the written addresses skips the scan for most reads
+        unsigned long long wf = 0ull;
         for (uint32_t r = 0; r < R; ++r) {
             ra[r] = addr[2 * r];
             bool hit = false;
-            for (uint32_t k = 1; k < 2 * r; k += 2) hit |= (addr[k] == ra[r]);
+            if (wf & (1ull << (ra[r] & 63u)))
+                for (uint32_t k = 1; k < 2 * r; k += 2) hit |= (addr[k] == ra[r]);
             raw[r] = hit;
+            if (2 * r + 1 < A) wf |= 1ull << (addr[2 * r + 1] & 63u);
         }
         c.read_many(ra, rv, raw, static_cast<int>(R));
+        if (!c.ok()) return;
+        c.will_write(addr + 1, static_cast<int>(A / 2), 2);     // addr[1], addr[3], ...: the write order
         if (!c.ok()) return;
         uint32_t acc = 0;
         for (uint32_t j = 0; j < A; ++j) {

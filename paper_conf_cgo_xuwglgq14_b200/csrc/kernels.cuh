@@ -5,6 +5,7 @@
 #include "gstm/tx.cuh"
 #include "gstm/tx_pair.cuh"
 #include "gstm/tx_vbv.cuh"
+#include "gstm/tx_irr.cuh"
 #include "gstm/workloads.cuh"
 
 namespace gstm {

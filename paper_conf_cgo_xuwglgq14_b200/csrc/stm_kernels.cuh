@@ -76,14 +76,6 @@ struct SmemLogs { static constexpr bool value = false; };
 template <class WL>
 struct SmemLogs<WL, std::void_t<decltype(WL::kSmemLogs)>> { static constexpr bool value = WL::kSmemLogs; };
 
-// WL::kSmemHead (optional, with kSmemLogs): only the first kSmemHead entries
-// of each log in shared memory, the rest in local memory (LogArr hybrid,
-// DESIGN.md §6.17); 0 = every entry in shared memory
-template <class WL, class = void>
-struct SmemHead { static constexpr int value = 0; };
-template <class WL>
-struct SmemHead<WL, std::void_t<decltype(WL::kSmemHead)>> { static constexpr int value = WL::kSmemHead; };
-
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
@@ -215,13 +207,13 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
 // other transaction STARTS an execution -- one that has aborted before joins
 // the queue instead, so a serial phase, once the contention test opened it,
 // serves every transaction that was failing -- and the holders run one at a time
-// in ticket order, the owner (ticket == serving) taking its locks in one
-// pipelined round.  The executions already in flight drain (they commit or
-// abort within their bounded lock rounds), so the owner soon runs alone;
-// when its transaction is done it serves the next ticket.  This only decides
-// WHEN executions start: each one still runs Algorithm 3 in full (reads,
-// validation, sorted locks, stamp), so the results and the replay checks are
-// those of any other schedule.
+// in ticket order: the owner (ticket == serving) runs its transaction
+// irrevocably -- in place, under encounter-time locks, stamped while it holds
+// them all (gstm/tx_irr.cuh) -- and then serves the next ticket.  The
+// executions already in flight finish under Algorithm 3 beside it (they see
+// the owner's words locked, as during any commit).  Every other execution
+// runs Algorithm 3 in full; the owner is serialised at its stamp like any
+// commit, so the replay checks hold for every schedule.
 // ---------------------------------------------------------------------------
 struct SerialState {
     uint32_t ticket = 0, serving = 0;
@@ -232,11 +224,6 @@ struct SerialState {
     __device__ __forceinline__ bool owner() const { return has_ticket && ticket == serving; }
 };
 
-// Only the FIRST lock round of an execution is pipelined, as for every
-// other transaction: a round after a failed one is the sequential sorted
-// acquisition, so the owner and an in-flight lane cannot defeat each other's
-// rounds forever (Q15, Q37).
-//
 // Called once per warp iteration by every lane; `fresh`: this lane would
 // start an execution of its current transaction (stage 0).  Returns whether
 // it may.  The ticket word is read when this warp takes or holds a ticket,
@@ -317,9 +304,9 @@ template <class WL, bool PAIR, int POL>
 using StmTx = std::conditional_t<
     PAIR,
     TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value,
-           HashedLog<WL>::value, SmemLogs<WL>::value, SmemHead<WL>::value>,
+           HashedLog<WL>::value, SmemLogs<WL>::value>,
     Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value, HashedLog<WL>::value,
-       SmemLogs<WL>::value, SmemHead<WL>::value>>;
+       SmemLogs<WL>::value>>;
 
 // dynamic shared memory of the STM kernel: the shared-memory logs, if any
 template <class WL, bool PAIR, int POL>
@@ -371,6 +358,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     uint32_t lock_aborts = 0;   // lock aborts of the current transaction
     SerialState ss;             // contention manager (p.serial_after)
     const bool serial_on = SerialGate<WL>::value && p.serial_after != 0;
+    // the serial owner's lock log: one slice per warp (one owner per warp at most)
+    constexpr int kIrrWords = SerialGate<WL>::value ? 2 * IrrCtx<TX>::kCap : 1;
+    __shared__ uint32_t irr_sh[(kMaxBlock / 32) * kIrrWords];
+    uint32_t* const irr_log = irr_sh + (threadIdx.x >> 5) * kIrrWords;
     tx.ph_init();
 
     while (__any_sync(FULL, t < p.T)) {
@@ -414,33 +405,57 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 result = 0;
                 tx.ph(PH_INIT);
                 const uint64_t x = gen::tx_key(p.seed, t, i);
-                tx.begin(lane_snap);                                  // TXBegin l.2-3
-                tx.sync_mask = body_mask;
-                StmCtx<TX> ctx{tx, m, MODE};
-                tx.ph(PH_NATIVE);
-                WL::body(ctx, p.w, x, t, i, result);                 // TXRead / TXWrite
-                if (!tx.opaque) {
-                    tx.ph_end(false);
-                    if (tx.overflow) { cnt.inc(S_ERRORS); next = true; }  // sticky ELOGOVF, give up this tx
-                    else { cnt.inc(S_AB_OPACITY); aborted = true; }  // Figure 1 / Q11
-                } else if (tx.read_only()) {                          // l.68: linearized at snapshot
+                if (serial_on && ss.owner()) {
+                    // the serial-ticket owner runs irrevocably: in place,
+                    // under encounter-time locks, stamped while it holds
+                    // them all (gstm/tx_irr.cuh)
+                    IrrCtx<TX> ic{irr_log, irr_log + IrrCtx<TX>::kCap, m, deadline};
+                    tx.ph(PH_NATIVE);
+                    WL::body(ic, p.w, x, t, i, result);
+                    tx.ph(PH_COMMIT);
+                    const uint32_t s = ic.commit(m.clock);
+                    tx.n_spin += ic.n_spin;
                     tx.ph_end(true);
+                    if (ic.bad) {
+                        cnt.inc(S_ERRORS);
+                        if (globaltimer() > deadline) timed_out = true;
+                    }
                     if (p.tx_stamp) {
-                        p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
+                        p.tx_stamp[tx_id] = (s & 0x80000000u) ? 0x80000000u | ((s & 0x7fffffffu) - clock_begin)
+                                                              : s - clock_begin;
                         p.tx_result[tx_id] = result;
                     }
-                    cnt.inc(S_COMMITS_RO);
-                    cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
+                    cnt.inc((s & 0x80000000u) ? S_COMMITS_RO : S_COMMITS);
                     next = true;
-                    cont = !(serial_on && ss.has_ticket);   // the serial owner hands over after one transaction
-                    lane_snap = tx.snapshot;
                 } else {
-                    tx.ph(PH_OTHER);                                  // waits for the warp's commit round
-                    stage = 1;
-                    // STM-HV-Backoff: an execution that follows a lock abort goes
-                    // straight to the sequential step -- its parallel attempt
-                    // already failed
-                    tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
+                    tx.begin(lane_snap);                                  // TXBegin l.2-3
+                    tx.sync_mask = body_mask;
+                    StmCtx<TX> ctx{tx, m, MODE};
+                    tx.ph(PH_NATIVE);
+                    WL::body(ctx, p.w, x, t, i, result);                 // TXRead / TXWrite
+                    if (!tx.opaque) {
+                        tx.ph_end(false);
+                        if (tx.overflow) { cnt.inc(S_ERRORS); next = true; }  // sticky ELOGOVF, give up this tx
+                        else { cnt.inc(S_AB_OPACITY); aborted = true; }  // Figure 1 / Q11
+                    } else if (tx.read_only()) {                          // l.68: linearized at snapshot
+                        tx.ph_end(true);
+                        if (p.tx_stamp) {
+                            p.tx_stamp[tx_id] = 0x80000000u | (tx.snapshot - clock_begin);
+                            p.tx_result[tx_id] = result;
+                        }
+                        cnt.inc(S_COMMITS_RO);
+                        cnt.inc(S_RD_RO, static_cast<uint32_t>(tx.nr));
+                        next = true;
+                        cont = true;
+                        lane_snap = tx.snapshot;
+                    } else {
+                        tx.ph(PH_OTHER);                                  // waits for the warp's commit round
+                        stage = 1;
+                        // STM-HV-Backoff: an execution that follows a lock abort goes
+                        // straight to the sequential step -- its parallel attempt
+                        // already failed
+                        tries = (POL == POL_BACKOFF && lock_aborts) ? 1u : 0u;
+                    }
                 }
                 if (next) {                                           // the next transaction of thread t
                     fin = true;
@@ -467,13 +482,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
-            // (the serial owner pipelines the first round of every execution,
-            // whatever its size: once the executions in flight drained it is
-            // the only one running, §6.16)
-            const bool owner = serial_on && ss.owner();
-            const bool want_pipe = tries == 0 && (lock_aborts < p.lock_pipeline || owner);
-            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe,
-                                            owner ? 0x7fffffffu : p.pipeline_max_locks);
+            const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline;
+            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks);
             if (tx.pipelined_round) cnt.inc(S_PIPELINED);
             if (r == C_OK) {
                 got = true;
@@ -899,8 +909,9 @@ template <class K>
 inline cudaError_t launch_stm(K kernel, const KParams& kp, int block, cudaStream_t s, int warps_per_sm = 0,
                               size_t smem = 0)
 {
-    if (smem > 48 * 1024) {
-        // opt in to > 48 KB of dynamic shared memory once per (kernel, device, size)
+    if (smem > 0) {
+        // opt in to the dynamic shared memory once per (kernel, device, size):
+        // static + dynamic above 48 KB needs it (the counters take ~20 KB)
         static std::mutex mu;
         static std::set<std::tuple<const void*, int, size_t>> done;
         int dev = 0;

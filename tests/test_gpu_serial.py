@@ -20,6 +20,7 @@ CASES = [
     ("eb", dict(n_words=1024, n_accesses=64), 1024, 4, 10),    # the EB contention corner, scaled down
     ("eb", dict(n_words=64, n_accesses=16), 512, 4, 6),        # A <= 16 kernel (shared-memory logs)
     ("eb", dict(n_words=256, n_accesses=32), 512, 4, 8),       # A <= 32 kernel
+    ("eb", dict(n_words=16, n_accesses=16), 512, 4, 4),        # duplicate lock ids inside every batch
     ("ra", dict(n_reads=4, n_writes=4, n_words=64), 512, 8, 6),
     ("ra", dict(n_reads=3, n_words=16, ra_kind=1), 256, 4, 4),
     ("km", dict(km_clusters=8, km_dims=4), 2048, 1, 10),
