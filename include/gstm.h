@@ -166,8 +166,9 @@ typedef struct {
                              /*    ticket order (FIFO), each IRREVOCABLY: in place,  */
                              /*    under encounter-time version locks, stamped while */
                              /*    it holds them all -- serialised like an A3 commit */
-                             /*    (gstm/tx_irr.cuh).  Kernels of EB, RA and KM only  */
-                             /*    (bank and HT ignore it).  0 = off.  Default 0     */
+                             /*    (gstm/tx_irr.cuh).  Kernels of RA, KM and EB with */
+                             /*    A > 16 only (bank, HT and EB A <= 16 ignore it).  */
+                             /*    0 = off.  Default 0                               */
     uint32_t serial_commits; /*    see serial_after; 0 = 4.  Default 4                */
 } gstm_params_t;
 

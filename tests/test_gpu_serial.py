@@ -18,9 +18,9 @@ FORCE = dict(serial_after=1, serial_commits=1 << 16)
 # (workload, params, T, K, lock bits)
 CASES = [
     ("eb", dict(n_words=1024, n_accesses=64), 1024, 4, 10),    # the EB contention corner, scaled down
-    ("eb", dict(n_words=64, n_accesses=16), 512, 4, 6),        # A <= 16 kernel (shared-memory logs)
+    ("eb", dict(n_words=64, n_accesses=20), 512, 4, 6),        # A <= 32 kernel, short transactions
     ("eb", dict(n_words=256, n_accesses=32), 512, 4, 8),       # A <= 32 kernel
-    ("eb", dict(n_words=16, n_accesses=16), 512, 4, 4),        # duplicate lock ids inside every batch
+    ("eb", dict(n_words=16, n_accesses=24), 512, 4, 4),        # duplicate lock ids inside every batch
     ("ra", dict(n_reads=4, n_writes=4, n_words=64), 512, 8, 6),
     ("ra", dict(n_reads=3, n_words=16, ra_kind=1), 256, 4, 4),
     ("km", dict(km_clusters=8, km_dims=4), 2048, 1, 10),
@@ -62,10 +62,12 @@ def test_serial_corner_completes(k_lock):
 
 
 @pytest.mark.parametrize("wl,kw,bits", [("bank", dict(n_words=64), 6),
-                                        ("ht", dict(ht_buckets=16, ht_key_range=64, ht_lookup_pct=50), 8)])
+                                        ("ht", dict(ht_buckets=16, ht_key_range=64, ht_lookup_pct=50), 8),
+                                        ("eb", dict(n_words=64, n_accesses=16), 6)])
 def test_serial_not_compiled_for_bank_ht(wl, kw, bits):
-    """Bank and HT kernels leave the contention manager out (WL::kSerialGate,
-    their register budget): serial_after is accepted and ignored."""
+    """Bank, HT and the EB A <= 16 kernels leave the contention manager out
+    (WL::kSerialGate, their register budget): serial_after is accepted and
+    ignored."""
     T, K = 512, 4
     g, gp, op, init = U.make(wl, T, K, bits, mode="hv", **FORCE, **kw)
     try:
