@@ -760,6 +760,8 @@ def bank_extras(args, G, R, g, stream, flush, dev, T, K, seed0, var, mode_used, 
         extra["cgl"] = {"value": cgl["value"], "unit": UNIT, "threads": cgl["threads"],
                         "backoff_ns": cgl["backoff_ns"], "kernel": "cgl_kernel<BankWL>"}
         extra["speedup_vs_cgl"] = value / world / cgl["value"]
+        # the paper's own figure, context only (its Figures 2-5 are lost)
+        extra["paper_speedup_vs_cgl"] = {"value": "up to 20x", "gpu": "Tesla C2070 (Fermi)", "cite": "P:11, P:246"}
         table = [Variant("auto", "split"), Variant("tbv", "split"), Variant("hv", "split"),
                  Variant("tbv", "paired"), Variant("hv", "paired", prelock=1),
                  Variant("hv_backoff", "split"), Variant("hv_backoff", "paired", k_lock=1),

@@ -330,7 +330,12 @@ struct HtWL {
     {
         uint32_t key, ins, bucket;
         key_of(p, x, key, ins, bucket);
-        const uint64_t B = p.ht_buckets, M = p.T * p.K;
+        // 32-bit word bases (check(): B + 2M < 2^32): one register each, so
+        // the walk's addresses are not rematerialised from 64-bit products
+        // under HV's 64-register budget
+        const uint32_t M = static_cast<uint32_t>(p.T * p.K);
+        const uint32_t kbase = p.ht_buckets - 1u;       // key[h] = heap[kbase + h]
+        const uint32_t nbase = kbase + M;               // next[h] = heap[nbase + h]
         // lanes that run their bodies together walk their chains in lockstep:
         // one warp-collective step per chain node, so a step's loads, lock
         // checks and log inserts are executed once for every walking lane
@@ -343,6 +348,8 @@ struct HtWL {
         // step s > 0: key and next of the s-th node), so PostValidation and
         // the lock spin are inlined once
         uint32_t h0 = 0, h = 0, found = 0;
+        uint32_t ka = bucket;   // the word a[0] reads: the bucket head, then key[h] (bucket is not
+                                // used inside the walk, so it is not rematerialised at every step)
         bool walking = live;
         for (int steps = 0;; ++steps) {
             if (walking && steps > 0 && h > M) { c.invalid(); walking = live = false; }
@@ -351,8 +358,8 @@ struct HtWL {
             if (!wm) break;
             if (walking) {
                 uint32_t a[2], v[2];
-                a[0] = steps ? static_cast<uint32_t>(B + h - 1) : bucket;          // key[h] / head
-                a[1] = static_cast<uint32_t>(B + M + h - 1);                      // next[h]
+                a[0] = ka;                                                        // head / key[h]
+                a[1] = nbase + h;                                                 // next[h]
                 if (mask) c.set_sync_mask(wm);               // read_batch reconverges the walking lanes
                 c.template read_batch<2>(a, v, steps ? 2 : 1);
                 if (!c.ok()) {
@@ -367,6 +374,7 @@ struct HtWL {
                     h = v[1];
                     walking = h != 0;
                 }
+                ka = kbase + h;
             }
         }
         if (mask) c.set_sync_mask(0u);
@@ -374,9 +382,9 @@ struct HtWL {
         if (!ins) { result = found; return; }
         if (found) { result = 2; return; }
         const uint32_t n = static_cast<uint32_t>(1 + i * p.T + t);
-        c.write(static_cast<uint32_t>(B + n - 1), key);
-        c.write(static_cast<uint32_t>(B + M + n - 1), h0);
-        c.write(bucket, n);
+        c.write(kbase + n, key);
+        c.write(nbase + n, h0);
+        c.write(static_cast<uint32_t>(gen::mix64(key) & (p.ht_buckets - 1)), n);   // the bucket (key_of)
         result = 3;
     }
     template <class F>
@@ -413,7 +421,10 @@ struct EbWLT {
     // kernel (hot set 2^26: 677 -> 650 M tx/s with it) never needs it (its worst sweep point, hot set
     // 2^10, runs 2.9x CGL)
     static constexpr bool kSerialGate = MAXA > 16;
-    static constexpr int kMinBlocks = 2;
+#ifndef GSTM_EB16_MINB
+#define GSTM_EB16_MINB 2
+#endif
+    static constexpr int kMinBlocks = MAXA <= 16 ? GSTM_EB16_MINB : 2;
     static constexpr int DESCR = 2 * MAXA;
     __host__ static bool check(const WlParams& p) { return p.n_accesses <= MAXA && p.n_words > 0; }
     __host__ static uint64_t footprint(const WlParams& p) { return p.n_words; }
