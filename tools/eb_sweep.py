@@ -4,7 +4,7 @@ study of P:319-325): hot-set size H x accesses per transaction A, with the
 STM, FGL and CGL measured at EVERY point, plus the version-lock count sweep
 at large H.
 
-    python tools/eb_sweep.py --out profiles/r02_eb_sweep.jsonl
+    python tools/eb_sweep.py --out profiles/r02_eb_sweep_cm.jsonl
 
 Every point runs over a 2^26-word heap (one fresh handle per measurement, one
 warm-up launch, then a timed launch with CUDA events, L2 flushed before it).
@@ -64,7 +64,8 @@ def main():
         return {"tx_per_s": done / (ms * 1e-3), "ms": ms, "abort_ratio": st.aborts / max(1, st.aborts + done),
                 "status": st.status, "completed": bool(st.status == 0 and done == T * K), "threads": T,
                 "tx_per_thread": K, "postvalidations": st.postvalidations, "aborts_opacity": st.aborts_opacity,
-                "aborts_prevbv": st.aborts_prevbv, "aborts_tbv": st.aborts_tbv, "aborts_lock": st.aborts_lock}
+                "aborts_prevbv": st.aborts_prevbv, "aborts_tbv": st.aborts_tbv, "aborts_lock": st.aborts_lock,
+                "serial_runs": st.serial_runs}
 
     def emit(rec):
         line = json.dumps(rec)
@@ -92,6 +93,10 @@ def main():
                    "max_threads": cap}
             rec["hv"] = run(h, A, bits, "hv", T, K, max_threads=cap)
             rec["tbv"] = run(h, A, bits, "tbv", T, K, max_threads=cap)
+            if A > 16:
+                # the contention manager (serial tickets, irrevocable owner;
+                # DESIGN.md §6.16), compiled into the A > 16 kernels
+                rec["hv_cm"] = run(h, A, bits, "hv", T, K, max_threads=cap, serial_after=4)
             rec["fgl"] = run(h, A, bits, "fgl", T, K)
             # CGL: fastest of 1 warp per SM / 2^14 threads, Scheme #3 / TTAS + backoff, ~4K transactions
             cg = {}
@@ -102,7 +107,9 @@ def main():
             rec["cgl"] = dict(cg[(Tc, bo)], backoff_ns=bo)
             best_stm = max(rec["hv"]["tx_per_s"], rec["tbv"]["tx_per_s"])
             rec["stm_over_cgl"] = best_stm / rec["cgl"]["tx_per_s"]
-            rec["completed"] = all(rec[m]["completed"] for m in ("hv", "tbv", "fgl", "cgl"))
+            if "hv_cm" in rec:
+                rec["stm_cm_over_cgl"] = rec["hv_cm"]["tx_per_s"] / rec["cgl"]["tx_per_s"]
+            rec["completed"] = all(rec[m]["completed"] for m in ("hv", "tbv", "fgl", "cgl", "hv_cm") if m in rec)
             rec["wall_s"] = round(time.perf_counter() - t0, 2)
             emit(rec)
     # version-lock count at the largest hot set
