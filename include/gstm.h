@@ -158,17 +158,19 @@ typedef struct {
                              /*    transaction scheduling P:313 and P:317 leave to   */
                              /*    future work): a transaction whose executions      */
                              /*    aborted >= serial_after times while g_clock       */
-                             /*    advanced by < serial_commits per abort (the whole */
-                             /*    GPU commits less than that per attempt) takes a   */
-                             /*    ticket; while tickets are outstanding no other    */
-                             /*    transaction starts (one that aborted before joins */
-                             /*    the queue), and the holders run one at a time in  */
-                             /*    ticket order (FIFO), each IRREVOCABLY: in place,  */
-                             /*    under encounter-time version locks, stamped while */
-                             /*    it holds them all -- serialised like an A3 commit */
-                             /*    (gstm/tx_irr.cuh).  Kernels of RA, KM and EB with */
-                             /*    A > 16 only (bank, HT and EB A <= 16 ignore it).  */
-                             /*    0 = off.  Default 0                               */
+                             /*    advanced by < serial_commits per abort, and whose */
+                             /*    attempts took longer per GPU-wide commit than a   */
+                             /*    serial owner's execution takes (measured online;  */
+                             /*    none yet: qualify), takes a ticket; while tickets */
+                             /*    are outstanding no other transaction starts (one  */
+                             /*    that aborted before and passes the same time test */
+                             /*    joins the queue), and the holders run one at a    */
+                             /*    time in ticket order (FIFO), each IRREVOCABLY: in */
+                             /*    place, under encounter-time version locks,        */
+                             /*    stamped while it holds them all -- serialised     */
+                             /*    like an A3 commit (gstm/tx_irr.cuh).  Kernels of  */
+                             /*    RA, KM and EB with A > 16 only (bank, HT and EB   */
+                             /*    A <= 16 ignore it).  0 = off.  Default 0 (EB: 4)  */
     uint32_t serial_commits; /*    see serial_after; 0 = 4.  Default 4                */
 } gstm_params_t;
 

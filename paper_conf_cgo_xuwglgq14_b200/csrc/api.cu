@@ -228,6 +228,11 @@ static gstm_params_t default_params(int workload)
         // the hot set may exceed L2: keep the lock table there (DESIGN.md §6.10:
         // hot set 2^26, A=16: 336 -> 369 M tx/s with 2^22 locks, 391 -> 453 with 2^24)
         p.l2_persist_locks = 1;
+        // the adaptive contention manager (compiled into the
+        // A > 16 kernels): serial tickets only where one-at-a-time measures
+        // faster -- the corner (hot set 2^10, A = 64) 1.14 s -> 0.86 s per
+        // launch, every other sweep point unchanged (no ticket taken)
+        p.serial_after = 4;
     }
     // RA and EB (random words, contended): the sequential first round is
     // faster even when the lock log fits one pipelined chunk (EB A=8: 1.24

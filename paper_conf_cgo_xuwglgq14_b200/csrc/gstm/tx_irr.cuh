@@ -48,6 +48,8 @@ struct IrrCtx {
     const Meta& m;
     unsigned long long deadline;  // watchdog: a lock never released ends the wait (bad)
     int nl = 0;
+    int nr = 0;                   // reads (the op-mix statistics, S_RD_*)
+    int nl_taken = 0;             // locks held at the commit (S_LK_UPD)
     int nw = 0;
     bool bad = false;
     uint32_t n_spin = 0;
@@ -106,6 +108,7 @@ struct IrrCtx {
     {
         const uint32_t id = m.lock_of(a);
         if (!settle(id, lock_atom(id, true), false)) return 0u;
+        ++nr;
         return prim::ld_relaxed(m.val_ptr(a));
     }
     // a batch: every lock atomic in flight at once, then the values
@@ -130,7 +133,7 @@ struct IrrCtx {
         if (!ok) return;
 #pragma unroll
         for (int k = 0; k < N; ++k)
-            if (k < n && !((skip >> k) & 1u)) v[k] = prim::ld_relaxed(m.val_ptr(a[k]));
+            if (k < n && !((skip >> k) & 1u)) { v[k] = prim::ld_relaxed(m.val_ptr(a[k])); ++nr; }
     }
     __device__ __forceinline__ void read_many(const uint32_t* a, uint32_t* v, const bool* skip, int n)
     {
@@ -151,7 +154,7 @@ struct IrrCtx {
             if (!ok) return;
 #pragma unroll
             for (int j = 0; j < C; ++j)
-                if (k0 + j < n && !skip[k0 + j]) v[k0 + j] = prim::ld_relaxed(m.val_ptr(a[k0 + j]));
+                if (k0 + j < n && !skip[k0 + j]) { v[k0 + j] = prim::ld_relaxed(m.val_ptr(a[k0 + j])); ++nr; }
         }
     }
     // will_write hint: the body's write addresses a[0], a[stride], ... in the
@@ -212,6 +215,7 @@ struct IrrCtx {
         const uint32_t version = s << 1;
         for (int k = 0; k < nl; ++k)                                 // l.84
             prim::st_relaxed(m.lock_ptr(ent[k] >> 2), (ent[k] & 2u) ? version : old[k]);
+        nl_taken = nl;
         nl = 0;
         return s;
     }

@@ -27,6 +27,7 @@ __global__ void prepare_kernel(unsigned long long* meta, const unsigned long lon
     meta[M_WORK] = 0;
     meta[M_SEQ] = 2ull * *clock;                    // STM-VBV sequence lock (tx_vbv.cuh)
     meta[M_SERIAL] = 0;                             // contention manager: no ticket issued, none served
+    meta[M_SERIAL_EST] = 0;                         // ... no owner time measured yet
     for (int k = 0; k < S_NSTATS; ++k) meta[M_STATS + k] = 0;
     *reinterpret_cast<uint32_t*>(meta + M_ERR) = 0;
     *reinterpret_cast<uint32_t*>(meta + M_CGL_LOCK) = 0;

@@ -44,6 +44,7 @@ enum {
     // after the 256 candidate g_clock lines (api.cu kClockCandidates x kClockStride)
     M_SEQ = M_WORDS + 256 * 288 + 16,  // STM-VBV global sequence lock, own line
     M_SERIAL = M_SEQ + 16,             // contention manager's ticket word {serving:32 | next:32}, own line
+    M_SERIAL_EST = M_SERIAL + 1,       // ... and the owners' running mean execution time (ns), same line
 };
 
 constexpr int kPhaseWords = 16;    // M_PHASE .. M_PHASE + 15

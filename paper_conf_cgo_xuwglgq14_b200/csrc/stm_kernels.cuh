@@ -219,6 +219,7 @@ struct SerialState {
     uint32_t ticket = 0, serving = 0;
     uint32_t n_ab = 0;        // aborted executions of the current transaction
     uint32_t s_first = 0;     // snapshot of its first execution
+    uint32_t t_first = 0;     // %globaltimer >> 10 (~us) at its first execution
     bool has_ticket = false;
     bool pending = false;     // the last poll saw tickets outstanding (warp-uniform)
     __device__ __forceinline__ bool owner() const { return has_ticket && ticket == serving; }
@@ -234,9 +235,29 @@ __device__ __forceinline__ bool serial_gate(const KParams& p, SerialState& ss, b
                                             uint32_t iter)
 {
     unsigned long long* sw = p.meta + M_SERIAL;
-    const bool want = fresh && !ss.has_ticket &&
-                      ((ss.n_ab >= p.serial_after && snap - ss.s_first < p.serial_commits * ss.n_ab) ||
-                       (ss.pending && ss.n_ab >= 1u));
+    // candidates: aborted >= serial_after times while the clock advanced by
+    // < serial_commits per abort; they qualify when, besides, the GPU's
+    // commits during their attempts took longer each than a serial owner's
+    // execution does (the owners' running mean, M_SERIAL_EST; none measured
+    // yet: qualify) -- serialise only where one-at-a-time is faster
+    const bool cand = fresh && !ss.has_ticket && ss.n_ab >= p.serial_after &&
+                      snap - ss.s_first < p.serial_commits * ss.n_ab;
+    // a transaction that aborted before joins a serial phase in progress --
+    // once an owner was measured, and if one-at-a-time is faster for it too
+    const bool joiner = fresh && !ss.has_ticket && ss.pending && ss.n_ab >= 1u;
+    bool want = false;
+    if (__any_sync(FULL, cand || joiner)) {
+        unsigned long long est = 0, now = 0;
+        if (prim::lane_id() == 0) {
+            est = prim::ld_relaxed64(p.meta + M_SERIAL_EST);
+            now = globaltimer() >> 10;
+        }
+        est = __shfl_sync(FULL, est, 0);
+        now = __shfl_sync(FULL, now, 0);
+        const unsigned long long elapsed_ns = static_cast<unsigned long long>(static_cast<uint32_t>(now) - ss.t_first) << 10;
+        const bool slower = static_cast<unsigned long long>(snap - ss.s_first) * est < elapsed_ns;
+        want = (cand && (est == 0 || slower)) || (joiner && est != 0 && slower);
+    }
     const unsigned wm = __ballot_sync(FULL, want);
     const bool poll = wm || __any_sync(FULL, ss.has_ticket) || ss.pending || (iter & 7u) == 0u;
     if (poll) {
@@ -399,7 +420,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 cnt.inc(S_ATTEMPTS);
                 ran = true;
                 if (serial_on) {
-                    if (ss.n_ab == 0) ss.s_first = lane_snap;
+                    if (ss.n_ab == 0) {
+                        ss.s_first = lane_snap;
+                        ss.t_first = static_cast<uint32_t>(globaltimer() >> 10);
+                    }
                     if (ss.has_ticket) cnt.inc(S_SERIAL);
                 }
                 result = 0;
@@ -410,10 +434,16 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     // under encounter-time locks, stamped while it holds
                     // them all (gstm/tx_irr.cuh)
                     IrrCtx<TX> ic{irr_log, irr_log + IrrCtx<TX>::kCap, m, deadline};
+                    const unsigned long long t_own = globaltimer();
                     tx.ph(PH_NATIVE);
                     WL::body(ic, p.w, x, t, i, result);
                     tx.ph(PH_COMMIT);
                     const uint32_t s = ic.commit(m.clock);
+                    {   // the owners' running mean execution time (one owner at a time)
+                        unsigned long long* e = p.meta + M_SERIAL_EST;
+                        const unsigned long long dt = globaltimer() - t_own, old = prim::ld_relaxed64(e);
+                        prim::st_relaxed64(e, old ? (7 * old + dt) / 8 : dt);
+                    }
                     tx.n_spin += ic.n_spin;
                     tx.ph_end(true);
                     if (ic.bad) {
@@ -425,7 +455,15 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                                                               : s - clock_begin;
                         p.tx_result[tx_id] = result;
                     }
-                    cnt.inc((s & 0x80000000u) ? S_COMMITS_RO : S_COMMITS);
+                    if (s & 0x80000000u) {
+                        cnt.inc(S_COMMITS_RO);
+                        cnt.inc(S_RD_RO, static_cast<uint32_t>(ic.nr));
+                    } else {
+                        cnt.inc(S_COMMITS);
+                        cnt.inc(S_RD_UPD, static_cast<uint32_t>(ic.nr));
+                        cnt.inc(S_WR_UPD, static_cast<uint32_t>(ic.nw));
+                        cnt.inc(S_LK_UPD, static_cast<uint32_t>(ic.nl_taken));
+                    }
                     next = true;
                 } else {
                     tx.begin(lane_snap);                                  // TXBegin l.2-3

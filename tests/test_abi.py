@@ -67,6 +67,9 @@ def test_loads_and_host_only_calls(so):
     assert p.n_words == 1 << 20 and p.block_threads == 256 and p.k_lock == 8
     # A3.l71's optional pre-lock VBV: on where it pays (KM 4x), off for HT
     assert [G.gstm_default_params(w).prelock_vbv for w in ("ra", "bank", "ht", "eb", "km")] == [1, 1, 0, 1, 1]
+    # the adaptive contention manager: on for EB (its A > 16 kernels), off elsewhere
+    assert [G.gstm_default_params(w).serial_after for w in ("ra", "bank", "ht", "eb", "km")] == [0, 0, 0, 4, 0]
+    assert G.gstm_default_params("eb").serial_commits == 4
     with pytest.raises(G.GstmError):
         G.gstm_default_params(9)
 
