@@ -22,9 +22,9 @@
 namespace gstm {
 
 template <int RCAP, int WCAP, int LCAP, bool LOCAL = false, bool SORTED = true, bool COMPACT = false,
-          bool HLOG = false, bool SMEM = false>
-struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM> {
-    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM>;
+          bool HLOG = false, bool SMEM = false, bool COLDPV = false>
+struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM, COLDPV> {
+    using B = Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM, COLDPV>;
     using B::kUnroll;
     using B::r_addr;
     using B::r_val;

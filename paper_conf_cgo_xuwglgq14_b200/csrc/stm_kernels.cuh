@@ -76,6 +76,13 @@ struct SmemLogs { static constexpr bool value = false; };
 template <class WL>
 struct SmemLogs<WL, std::void_t<decltype(WL::kSmemLogs)>> { static constexpr bool value = WL::kSmemLogs; };
 
+// WL::kColdPostValidation (optional): PostValidation in its smallest form
+// (Tx COLDPV) -- RA
+template <class WL, class = void>
+struct ColdPv { static constexpr bool value = false; };
+template <class WL>
+struct ColdPv<WL, std::void_t<decltype(WL::kColdPostValidation)>> { static constexpr bool value = WL::kColdPostValidation; };
+
 // WL::kRunWriteback (optional): the write-set is runs of consecutive words
 // (a record): write back with 16-byte vector stores (Tx::writeback_runs)
 template <class WL, class = void>
@@ -325,9 +332,9 @@ template <class WL, bool PAIR, int POL>
 using StmTx = std::conditional_t<
     PAIR,
     TxPair<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value,
-           HashedLog<WL>::value, SmemLogs<WL>::value>,
+           HashedLog<WL>::value, SmemLogs<WL>::value, ColdPv<WL>::value>,
     Tx<WL::RCAP, WL::WCAP, WL::LCAP, LocalLogs<WL>::value, POL == POL_SORTED, Compact<WL>::value, HashedLog<WL>::value,
-       SmemLogs<WL>::value>>;
+       SmemLogs<WL>::value, ColdPv<WL>::value>>;
 
 // dynamic shared memory of the STM kernel: the shared-memory logs, if any
 template <class WL, bool PAIR, int POL>
