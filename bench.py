@@ -498,15 +498,19 @@ def sig(x: float, n: int = 4) -> float:
     return float(f"{x:.{n}g}")
 
 
-def first_round_pipelined(wl, gp, st) -> bool:
+def first_round_pipelined(wl, gp, st):
     """Does the kernel issue a transaction's first lock round all at once
     ?  Register logs (bank) always may; local-memory logs only
-    when the lock log fits one 8-atomic chunk (Q36)."""
+    when the lock log fits one 8-atomic chunk (Q36) -- longer ones take the
+    gated round ("gated": the lowest lock, then the rest) with
+    lock_pipeline_gated, else the sequential one."""
     if gp.lock_pipeline == 0:
         return False
     if wl == "bank":
         return True
-    return st.commits > 0 and st.locks_update / st.commits <= 8
+    if st.commits > 0 and st.locks_update / st.commits <= 8:
+        return True
+    return "gated" if gp.lock_pipeline_gated else False
 
 
 def run_config(G, R, stream, flush, name, seed):

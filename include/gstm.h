@@ -172,6 +172,13 @@ typedef struct {
                              /*    RA, KM and EB with A > 16 only (bank, HT and EB   */
                              /*    A <= 16 ignore it).  0 = off.  Default 0 (EB: 4)  */
     uint32_t serial_commits; /*    see serial_after; 0 = 4.  Default 4                */
+    uint32_t lock_pipeline_gated; /* 1: a transaction's pipelined lock round (see    */
+                             /*    lock_pipeline) whose local/shared-memory lock log */
+                             /*    is longer than pipeline_max_locks takes its LOWEST */
+                             /*    lock alone first (held: the round fails having    */
+                             /*    touched nothing else) and then every other lock   */
+                             /*    at once.  0: such logs take the  */
+                             /*    sequential round.  Default 0 (KM: 1)              */
 } gstm_params_t;
 
 typedef struct {

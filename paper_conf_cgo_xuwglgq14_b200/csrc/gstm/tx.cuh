@@ -921,6 +921,45 @@ struct Tx {
         return true;
     }
 
+    // The gated pipelined round (local/shared-memory logs longer than one
+    // pipelined chunk; `lock_pipeline_gated`): the lowest
+    // lock alone first -- held by someone: the round fails having touched
+    // nothing else, as the sequential round would -- then every other lock
+    // at once (kChunk atomics in flight).  Where all contenders of a record
+    // need the same lowest lock (k-means: 17 consecutive lock words), the
+    // gate picks the winner and the lock-holding time drops from nl
+    // dependent round trips to two.
+    __device__ __forceinline__ bool get_locks_and_tbv_gated_local(const Meta& m)
+    {
+        n_acq = 0;
+        const uint32_t v0 = prim::atom_or_acquire(m.lock_ptr(l_ent[0] >> 2), 1u);   // l.45, the gate
+        if (v0 & 1u) return false;                                   // l.46-48: nothing held
+        l_old[0] = v0;
+        bool ok = true;
+        for (int k0 = 1; k0 < nl; k0 += kChunk) {
+            uint32_t vl[kChunk];
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) vl[j] = prim::atom_or_relaxed(m.lock_ptr(l_ent[k0 + j] >> 2), 1u);
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) {
+                    l_old[k0 + j] = vl[j];
+                    ok &= !(vl[j] & 1u);
+                }
+        }
+        prim::fence_acquire();
+        if (!ok) {
+            GSTM_LLOOP(for (int k = 0; k < nl; ++k)                  // l.47: undo what this round set
+                if (!(l_old[k] & 1u)) prim::st_relaxed(m.lock_ptr(l_ent[k] >> 2), l_old[k]););
+            return false;
+        }
+        GSTM_LLOOP(for (int k = 0; k < nl; ++k)
+            if ((l_ent[k] & 1u) && (l_old[k] >> 1) > snapshot) passTBV = false;);   // l.49-51
+        n_acq = nl;
+        return true;
+    }
+
     // Commit steps up to the write-back (A3.l67-78).  Returns C_OK when all
     // locks are held and the read-set is valid, C_LOCK on a lock conflict
     // (nothing held; retry, l.73-74), or an abort cause (nothing held).
@@ -928,20 +967,22 @@ struct Tx {
     // for local-memory logs, only if the (complete) log has at most
     // max_pipe_locks entries -- pipelined_round reports the decision
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool want_pipe = false,
-                                                  uint32_t max_pipe_locks = 8u)
+                                                  uint32_t max_pipe_locks = 8u, bool gated = false)
     {
         ph(PH_BUFFER);
         insert_deferred_reads(m);
         compact();
         const bool pipelined = want_pipe && (kUnroll || nl <= static_cast<int>(max_pipe_locks));
-        pipelined_round = pipelined;
+        const bool gate = want_pipe && gated && !pipelined && !kUnroll;   // (kUnroll: pipelined already)
+        pipelined_round = pipelined || gate;
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
         ph(PH_LOCKS);
         bool got;
         if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
-        else got = pipelined ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
+        else got = pipelined ? get_locks_and_tbv_pipelined_local(m)
+                             : gate ? get_locks_and_tbv_gated_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; } // Q18

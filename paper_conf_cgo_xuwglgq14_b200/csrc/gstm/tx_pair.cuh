@@ -432,24 +432,60 @@ struct TxPair : Tx<RCAP, WCAP, LCAP, LOCAL, SORTED, COMPACT, HLOG, SMEM, COLDPV>
         return true;
     }
 
+    // the gated pipelined round (tx.cuh get_locks_and_tbv_gated_local) on pairs
+    __device__ __forceinline__ bool get_locks_and_tbv_gated_local(const Meta& m)
+    {
+        n_acq = 0;
+        const unsigned long long o0 = prim::atom_or_acquire_u64(m.pair_ptr(l_ent[0] >> 2), 1ull << 32);   // the gate
+        if (hi(o0) & 1u) return false;
+        l_old[0] = hi(o0);
+        l_val[0] = lo(o0);
+        bool ok = true;
+        for (int k0 = 1; k0 < nl; k0 += kChunk) {
+            unsigned long long old[kChunk];
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) old[j] = prim::atom_or_relaxed_u64(m.pair_ptr(l_ent[k0 + j] >> 2), 1ull << 32);
+#pragma unroll
+            for (int j = 0; j < kChunk; ++j)
+                if (k0 + j < nl) {
+                    l_old[k0 + j] = hi(old[j]);
+                    l_val[k0 + j] = lo(old[j]);
+                    ok &= !(hi(old[j]) & 1u);
+                }
+        }
+        prim::fence_acquire();
+        if (!ok) {
+            for (int k = 0; k < nl; ++k)
+                if (!(l_old[k] & 1u)) prim::st_relaxed_u64(m.pair_ptr(l_ent[k] >> 2), mk(l_val[k], l_old[k]));
+            return false;
+        }
+        for (int k = 0; k < nl; ++k)
+            if ((l_ent[k] & 1u) && (l_old[k] >> 1) > snapshot) passTBV = false;
+        n_acq = nl;
+        return true;
+    }
+
     // want_pipe: this round may be the pipelined first round (§6.4); it is,
     // for local-memory logs, only if the (complete) log has at most
     // max_pipe_locks entries -- pipelined_round reports the decision
     __device__ __forceinline__ int commit_acquire(const Meta& m, int mode, bool prelock_vbv, bool want_pipe = false,
-                                                  uint32_t max_pipe_locks = 8u)
+                                                  uint32_t max_pipe_locks = 8u, bool gated = false)
     {
         ph(PH_BUFFER);
         B::insert_deferred_reads(m);
         B::compact();
         const bool pipelined = want_pipe && (kUnroll || nl <= static_cast<int>(max_pipe_locks));
-        B::pipelined_round = pipelined;
+        const bool gate = want_pipe && gated && !pipelined && !kUnroll;
+        B::pipelined_round = pipelined || gate;
         ph(PH_CONSIST);
         if (mode == MODE_HV && prelock_vbv)
             if (!vbv(m)) return C_PREVBV;                            // l.71-72
         ph(PH_LOCKS);
         bool got;
         if constexpr (kUnroll) got = get_locks_and_tbv_converged(m, pipelined);
-        else got = pipelined ? get_locks_and_tbv_pipelined_local(m) : get_locks_and_tbv(m);
+        else got = pipelined ? get_locks_and_tbv_pipelined_local(m)
+                             : gate ? get_locks_and_tbv_gated_local(m) : get_locks_and_tbv(m);
         if (!got) return C_LOCK;                                     // l.73
         if (!passTBV) {                                              // l.75
             if (mode != MODE_HV) { release_locks(m); return C_TBV; }

@@ -73,6 +73,7 @@ struct KParams {
     uint32_t lock_log_at_commit;   // read locks enter the sorted lock log at TXCommit (Tx::insert_read_lock)
     uint32_t serial_after;         // contention manager: aborts before a transaction may take a serial ticket (0 = off)
     uint32_t serial_commits;       // ... only while the clock advanced by < serial_commits per abort
+    uint32_t lock_pipeline_gated;  // pipelined rounds of longer local/shared logs: the lowest lock first, then the rest
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);

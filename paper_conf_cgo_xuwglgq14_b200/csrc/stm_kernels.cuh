@@ -528,7 +528,8 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
             const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline;
-            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks);
+            const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks,
+                                            p.lock_pipeline_gated != 0);
             if (tx.pipelined_round) cnt.inc(S_PIPELINED);
             if (r == C_OK) {
                 got = true;

@@ -47,8 +47,10 @@ class TxShape:
         return sum(self.read_batches)
 
 
-def stm_program(shape: TxShape, paired: bool, hv_prelock: bool, pipelined: bool) -> list:
-    """Phases of one transaction under STM-HV/TBV (tx.cuh / tx_pair.cuh)."""
+def stm_program(shape: TxShape, paired: bool, hv_prelock: bool, pipelined) -> list:
+    """Phases of one transaction under STM-HV/TBV (tx.cuh / tx_pair.cuh).
+    pipelined: False (sorted, one lock at a time), True (one round trip) or
+    "gated" (the lowest lock, then the rest in one round trip)."""
     p, slot = [], 0
     for n in shape.read_batches:                       # TXRead batches (A3.l21-35)
         if n <= 0:
@@ -64,7 +66,10 @@ def stm_program(shape: TxShape, paired: bool, hv_prelock: bool, pipelined: bool)
     if hv_prelock and R:
         p.append(ph(LD_V, R, 0))                       # l.71 pre-lock VBV, all reads at once
     n = shape.locks
-    if pipelined:
+    if pipelined == "gated" and n > 1:                 # the gated round (§6.4): the lowest lock, then the rest
+        p.append(ph(ATOM_L, 1, 0))
+        p.append(ph(ATOM_L, n - 1, 1))
+    elif pipelined:
         p.append(ph(ATOM_L, n, 0))                     # l.45, one round trip
     else:
         p += [ph(ATOM_L, 1, k) for k in range(n)]      # l.44-48: sorted, one at a time (Q15)

@@ -70,6 +70,8 @@ def test_loads_and_host_only_calls(so):
     # the adaptive contention manager: on for EB (its A > 16 kernels), off elsewhere
     assert [G.gstm_default_params(w).serial_after for w in ("ra", "bank", "ht", "eb", "km")] == [0, 0, 0, 4, 0]
     assert G.gstm_default_params("eb").serial_commits == 4
+    # the gated pipelined lock round: k-means only
+    assert [G.gstm_default_params(w).lock_pipeline_gated for w in ("ra", "bank", "ht", "eb", "km")] == [0, 0, 0, 0, 1]
     with pytest.raises(G.GstmError):
         G.gstm_default_params(9)
 

@@ -189,6 +189,11 @@ def test_op_mix_programs_follow_algorithm_3():
     assert R.op_counts(p)["atom"] == 17.0
     assert R.op_counts(p)["ld"] == 0.0                        # the lock-holding critical section only
     assert p[3 + 2] & 0xff == R.ATOM_L
+    # the gated round (lock_pipeline_gated): the lowest lock alone, then the other 16 at once
+    p = R.programs_from_stats("km", st, paired=False, mode="hv", prelock=True, pipelined="gated", records=(1024, 17))
+    atoms = [c for c in p[5:5 + p[4]] if c & 0xff == R.ATOM_L]
+    assert [((c >> 8) & 0xff, c >> 16) for c in atoms] == [(1, 0), (16, 1)]
+    assert R.op_counts(p)["atom"] == 17.0
 
 
 def test_bench_self_launches_n_ranks_with_gloo():
