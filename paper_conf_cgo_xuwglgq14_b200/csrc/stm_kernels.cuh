@@ -402,6 +402,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
         have_snap = false;
         bool done = false, aborted = false, fin = false, ran = false;
         const bool may_start = serial_on ? serial_gate(p, ss, act && stage == 0 && i < p.K, snap, iter) : true;
+        if (!may_start && act && stage == 0) tx.ph(PH_OTHER);   // held back by the serial queue: not in a transaction
         // Body rounds (p.body_rounds): a lane whose
         // transaction committed read-only (A3.l68: no locks, no stamp) starts
         // its next transaction in the same warp iteration, up to body_rounds
