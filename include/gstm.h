@@ -31,7 +31,10 @@
 extern "C" {
 #endif
 
-#define GSTM_API_VERSION 1
+/* 2: gstm_params_t gained serial_after, serial_commits, lock_pipeline_gated and
+ *    gstm_stats_t gained serial_runs (appended; the structs are passed by
+ *    pointer, so a client built against version 1 must be rebuilt) */
+#define GSTM_API_VERSION 2
 
 typedef struct gstm_handle gstm_t;   /* opaque; owns the lock table, clock, stats, logs, heap */
 

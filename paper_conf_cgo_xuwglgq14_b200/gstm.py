@@ -26,6 +26,7 @@ MODES = {"auto": MODE_AUTO, "hv": MODE_HV, "tbv": MODE_TBV, "cgl": MODE_CGL, "fg
          "hv_backoff": MODE_HV_BACKOFF, "vbv": MODE_VBV, "hv_unsorted": MODE_HV_UNSORTED}
 MODE_NAMES = {v: k for k, v in MODES.items()}
 RO_FLAG = 0x80000000
+API_VERSION = 2          # include/gstm.h GSTM_API_VERSION these structs mirror
 
 STATUS = {0: "GSTM_OK", -1: "GSTM_EINVAL", -2: "GSTM_ENOMEM", -3: "GSTM_ECUDA", -4: "GSTM_ELOGOVF",
           -5: "GSTM_EOVERFLOW", -6: "GSTM_ETIMEOUT", -7: "GSTM_EBUSY", -8: "GSTM_ENODEV"}
@@ -147,6 +148,10 @@ def lib(flavour: str = ""):
             f = getattr(L, name)
             f.restype = res
             f.argtypes = args
+        if L.gstm_api_version() != API_VERSION:
+            # the ctypes structs below mirror include/gstm.h of this version
+            raise GstmError(f"{path}: API version {L.gstm_api_version()}, binding expects {API_VERSION} "
+                            "(rebuild: python -m paper_conf_cgo_xuwglgq14_b200.build --force)")
         _libs[flavour] = L
     return _libs[flavour]
 

@@ -62,7 +62,7 @@ def test_library_is_sm100a_and_self_contained(so):
 
 def test_loads_and_host_only_calls(so):
     L = G.lib()
-    assert L.gstm_api_version() == 1
+    assert L.gstm_api_version() == 2
     p = G.gstm_default_params("bank")
     assert p.n_words == 1 << 20 and p.block_threads == 256 and p.k_lock == 8
     # A3.l71's optional pre-lock VBV: on where it pays (KM 4x), off for HT
