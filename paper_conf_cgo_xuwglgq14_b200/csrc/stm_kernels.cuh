@@ -395,10 +395,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     while (__any_sync(FULL, t < p.T)) {
         if (warp_late(iter++, deadline)) { timed_out = true; break; }
         const bool act = t < p.T;
-        // (a lane the serial queue held back last iteration waits outside a
-        // transaction: "other", like the check below once the gate decided)
+        // (a lane the serial queue may hold back waits outside a transaction:
+        // "other" until its execution starts, PH_INIT below)
         tx.ph(!act ? PH_OTHER : stage == 1 ? PH_LOCKS
-              : (serial_on && ss.pending && !ss.has_ticket) ? PH_OTHER : PH_INIT);
+              : (serial_on && (ss.pending || ss.has_ticket)) ? PH_OTHER : PH_INIT);
         // TXBegin l.4-5: a fresh clock read, or the clock value right after
         // this warp's own last commit (p.snapshot_reuse)
         const uint32_t snap = (have_snap && p.snapshot_reuse) ? next_snap : warp_snapshot(m.clock);
