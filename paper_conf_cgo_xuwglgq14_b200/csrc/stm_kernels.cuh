@@ -210,10 +210,10 @@ __device__ __forceinline__ bool warp_late(uint32_t iter, unsigned long long dead
 // One 64-bit word in the metadata block, M_SERIAL = {serving:32 | next:32},
 // is a ticket queue.  A transaction that keeps aborting while the whole GPU
 // commits little (g_clock advanced by < serial_commits per abort of its
-// own) takes a ticket; while any ticket is outstanding (next != serving) no
-// other transaction STARTS an execution -- one that has aborted before joins
-// the queue instead, so a serial phase, once the contention test opened it,
-// serves every transaction that was failing -- and the holders run one at a time
+// own), and for which one-at-a-time measures faster (serial_gate), takes a
+// ticket; while any ticket is outstanding (next != serving) no other
+// transaction STARTS an execution -- one that has aborted before and passes
+// the same time test joins the queue instead -- and the holders run one at a time
 // in ticket order: the owner (ticket == serving) runs its transaction
 // irrevocably -- in place, under encounter-time locks, stamped while it holds
 // them all (gstm/tx_irr.cuh) -- and then serves the next ticket.  The
@@ -236,8 +236,8 @@ struct SerialState {
 // start an execution of its current transaction (stage 0).  Returns whether
 // it may.  The ticket word is read when this warp takes or holds a ticket,
 // after a poll that saw tickets outstanding, and every 8th iteration
-// otherwise (a stale "none outstanding" only lets an execution start that
-// the owner then waits to drain).
+// otherwise (a stale "none outstanding" only lets an execution start beside
+// the owner, where it meets the owner's words locked as during any commit).
 __device__ __forceinline__ bool serial_gate(const KParams& p, SerialState& ss, bool fresh, uint32_t snap,
                                             uint32_t iter)
 {
