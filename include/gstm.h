@@ -31,7 +31,8 @@
 extern "C" {
 #endif
 
-/* 2: gstm_params_t gained serial_after, serial_commits, lock_pipeline_gated and
+/* 2: gstm_params_t gained serial_after, serial_commits, lock_pipeline_gated,
+ *    pipeline_abort and
  *    gstm_stats_t gained serial_runs (appended; the structs are passed by
  *    pointer, so a client built against version 1 must be rebuilt) */
 #define GSTM_API_VERSION 2
@@ -182,6 +183,12 @@ typedef struct {
                              /*    touched nothing else) and then every other lock   */
                              /*    at once.  0: such logs take the  */
                              /*    sequential round.  Default 0 (KM: 1)              */
+    uint32_t pipeline_abort; /* 1: a pipelined lock round that finds a lock held    */
+                             /*    aborts the execution (re-executed with fresh     */
+                             /*    reads) instead of retrying sequential rounds;    */
+                             /*    after lock_pipeline such aborts the rounds are   */
+                             /*    sequential (progress as for any lock_pipeline,   */
+                             /*    DESIGN.md §6.4).  Default 0                      */
 } gstm_params_t;
 
 typedef struct {

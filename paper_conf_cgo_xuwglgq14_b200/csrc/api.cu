@@ -206,6 +206,7 @@ static gstm_params_t default_params(int workload)
     p.serial_after = 0;
     p.serial_commits = 4;
     p.lock_pipeline_gated = 0;
+    p.pipeline_abort = 0;
     // k-means: every contender of a record needs its lowest lock first; the
     // gated round holds the 17 locks for two round trips instead of 17
     // (26.5 -> 32.7 M tx/s; EB's random words lose with it)
@@ -708,6 +709,7 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.serial_after = P.serial_after;
     kp.serial_commits = P.serial_commits ? P.serial_commits : 4u;
     kp.lock_pipeline_gated = P.lock_pipeline_gated;
+    kp.pipeline_abort = P.pipeline_abort;
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));

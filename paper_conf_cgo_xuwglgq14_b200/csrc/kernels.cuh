@@ -74,6 +74,7 @@ struct KParams {
     uint32_t serial_after;         // contention manager: aborts before a transaction may take a serial ticket (0 = off)
     uint32_t serial_commits;       // ... only while the clock advanced by < serial_commits per abort
     uint32_t lock_pipeline_gated;  // pipelined rounds of longer local/shared logs: the lowest lock first, then the rest
+    uint32_t pipeline_abort;       // a failed pipelined round aborts the execution (re-execute, fresh reads)
 };
 
 cudaError_t launch_prepare(unsigned long long* meta, const unsigned long long* clock, uint64_t timeout_ns, cudaStream_t s);

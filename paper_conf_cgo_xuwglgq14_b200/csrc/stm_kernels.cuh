@@ -384,6 +384,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     int stage = 0;
     bool timed_out = false, have_snap = false;
     uint32_t lock_aborts = 0;   // lock aborts of the current transaction
+    uint32_t ab_exec = 0;       // aborted executions of the current transaction, any cause
     SerialState ss;             // contention manager (p.serial_after)
     const bool serial_on = SerialGate<WL>::value && p.serial_after != 0;
     // the serial owner's lock log: one slice per warp (one owner per warp at most)
@@ -511,6 +512,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     ++i;
                     backoff = 0;
                     lock_aborts = 0;
+                    ab_exec = 0;
                 }
             }
         }
@@ -531,7 +533,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
-            const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline;
+            // (with pipeline_abort the budget counts every aborted execution:
+            // a transaction that keeps failing for any reason is contended,
+            // and its rounds turn sequential after lock_pipeline of them)
+            const bool want_pipe = tries == 0 && (p.pipeline_abort ? ab_exec : lock_aborts) < p.lock_pipeline;
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks,
                                             p.lock_pipeline_gated != 0);
             if (tx.pipelined_round) cnt.inc(S_PIPELINED);
@@ -548,7 +553,13 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                 tries += (tries != ~0u) ? 1u : 0u;
                 if (POL == POL_BACKOFF) {
                     tries = 1;                                        // -> the sequential step below
-                } else if (p.k_lock && tries >= p.k_lock) {
+                } else if ((p.k_lock && tries >= p.k_lock) || (p.pipeline_abort && tx.pipelined_round)) {
+                    // (pipeline_abort: a lock another transaction holds in a
+                    // failed pipelined round is being committed, so this
+                    // execution's read of its word is stale -- re-execute now
+                    // instead of retrying sequential rounds toward a failing
+                    // VBV; after lock_pipeline such aborts the rounds are
+                    // sequential again, §6.4)
                     stage = 0;
                     aborted = true;
                     ++lock_aborts;
@@ -654,7 +665,11 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             ++i;
             backoff = 0;
             lock_aborts = 0;
-        } else if (p.backoff_ns && aborted) {
+            ab_exec = 0;
+        } else if (aborted) {
+            ++ab_exec;
+        }
+        if (!done && p.backoff_ns && aborted) {
             // exponential backoff after an abort (P:111 argues per-lane
             // delays cannot work under SIMT; lanes here sleep independently
             // under independent thread scheduling)

@@ -61,6 +61,7 @@ class gstm_params_t(C.Structure):
         ("km_assign", C.c_uint32), ("l2_persist_locks", C.c_uint32), ("ra_partition", C.c_uint32),
         ("body_rounds", C.c_uint32), ("pipeline_max_locks", C.c_uint32), ("lock_log_at_commit", C.c_uint32),
         ("serial_after", C.c_uint32), ("serial_commits", C.c_uint32), ("lock_pipeline_gated", C.c_uint32),
+        ("pipeline_abort", C.c_uint32),
     ]
 
 

@@ -53,3 +53,22 @@ def test_gated_round_progress_under_contention(k_lock):
     finally:
         g.close()
     assert st.pipelined_rounds > 0
+
+
+@pytest.mark.parametrize("wl,kw,T,K,bits", [("eb", dict(n_words=256, n_accesses=16), 1024, 4, 8),
+                                          ("ra", dict(n_reads=4, n_writes=4, n_words=64), 512, 8, 6),
+                                          ("bank", dict(n_words=256), 2048, 4, 8)])
+@pytest.mark.parametrize("k_lock", [0, 8])
+def test_pipeline_abort_replay(wl, kw, T, K, bits, k_lock):
+    """pipeline_abort: a failed pipelined round aborts the
+    execution; the pipelined budget then counts every aborted execution.
+    Replays bit-exactly and completes for k_lock 0 (infinite sequential
+    rounds after the budget) and 8."""
+    g, gp, op, init = U.make(wl, T, K, bits, mode="hv", lock_pipeline=4, pipeline_max_locks=16,
+                             pipeline_abort=1, k_lock=k_lock, timeout_ms=30000, **kw)
+    try:
+        st, _, _, _ = U.run_verified(g, wl, op, init, T, K, 29)
+    finally:
+        g.close()
+    assert st.pipelined_rounds > 0
+    assert st.pipelined_rounds <= st.attempts
