@@ -110,7 +110,7 @@ typedef struct {
                              /*    failed one, for any k_lock; progress is kept for    */
                              /*    any N).  0: always sequential.  Local-memory        */
                              /*    logs pipeline only logs of <= 8 locks.              */
-                             /*    Default 1 (RA, EB: 0)                               */
+                             /*    Default 1 (RA: 0; EB: 16)                           */
     uint32_t max_threads;    /* concurrency cap: at most this many CUDA threads run the */
                              /*    n_threads STM threads; 0 = the workload's default:  */
                              /*    what fits on the chip, at most 16 resident warps   */
@@ -151,7 +151,7 @@ typedef struct {
     uint32_t pipeline_max_locks; /* local-memory lock logs: the pipelined first round */
                              /*    (lock_pipeline) is used only for logs of at most  */
                              /*    this many locks (issued 8 atom.or at a time);     */
-                             /*    0 = 8.  Default 8                                 */
+                             /*    0 = 8.  Default 8 (EB: 16)                        */
     uint32_t lock_log_at_commit; /* 1: a read's lock enters the sorted lock log when   */
                              /*    the transaction reaches TXCommit with a write-set */
                              /*    instead of at the read (P:113's encounter time):  */
@@ -183,12 +183,15 @@ typedef struct {
                              /*    touched nothing else) and then every other lock   */
                              /*    at once.  0: such logs take the  */
                              /*    sequential round.  Default 0 (KM: 1)              */
-    uint32_t pipeline_abort; /* 1: a pipelined lock round that finds a lock held    */
-                             /*    aborts the execution (re-executed with fresh     */
-                             /*    reads) instead of retrying sequential rounds;    */
-                             /*    after lock_pipeline such aborts the rounds are   */
-                             /*    sequential (progress as for any lock_pipeline,   */
-                             /*    DESIGN.md §6.4).  Default 0                      */
+    uint32_t pipeline_abort; /* N > 0: a pipelined lock round that finds a lock     */
+                             /*    held aborts the execution (re-executed with fresh */
+                             /*    reads) instead of retrying sequential rounds, and */
+                             /*    a warp pipelines only while its recent abort rate */
+                             /*    (EMA x 256 over its lanes' executions) is below   */
+                             /*    N; lock_pipeline still bounds a transaction's     */
+                             /*    pipelined executions (progress).  */
+                             /*    Default 0 (EB: 100, with lock_pipeline 16 and     */
+                             /*    pipeline_max_locks 16)                            */
 } gstm_params_t;
 
 typedef struct {

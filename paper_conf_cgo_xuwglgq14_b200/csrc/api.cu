@@ -240,10 +240,20 @@ static gstm_params_t default_params(int workload)
         // launch, every other sweep point unchanged (no ticket taken)
         p.serial_after = 4;
     }
-    // RA and EB (random words, contended): the sequential first round is
-    // faster even when the lock log fits one pipelined chunk (EB A=8: 1.24
-    // vs 0.94 G tx/s; RA 8M words: 0.76 vs 0.53 G tx/s)
-    if (workload == GSTM_WL_EB || workload == GSTM_WL_RA) p.lock_pipeline = 0;
+    // RA (random words, contended): the sequential first round is faster
+    // even when the lock log fits one pipelined chunk (RA 8M words: 0.76 vs
+    // 0.53 G tx/s)
+    if (workload == GSTM_WL_RA) p.lock_pipeline = 0;
+    // EB: logs of up to 16 locks take one pipelined round while the warp's
+    // recent abort rate is below 100/256, and a failed pipelined round
+    // re-executes at once (pipeline_abort): hot set 2^26 A=16 681 -> 761,
+    // A=8 1535 -> 1729 M tx/s; the contended points run sequential rounds as
+    // before (hot set 2^18-2^22 within 4%, the 2^10 corners unchanged)
+    if (workload == GSTM_WL_EB) {
+        p.lock_pipeline = 16;
+        p.pipeline_max_locks = 16;
+        p.pipeline_abort = 100;
+    }
     return p;
 }
 

@@ -384,7 +384,7 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
     int stage = 0;
     bool timed_out = false, have_snap = false;
     uint32_t lock_aborts = 0;   // lock aborts of the current transaction
-    uint32_t ab_exec = 0;       // aborted executions of the current transaction, any cause
+    int32_t ab_warp = 0;        // pipeline_abort: the warp's recent abort rate, EMA x 256 (warp-uniform)
     SerialState ss;             // contention manager (p.serial_after)
     const bool serial_on = SerialGate<WL>::value && p.serial_after != 0;
     // the serial owner's lock log: one slice per warp (one owner per warp at most)
@@ -512,7 +512,6 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
                     ++i;
                     backoff = 0;
                     lock_aborts = 0;
-                    ab_exec = 0;
                 }
             }
         }
@@ -533,10 +532,12 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             // a round that follows a failed round is sequential, and among
             // sequential lanes the holder of the highest contended lock
             // always progresses (Q15, Q37).
-            // (with pipeline_abort the budget counts every aborted execution:
-            // a transaction that keeps failing for any reason is contended,
-            // and its rounds turn sequential after lock_pipeline of them)
-            const bool want_pipe = tries == 0 && (p.pipeline_abort ? ab_exec : lock_aborts) < p.lock_pipeline;
+            // (pipeline_abort: only while the WARP's recent executions rarely
+            // aborted -- a warp-uniform choice, so its lanes do not split
+            // between the two acquisition paths; under contention a pipelined
+            // round holds every lock of a doomed commit, §6.4)
+            const bool want_pipe = tries == 0 && lock_aborts < p.lock_pipeline &&
+                                   (!p.pipeline_abort || ab_warp < static_cast<int32_t>(p.pipeline_abort));
             const int r = tx.commit_acquire(m, MODE, p.prelock_vbv != 0, want_pipe, p.pipeline_max_locks,
                                             p.lock_pipeline_gated != 0);
             if (tx.pipelined_round) cnt.inc(S_PIPELINED);
@@ -665,9 +666,10 @@ __global__ void __launch_bounds__(256, WL::kMinBlocks) stm_kernel(const KParams 
             ++i;
             backoff = 0;
             lock_aborts = 0;
-            ab_exec = 0;
-        } else if (aborted) {
-            ++ab_exec;
+        }
+        if (p.pipeline_abort) {
+            const int na = __popc(__ballot_sync(FULL, aborted)), nc = __popc(__ballot_sync(FULL, done));
+            if (na + nc) ab_warp += (na * 256 / (na + nc) - ab_warp) / 8;
         }
         if (!done && p.backoff_ns && aborted) {
             // exponential backoff after an abort (P:111 argues per-lane

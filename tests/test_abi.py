@@ -72,6 +72,10 @@ def test_loads_and_host_only_calls(so):
     assert G.gstm_default_params("eb").serial_commits == 4
     # the gated pipelined lock round: k-means only
     assert [G.gstm_default_params(w).lock_pipeline_gated for w in ("ra", "bank", "ht", "eb", "km")] == [0, 0, 0, 0, 1]
+    # EB's adaptive pipelined round
+    e = G.gstm_default_params("eb")
+    assert (e.lock_pipeline, e.pipeline_max_locks, e.pipeline_abort) == (16, 16, 100)
+    assert [G.gstm_default_params(w).pipeline_abort for w in ("ra", "bank", "ht", "km")] == [0, 0, 0, 0]
     with pytest.raises(G.GstmError):
         G.gstm_default_params(9)
 
