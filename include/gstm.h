@@ -190,7 +190,10 @@ typedef struct {
                              /*    (EMA x 256 over its lanes' executions) is below   */
                              /*    N; lock_pipeline still bounds a transaction's     */
                              /*    pipelined executions (progress).  */
-                             /*    Default 0 (EB: 100, with lock_pipeline 16 and     */
+                             /*    Applied only where it pays: a shared footprint   */
+                             /*    larger than L2 and >= 1 lock per 4 words (else   */
+                             /*    the launch runs sequential rounds).  Default 0   */
+                             /*    (EB: 100, with lock_pipeline 16 and              */
                              /*    pipeline_max_locks 16)                            */
 } gstm_params_t;
 

@@ -115,6 +115,21 @@ static cudaError_t l2_limits(int dev, size_t* max_persist, size_t* max_window)
     return cudaSuccess;
 }
 
+// L2 size of a device (cached; the adaptive pipelined round's rule, launch)
+static uint64_t l2_cache_bytes(int dev)
+{
+    static std::mutex mu;
+    static uint64_t b[kMaxDevices];
+    if (dev < 0 || dev >= kMaxDevices) return 0;
+    std::lock_guard<std::mutex> g(mu);
+    if (!b[dev]) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrL2CacheSize, dev) != cudaSuccess) return 0;
+        b[dev] = static_cast<uint64_t>(v);
+    }
+    return b[dev];
+}
+
 // does the handle's lock table fit the persisting set-aside?  A larger table
 // would only shrink the L2 left for everything else (measured: EB with 2^26
 // locks, 256 MiB, 384 -> 146 M tx/s), so the knob then does nothing.
@@ -720,6 +735,20 @@ int gstm_launch(gstm_t* h, int workload, uint64_t n_threads, uint32_t tx_per_thr
     kp.serial_commits = P.serial_commits ? P.serial_commits : 4u;
     kp.lock_pipeline_gated = P.lock_pipeline_gated;
     kp.pipeline_abort = P.pipeline_abort;
+    if (P.pipeline_abort) {
+        // the adaptive pipelined round pays where sequential rounds are slow
+        // and false conflicts rare: a shared footprint larger than L2 (every
+        // commit's VBV and write-back go to HBM) and at least one version lock
+        // per 4 words; elsewhere (L2-resident hot sets, few locks) the rounds
+        // stay sequential (EB hot set 2^26 with 2^24 locks
+        // +11%, with 2^20-2^22 locks -6..-32% if it were on)
+        const uint64_t l2 = l2_cache_bytes(h->dev);
+        const bool pays = l2 && fp * 4 > l2 && (1ull << h->bits) * 4 >= fp;
+        if (!pays) {
+            kp.lock_pipeline = 0;
+            kp.pipeline_abort = 0;
+        }
+    }
     const uint64_t timeout_ns = static_cast<uint64_t>(P.timeout_ms ? P.timeout_ms : 60000) * 1000000ull;
     CUDA_TRY(cudaEventRecord(h->ev0, h->stream));
     CUDA_TRY(launch_prepare(h->meta, h->clock, timeout_ns, h->stream));

@@ -10,7 +10,7 @@ import gpu_util as U
 
 pytestmark = pytest.mark.gpu
 
-GATED = dict(lock_pipeline=1000, lock_pipeline_gated=1)
+GATED = dict(lock_pipeline=1000, lock_pipeline_gated=1, pipeline_abort=0)
 
 # (workload, params, T, K, lock bits): lock logs of 9-32 entries
 CASES = [
@@ -55,20 +55,34 @@ def test_gated_round_progress_under_contention(k_lock):
     assert st.pipelined_rounds > 0
 
 
-@pytest.mark.parametrize("wl,kw,T,K,bits", [("eb", dict(n_words=256, n_accesses=16), 1024, 4, 8),
-                                          ("ra", dict(n_reads=4, n_writes=4, n_words=64), 512, 8, 6),
-                                          ("bank", dict(n_words=256), 2048, 4, 8)])
+@pytest.mark.parametrize("paired", [False, True])
 @pytest.mark.parametrize("k_lock", [0, 8])
-def test_pipeline_abort_replay(wl, kw, T, K, bits, k_lock):
-    """pipeline_abort: a failed pipelined round aborts the
-    execution; the pipelined budget then counts every aborted execution.
-    Replays bit-exactly and completes for k_lock 0 (infinite sequential
-    rounds after the budget) and 8."""
-    g, gp, op, init = U.make(wl, T, K, bits, mode="hv", lock_pipeline=4, pipeline_max_locks=16,
-                             pipeline_abort=1, k_lock=k_lock, timeout_ms=30000, **kw)
+def test_pipeline_abort_replay(paired, k_lock):
+    """EB's adaptive pipelined round (pipeline_abort): a
+    failed pipelined round aborts the execution, a warp pipelines only while
+    its recent abort rate is low.  It applies where the footprint exceeds L2
+    and there is a lock per <= 4 words: a 2^25-word hot set with 2^23 locks
+    (2^25 paired).  Replays bit-exactly and completes for k_lock 0 and 8."""
+    T, K, words = 8192, 4, 1 << 25
+    bits = 25 if paired else 23
+    g, gp, op, init = U.make("eb", T, K, bits, mode="hv", paired=paired, n_words=words, n_accesses=16,
+                             k_lock=k_lock, timeout_ms=30000)
+    assert gp.pipeline_abort and gp.lock_pipeline and gp.pipeline_max_locks >= 16   # EB's defaults
     try:
-        st, _, _, _ = U.run_verified(g, wl, op, init, T, K, 29)
+        st, _, _, _ = U.run_verified(g, "eb", op, init, T, K, 29)
     finally:
         g.close()
     assert st.pipelined_rounds > 0
     assert st.pipelined_rounds <= st.attempts
+
+
+def test_pipeline_abort_stays_off_where_it_does_not_pay():
+    """An L2-resident hot set keeps the sequential rounds (no pipelined
+    round at all) although pipeline_abort is on."""
+    T, K = 2048, 4
+    g, gp, op, init = U.make("eb", T, K, 12, mode="hv", n_words=4096, n_accesses=16)
+    try:
+        st, _, _, _ = U.run_verified(g, "eb", op, init, T, K, 31)
+    finally:
+        g.close()
+    assert st.pipelined_rounds == 0
