@@ -192,7 +192,9 @@ typedef struct {
                              /*    pipelined executions (progress).  */
                              /*    Applied only where it pays: a shared footprint   */
                              /*    larger than L2 and >= 1 lock per 4 words (else   */
-                             /*    the launch runs sequential rounds).  Default 0   */
+                             /*    the launch runs sequential rounds); there the    */
+                             /*    launch also skips the optional pre-lock VBV      */
+                             /*    (A3.l71).  Default 0                             */
                              /*    (EB: 100, with lock_pipeline 16 and              */
                              /*    pipeline_max_locks 16)                            */
 } gstm_params_t;
