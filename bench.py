@@ -498,17 +498,35 @@ def sig(x: float, n: int = 4) -> float:
     return float(f"{x:.{n}g}")
 
 
-def first_round_pipelined(wl, gp, st):
+def fp_words(wl, heap_words, kw, T, K) -> int:
+    """The workload footprint api.cu's rules use (words the transactions
+    address): EB/RA/bank n_words; HT/KM the heap they are sized to."""
+    return int(kw.get("n_words", heap_words)) if wl in ("eb", "ra", "bank") else int(heap_words)
+
+
+def adaptive_pipelining_applies(gp, words, bits) -> bool:
+    """api.cu's rule for pipeline_abort: the launch keeps
+    it (and then skips the pre-lock VBV) only for a shared footprint larger
+    than L2 with at least one version lock per 4 words."""
+    import torch
+    l2 = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+    return bool(gp.pipeline_abort) and words * 4 > l2 and (1 << bits) * 4 >= words
+
+
+def first_round_pipelined(wl, gp, st, words=0, bits=0):
     """Does the kernel issue a transaction's first lock round all at once
     ?  Register logs (bank) always may; local-memory logs only
-    when the lock log fits one 8-atomic chunk (Q36) -- longer ones take the
-    gated round ("gated": the lowest lock, then the rest) with
-    lock_pipeline_gated, else the sequential one."""
+    when the lock log fits pipeline_max_locks (Q36; 8 by default, EB's 16
+    where its adaptive round applies) -- longer ones take the gated round
+    ("gated": the lowest lock, then the rest) with lock_pipeline_gated, else
+    the sequential one."""
     if gp.lock_pipeline == 0:
+        return False
+    if gp.pipeline_abort and not adaptive_pipelining_applies(gp, words, bits):
         return False
     if wl == "bank":
         return True
-    if st.commits > 0 and st.locks_update / st.commits <= 8:
+    if st.commits > 0 and st.locks_update / st.commits <= (gp.pipeline_max_locks or 8):
         return True
     return "gated" if gp.lock_pipeline_gated else False
 
@@ -570,7 +588,9 @@ def run_config(G, R, stream, flush, name, seed):
         out["stm_hv_no_cm"] = sig(res["hv_no_cm"][0])
         out["serial_runs_hv"] = int(st.serial_runs)
     records = (1024, kw.get("km_stride", 17)) if wl == "km" else None
-    roof = op_mix_roof(G, R, stream, wl, st, "hv", bool(gp.prelock_vbv), first_round_pipelined(wl, gp, st),
+    prelock = bool(gp.prelock_vbv) and not adaptive_pipelining_applies(gp, fp_words(wl, words, kw, T, K), bits)
+    roof = op_mix_roof(G, R, stream, wl, st, "hv", prelock,
+                       first_round_pipelined(wl, gp, st, fp_words(wl, words, kw, T, K), bits),
                        words, bits, False, T, records=records)
     per_tx = roof["ops_per_tx"]
     sectors = per_tx["ld"] + per_tx["atom"] + per_tx["st"]
