@@ -22,8 +22,10 @@
 // lock, as A3.l68 places a read-only transaction at its snapshot), and the
 // transactions running beside it see its words locked, as during any commit
 // (A3.l27-29: they spin, then validate or abort).  It never aborts: the
-// locks it holds only grow.  The lock log (l_ent: id<<2 | wr<<1 | 1, l_old:
-// the word before locking) is in encounter order.
+// locks it holds only grow.  Its lock log (ent: id<<2 | wr<<1 | 1, old: the
+// word before locking) is in encounter order; one atomic per distinct lock,
+// batched 8 at a time where the body reads or declares (will_write) several
+// words at once.
 #pragma once
 #include "tx.cuh"
 
