@@ -75,3 +75,17 @@ def test_serial_not_compiled_for_bank_ht(wl, kw, bits):
     finally:
         g.close()
     assert st.serial_runs == 0
+
+
+def test_eb_default_manager_idle_at_low_contention():
+    """EB enables the contention manager by default (serial_after 4); at low
+    contention no transaction qualifies (the GPU commits far more than
+    serial_commits per abort), so no ticket is ever taken."""
+    T, K = 8192, 4
+    g, gp, op, init = U.make("eb", T, K, 20, mode="hv", heap_words=1 << 20, n_words=1 << 20, n_accesses=32)
+    assert gp.serial_after == 4
+    try:
+        st, _, _, _ = U.run_verified(g, "eb", op, init, T, K, 41)
+    finally:
+        g.close()
+    assert st.serial_runs == 0, st.as_dict()
