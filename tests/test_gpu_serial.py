@@ -89,3 +89,16 @@ def test_eb_default_manager_idle_at_low_contention():
     finally:
         g.close()
     assert st.serial_runs == 0, st.as_dict()
+
+
+@pytest.mark.parametrize("flavour", ["strict", "phase", "hlog", "smem"])
+def test_serial_tickets_in_build_flavours(flavour):
+    """The serial owner path replays in every build flavour (strict PTX
+    fences, Figure-5 phase timing, hashed and shared-memory lock logs)."""
+    T, K = 1024, 4
+    g, gp, op, init = U.make("eb", T, K, 10, mode="hv", flavour=flavour, n_words=1024, n_accesses=64, **FORCE)
+    try:
+        st, _, _, _ = U.run_verified(g, "eb", op, init, T, K, 43)
+    finally:
+        g.close()
+    assert st.serial_runs > 0
