@@ -61,10 +61,10 @@ def test_pipeline_abort_replay(paired, k_lock):
     """EB's adaptive pipelined round (pipeline_abort): a
     failed pipelined round aborts the execution, a warp pipelines only while
     its recent abort rate is low.  It applies where the footprint exceeds L2
-    and there is a lock per <= 4 words: a 2^25-word hot set with 2^23 locks
-    (2^25 paired).  Replays bit-exactly and completes for k_lock 0 and 8."""
-    T, K, words = 8192, 4, 1 << 25
-    bits = 25 if paired else 23
+    and there is a lock per <= 4 words: a 3 x 2^24-word hot set with 2^24
+    locks (2^26 paired).  Replays bit-exactly and completes for k_lock 0 and 8."""
+    T, K, words = 8192, 4, 3 << 24          # 192 MiB: clearly larger than the B200's L2
+    bits = 26 if paired else 24
     g, gp, op, init = U.make("eb", T, K, bits, mode="hv", paired=paired, n_words=words, n_accesses=16,
                              k_lock=k_lock, timeout_ms=30000)
     assert gp.pipeline_abort and gp.lock_pipeline and gp.pipeline_max_locks >= 16   # EB's defaults
